@@ -1,0 +1,227 @@
+/*
+ * xs.h — C-ABI of libxs.so, the B200-native XSBench event-based macroscopic
+ * neutron cross-section (XS) lookup (the data-parallel hot path of Tian et
+ * al., "OpenMP Kernel Language Extensions for Performance Portable GPU
+ * Codes", SC-W 2023: XSBench "-m event"; "computing the
+ * continuous energy macroscopic neutron cross-section lookup",
+ * PAPER.md:911-915; self-verified by a checksum).
+ *
+ * One lookup (BASELINE.json north_star; DESIGN.md §1 and readings R1-R17):
+ *   A1  sample energy p and material m from a counter-based LCG stream
+ *   A2  (optional) sort the batch by (material, energy) — XS_FLAG_SORT
+ *   A3  find p on the unionized energy grid (binary search) or hash grid
+ *   A4  gather the bracket index k_n of every nuclide n in material m
+ *   A5  gather the record pair (k_n, k_n+1) of each nuclide
+ *   A6  interpolate the five channels (total, elastic, absorption, fission,
+ *       nu-fission) linearly in energy
+ *   A7  accumulate M_c += x_c * conc_j over the material's nuclides
+ *   A8  verification value v = 1 + argmax_c M_c; vsum += {v, 1}
+ *   A9  (caller) all-reduce vsum across ranks; hash = sum mod 999983
+ *
+ * Conventions (all entry points):
+ *   - extern "C", plain pointers and sizes; no C++ types cross the ABI.
+ *   - Every call returns xs_status; on failure xs_last_error() returns a
+ *     thread-local message.  No exceptions, no abort().
+ *   - "device pointer" = memory on the grid's device (e.g. a torch tensor's
+ *     data_ptr()); the caller owns it and must keep it alive until the work
+ *     enqueued on `cuda_stream` completes.  `cuda_stream` is a cudaStream_t
+ *     (NULL = legacy default stream), e.g. torch.cuda.current_stream().
+ *   - Work is enqueued asynchronously on the stream; device faults surface
+ *     as XS_ERR_CUDA at the next call that synchronizes.
+ *   - Results depend only on (grid, global lookup id), never on batching,
+ *     sharding, sorting or launch configuration (shard = [first, first+count)).
+ *   - The library owns the grid tables (freed by xs_free_grid).  One grid
+ *     lives on one device; calls on one grid are ordered by the caller.
+ *   - There is no CPU fallback: without a usable sm_100 device every
+ *     compute entry point fails with XS_ERR_CUDA / XS_ERR_UNSUPPORTED.
+ */
+#ifndef XS_H
+#define XS_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define XS_ABI_VERSION 1u
+
+typedef enum {
+  XS_OK = 0,
+  XS_ERR_INVALID_ARG = 1,   /* NULL/inconsistent argument, bad spec, range error */
+  XS_ERR_OUT_OF_MEMORY = 2, /* device or host allocation failed                 */
+  XS_ERR_CUDA = 3,          /* CUDA runtime/launch error (message has details)  */
+  XS_ERR_UNSUPPORTED = 4,   /* feature not available for this grid/device       */
+  XS_ERR_STATE = 5,         /* call made in the wrong state (e.g. wrong device) */
+  XS_ERR_DATA = 6           /* input data invalid (e.g. duplicate energies)     */
+} xs_status;
+
+/* Energy-search acceleration (north_star: "binary-searches the unionized (or
+ * hash-accelerated) energy grid"; R6-R9). */
+typedef enum {
+  XS_GRID_UNIONIZED = 0, /* U = sorted union of all energies + index grid IG[NU][I] */
+  XS_GRID_NUCLIDE = 1,   /* no acceleration: binary search per nuclide            */
+  XS_GRID_HASH = 2       /* hash grid HG[B][I] over equal-width energy bins        */
+} xs_grid_type;
+
+/* Synthetic XSBench problem, regenerated from seeds by the shared input
+ * generator (gen/xs_gen.h; R1).  Presets: tiny (12, 1000, rule 1),
+ * small (68, 11303), large (355, 11303), XL (355, 238847); grid_seed 42,
+ * conc_seed 1070^2, lookup_seed 1070. */
+typedef struct {
+  uint32_t abi_version;   /* = XS_ABI_VERSION                                   */
+  int32_t n_isotopes;     /* I >= 1 (rule 0 requires 68 or 355)                */
+  int64_t n_gridpoints;   /* N >= 2 points per nuclide                          */
+  int32_t grid_type;      /* xs_grid_type                                       */
+  int32_t hash_bins;      /* B >= 1, used iff grid_type == XS_GRID_HASH         */
+  uint64_t grid_seed;     /* nuclide grid draws                                 */
+  uint64_t conc_seed;     /* concentration draws                                */
+  uint64_t lookup_seed;   /* lookup stream seed (A1)                            */
+  int32_t material_rule;  /* 0 = XSBench H-M tables, 1 = ids mod I (tiny)       */
+  int32_t reserved0;      /* must be 0                                          */
+} xs_grid_spec;
+
+/* Caller-supplied nuclear data (HOST pointers, copied during init).  The
+ * nuclide grid is [I][N][6] doubles (E, total, elastic, absorption, fission,
+ * nu-fission) with E strictly increasing per nuclide; mats/concs are
+ * [n_mats][max_num_nucs] row-major, only the first num_nucs[m] entries of
+ * row m are read.  Sampled batches (xs_lookup_batch) need n_mats == 12 (the
+ * XSBench material distribution); explicit lookups accept any n_mats >= 1. */
+typedef struct {
+  uint32_t abi_version;
+  int32_t n_isotopes;
+  int64_t n_gridpoints;
+  const double* nuclide_grid;
+  int32_t n_mats;
+  int32_t max_num_nucs;
+  const int32_t* num_nucs;
+  const int32_t* mats;
+  const double* concs;
+  int32_t grid_type;
+  int32_t hash_bins;
+  uint64_t lookup_seed;
+} xs_grid_data;
+
+typedef struct xs_grid xs_grid; /* opaque: one replica of the tables on one device */
+
+typedef struct {
+  int32_t n_isotopes, n_mats, max_num_nucs, grid_type, hash_bins, device;
+  int64_t n_gridpoints;
+  int64_t n_union;        /* NU = I*N for UNIONIZED, else 0                     */
+  int64_t index_grid_len; /* NU*I (UNIONIZED), B*I (HASH), 0 (NUCLIDE)          */
+  uint64_t device_bytes;  /* bytes of device memory the grid holds              */
+  uint64_t lookup_seed;
+} xs_grid_info;
+
+/* Per-lookup outputs, indexed by position i in the batch (lookup id
+ * first_id + i).  Every pointer may be NULL except vsum.  DEVICE pointers
+ * unless XS_FLAG_HOST_IO is set, in which case they are HOST pointers
+ * (pageable or pinned) and the library stages them through the workspace. */
+typedef struct {
+  double* macro_xs;      /* [count][5]  M_c, channel order as above          */
+  double* energy;        /* [count]     sampled p                            */
+  int32_t* mat;          /* [count]     sampled material                     */
+  int64_t* grid_index;   /* [count]     u (UNIONIZED), b (HASH), -1 (NUCLIDE) */
+  int32_t* verification; /* [count]     v in 1..5 (0 for an invalid lookup)   */
+  uint64_t* vsum;        /* [2]         ACCUMULATED: += {sum v, #valid}       */
+} xs_outputs;
+
+/* flags */
+#define XS_FLAG_SORT 0x1u     /* A2: radix-sort the batch by (material, energy)  */
+#define XS_FLAG_HOST_IO 0x2u  /* inputs/outputs are host pointers               */
+#define XS_FLAG_BASELINE 0x4u /* thread-per-lookup, unbucketed kernel (XSBench's
+                                 CUDA baseline shape; for comparison only)     */
+
+/* tables for xs_get_table (element type in brackets) */
+#define XS_TABLE_NUCLIDE_GRID 0 /* [double] I*N*6                               */
+#define XS_TABLE_UNION_ENERGY 1 /* [double] NU                                  */
+#define XS_TABLE_INDEX_GRID 2   /* [int32]  IG (NU*I) or HG (B*I), row-major     */
+#define XS_TABLE_NUM_NUCS 3     /* [int32]  n_mats                              */
+#define XS_TABLE_MATS 4         /* [int32]  n_mats*max_num_nucs                 */
+#define XS_TABLE_CONCS 5        /* [double] n_mats*max_num_nucs                 */
+
+uint32_t xs_abi_version(void);
+
+/* Generate the problem from `spec` on the host (gen/xs_gen.h), upload it to
+ * `device` and build the acceleration tables there (unionized energy sort,
+ * index grid or hash grid).  Synchronizes `cuda_stream` before returning.
+ * Errors: INVALID_ARG (bad spec), DATA (duplicate energy in a nuclide),
+ * OUT_OF_MEMORY, CUDA.  On success *out owns all device tables. */
+xs_status xs_init_grid(const xs_grid_spec* spec, int device, void* cuda_stream, xs_grid** out);
+
+/* Same with caller-supplied nuclear data (host arrays, copied). */
+xs_status xs_init_grid_data(const xs_grid_data* data, int device, void* cuda_stream,
+                            xs_grid** out);
+
+xs_status xs_grid_get_info(const xs_grid* g, xs_grid_info* info);
+
+/* Bytes of device workspace xs_lookup_batch / xs_lookup_explicit need for a
+ * batch of `count` lookups with `flags`.  Workspace must be 256-B aligned. */
+xs_status xs_workspace_size(const xs_grid* g, uint64_t count, uint32_t flags, size_t* bytes);
+
+/* A1-A8 for lookup ids [first_id, first_id + count), enqueued on the stream.
+ * 0 <= count < 2^32.  vsum is accumulated (+=), so shards can share it.
+ * Requires n_mats == 12 (sampling distribution).  count == 0 is a no-op. */
+xs_status xs_lookup_batch(xs_grid* g, uint64_t first_id, uint64_t count, uint32_t flags,
+                          const xs_outputs* out, void* workspace, size_t workspace_bytes,
+                          void* cuda_stream);
+
+/* A2-A8 for caller-given lookups: energy[i] (any double; outside the grid the
+ * XS are extrapolated) and mat[i] (0 <= mat < n_mats; an out-of-range mat
+ * gives v = 0, NaN macro_xs and is not counted in vsum[1]).  energy/mat are
+ * device pointers, or host pointers with XS_FLAG_HOST_IO (then the outputs
+ * are host pointers too and the call synchronizes the stream on return). */
+xs_status xs_lookup_explicit(xs_grid* g, const double* energy, const int32_t* mat,
+                             uint64_t count, uint32_t flags, const xs_outputs* out,
+                             void* workspace, size_t workspace_bytes, void* cuda_stream);
+
+/* A8 alone on stored results: vsum += {sum_i (1 + argmax_c macro_xs[i][c]), count}
+ * (device pointers). */
+xs_status xs_verify(const xs_grid* g, const double* macro_xs, uint64_t count, uint64_t* vsum,
+                    void* cuda_stream);
+
+/* Diagnostic for A3/A4 parity: k_out[i] = bracket of nuclide nuclide[i] at
+ * energy[i] found through the grid's own acceleration structure (device
+ * pointers; 0 <= nuclide < I). */
+xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t* nuclide,
+                           uint64_t count, int32_t* k_out, void* cuda_stream);
+
+/* Synchronous copy of elements [offset, offset+count) of a device table to
+ * host memory (parity checks of the device-built tables). */
+xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
+                       void* host_dst);
+
+/* Tuning knobs: "unroll" (nuclides per round per lookup group: 3, 6 or 9)
+ * and "blocks_per_sm" (0 = occupancy calculator).  INVALID_ARG for an
+ * unknown name or value.  Never changes results. */
+xs_status xs_set_param(xs_grid* g, const char* name, int64_t value);
+
+/* Per-phase device timing of lookup calls, measured with CUDA events
+ * recorded on the caller's stream around each phase (enable costs four
+ * event records per call).  kernel_launches counts the library's own kernel
+ * launches (always on). */
+typedef struct {
+  uint64_t calls;           /* lookup calls since the last read              */
+  uint64_t kernel_launches; /* kernels those calls launched                  */
+  double ms_prepare;        /* A1+A3: material count, sample+search, bucket  */
+  double ms_sort;           /* A2: radix sort (0 without XS_FLAG_SORT)       */
+  double ms_gather;         /* A4-A8: the gather/interpolate/verify kernel   */
+  double ms_total;          /* sum of the above                              */
+} xs_timing;
+
+xs_status xs_timing_enable(xs_grid* g, int enable);
+/* Waits for the recorded events, returns the sums since the previous read
+ * (or enable) and resets them. */
+xs_status xs_timing_read(xs_grid* g, xs_timing* out);
+
+/* A9 epilogue: hash = global sum mod 999983 (R13). */
+uint64_t xs_hash_finalize(uint64_t global_sum);
+
+void xs_free_grid(xs_grid* g);
+
+const char* xs_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,306 @@
+"""CPU ORACLE for the XSBench event-based macroscopic XS lookup.
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and
+``bench.py``'s ``cpu_baseline`` / ``--impl reference`` leg may import this
+package.  The product path (``paper_conf_sc_tianscd23_b200``) never imports
+it and shares no code with it; the single shared module is the seeded input
+generator ``gen/xs_gen.h`` (inputs only, none of the method's arithmetic).
+
+This is a thin ctypes binding over ``oracle/xs_oracle.c`` (plain serial C,
+fp64, ``-O2 -ffp-contract=off``); every step it exposes cites its reading in
+DESIGN.md and is pinned by ``tests/test_oracle_*.py``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_ROOT = os.path.dirname(_HERE)
+LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_SOURCES = [os.path.join(_HERE, "xs_oracle.c"), os.path.join(_HERE, "xs_oracle.h"),
+            os.path.join(_ROOT, "gen", "xs_gen.cpp"), os.path.join(_ROOT, "gen", "xs_gen.h")]
+
+UNIONIZED, NUCLIDE, HASH = 0, 1, 2
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so (C oracle + the shared input generator)."""
+    stale = force or not os.path.exists(LIB_PATH) or any(
+        os.path.getmtime(s) > os.path.getmtime(LIB_PATH) for s in _SOURCES)
+    if not stale:
+        return LIB_PATH
+    tmp_o = LIB_PATH + ".oracle.o"
+    tmp_g = LIB_PATH + ".gen.o"
+    flags = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC"]
+    subprocess.check_call(["gcc", *flags, "-std=c11", "-c", _SOURCES[0], "-o", tmp_o])
+    subprocess.check_call(["g++", *flags, "-std=c++17", "-c", _SOURCES[2], "-o", tmp_g])
+    subprocess.check_call(["g++", "-shared", "-o", LIB_PATH + ".tmp", tmp_o, tmp_g, "-lpthread"])
+    os.replace(LIB_PATH + ".tmp", LIB_PATH)
+    for f in (tmp_o, tmp_g):
+        os.remove(f)
+    return LIB_PATH
+
+
+def lib() -> C.CDLL:
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            L = C.CDLL(LIB_PATH)
+            u64, i64, i32, d = C.c_uint64, C.c_int64, C.c_int32, C.c_double
+            P = C.c_void_p
+            sig = {
+                "oracle_lcg_step": (u64, [u64]),
+                "oracle_lcg_to_double": (d, [u64]),
+                "oracle_fast_forward": (u64, [u64, u64]),
+                "oracle_thresholds": (None, [P]),
+                "oracle_pick_mat": (i32, [d]),
+                "oracle_sample": (None, [u64, u64, P, P]),
+                "oracle_grid_search": (i64, [P, i64, i64, d]),
+                "oracle_upper_bound": (i64, [P, i64, d]),
+                "oracle_create_spec": (P, [i32, i64, u64, u64, i32, u64, i32, C.c_int, P]),
+                "oracle_create_arrays": (P, [i32, i64, P, i32, i32, P, P, P, u64, i32, P]),
+                "oracle_free": (None, [P]),
+                "oracle_n_isotopes": (i32, [P]),
+                "oracle_n_gridpoints": (i64, [P]),
+                "oracle_n_mats": (i32, [P]),
+                "oracle_max_num_nucs": (i32, [P]),
+                "oracle_union_len": (i64, [P]),
+                "oracle_grid": (P, [P]),
+                "oracle_union": (P, [P]),
+                "oracle_num_nucs": (P, [P]),
+                "oracle_mats": (P, [P]),
+                "oracle_concs": (P, [P]),
+                "oracle_nuclide_bracket": (i64, [P, i32, d]),
+                "oracle_union_index": (i64, [P, d]),
+                "oracle_index_grid_entry": (i32, [P, i64, i32]),
+                "oracle_index_grid_sweep": (C.c_int, [P, P]),
+                "oracle_hash_bin": (i64, [P, d]),
+                "oracle_hash_entry": (i32, [P, i64, i32]),
+                "oracle_hash_bracket": (i64, [P, i64, i32, d]),
+                "oracle_micro_xs": (None, [P, i32, i64, d, P]),
+                "oracle_macro_xs": (None, [P, d, i32, C.c_int, P, P]),
+                "oracle_verify": (C.c_int, [P]),
+                "oracle_lookup": (None, [P, u64, C.c_int, P, P, P, P, P]),
+                "oracle_run": (u64, [P, u64, u64, C.c_int, C.c_int, P, P, P, P, P]),
+                "oracle_run_explicit": (u64, [P, P, P, u64, C.c_int, C.c_int, P, P]),
+                "oracle_hash_finalize": (u64, [u64]),
+                "xsgen_num_nucs": (C.c_int, [i32, i32, P]),
+                "xsgen_max_num_nucs": (i32, [i32, i32]),
+                "xsgen_mats": (C.c_int, [i32, i32, i32, P]),
+                "xsgen_concs": (C.c_int, [u64, P, i32, P]),
+                "xsgen_nuclide_grid": (C.c_int, [i32, i64, u64, P, C.c_int]),
+            }
+            for name, (res, args) in sig.items():
+                f = getattr(L, name)
+                f.restype = res
+                f.argtypes = args
+            _lib = L
+    return _lib
+
+
+def _ptr(a: np.ndarray | None):
+    return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+# ------------------------------------------------------------- free helpers
+def lcg_step(s: int) -> int:
+    return lib().oracle_lcg_step(s)
+
+
+def lcg_to_double(s: int) -> float:
+    return lib().oracle_lcg_to_double(s)
+
+
+def fast_forward(s: int, n: int) -> int:
+    return lib().oracle_fast_forward(s, n)
+
+
+def thresholds() -> np.ndarray:
+    T = np.zeros(12, np.float64)
+    lib().oracle_thresholds(_ptr(T))
+    return T
+
+
+def pick_mat(roll: float) -> int:
+    return lib().oracle_pick_mat(roll)
+
+
+def sample(lookup_seed: int, i: int) -> tuple[float, int]:
+    p, m = C.c_double(), C.c_int32()
+    lib().oracle_sample(lookup_seed, i, C.byref(p), C.byref(m))
+    return p.value, m.value
+
+
+def grid_search(A: np.ndarray, lo: int, hi: int, q: float) -> int:
+    A = np.ascontiguousarray(A, np.float64)
+    return lib().oracle_grid_search(_ptr(A), lo, hi, q)
+
+
+def upper_bound(A: np.ndarray, q: float) -> int:
+    A = np.ascontiguousarray(A, np.float64)
+    return lib().oracle_upper_bound(_ptr(A), len(A), q)
+
+
+def verify(M) -> int:
+    M = np.ascontiguousarray(M, np.float64)
+    return lib().oracle_verify(_ptr(M))
+
+
+def hash_finalize(S: int) -> int:
+    return lib().oracle_hash_finalize(S)
+
+
+# ------------------------------------------------------------- generator view
+def gen_num_nucs(I: int, rule: int) -> np.ndarray:
+    out = np.zeros(12, np.int32)
+    if lib().xsgen_num_nucs(I, rule, _ptr(out)):
+        raise ValueError("bad (I, rule)")
+    return out
+
+
+# ------------------------------------------------------------------ context
+class Oracle:
+    """An oracle context: problem data + the oracle's own U / HG tables."""
+
+    def __init__(self, handle):
+        self._h = handle
+        L = lib()
+        self.I = L.oracle_n_isotopes(handle)
+        self.N = L.oracle_n_gridpoints(handle)
+        self.n_mats = L.oracle_n_mats(handle)
+        self.max_num_nucs = L.oracle_max_num_nucs(handle)
+        self.NU = L.oracle_union_len(handle)
+
+    @classmethod
+    def from_spec(cls, n_isotopes, n_gridpoints, grid_seed=42, conc_seed=0, material_rule=0,
+                  lookup_seed=1070, hash_bins=0, nthreads=0):
+        err = C.c_int(0)
+        h = lib().oracle_create_spec(n_isotopes, n_gridpoints, grid_seed, conc_seed,
+                                     material_rule, lookup_seed, hash_bins, nthreads,
+                                     C.byref(err))
+        if not h:
+            raise ValueError(f"oracle_create_spec failed (err {err.value})")
+        return cls(h)
+
+    @classmethod
+    def from_arrays(cls, grid, num_nucs, mats, concs, lookup_seed=1070, hash_bins=0):
+        grid = np.ascontiguousarray(grid, np.float64)
+        I, N, six = grid.shape
+        assert six == 6
+        num_nucs = np.ascontiguousarray(num_nucs, np.int32)
+        mats = np.ascontiguousarray(mats, np.int32)
+        concs = np.ascontiguousarray(concs, np.float64)
+        n_mats, mx = mats.shape
+        err = C.c_int(0)
+        h = lib().oracle_create_arrays(I, N, _ptr(grid), n_mats, mx, _ptr(num_nucs), _ptr(mats),
+                                       _ptr(concs), lookup_seed, hash_bins, C.byref(err))
+        if not h:
+            raise ValueError(f"oracle_create_arrays failed (err {err.value})")
+        return cls(h)
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and lib is not None:
+            try:
+                lib().oracle_free(h)
+            except Exception:
+                pass
+
+    # views (copies) of the tables
+    def grid(self) -> np.ndarray:
+        a = np.ctypeslib.as_array(C.cast(lib().oracle_grid(self._h), C.POINTER(C.c_double)),
+                                  shape=(self.I * self.N * 6,))
+        return a.reshape(self.I, self.N, 6).copy()
+
+    def union(self) -> np.ndarray:
+        a = np.ctypeslib.as_array(C.cast(lib().oracle_union(self._h), C.POINTER(C.c_double)),
+                                  shape=(self.NU,))
+        return a.copy()
+
+    def num_nucs(self) -> np.ndarray:
+        return np.ctypeslib.as_array(C.cast(lib().oracle_num_nucs(self._h), C.POINTER(C.c_int32)),
+                                     shape=(self.n_mats,)).copy()
+
+    def mats(self) -> np.ndarray:
+        return np.ctypeslib.as_array(C.cast(lib().oracle_mats(self._h), C.POINTER(C.c_int32)),
+                                     shape=(self.n_mats, self.max_num_nucs)).copy()
+
+    def concs(self) -> np.ndarray:
+        return np.ctypeslib.as_array(C.cast(lib().oracle_concs(self._h), C.POINTER(C.c_double)),
+                                     shape=(self.n_mats, self.max_num_nucs)).copy()
+
+    # steps
+    def nuclide_bracket(self, n: int, p: float) -> int:
+        return lib().oracle_nuclide_bracket(self._h, n, p)
+
+    def union_index(self, p: float) -> int:
+        return lib().oracle_union_index(self._h, p)
+
+    def index_grid_entry(self, e: int, n: int) -> int:
+        return lib().oracle_index_grid_entry(self._h, e, n)
+
+    def index_grid_sweep(self) -> np.ndarray:
+        out = np.empty((self.NU, self.I), np.int32)
+        if lib().oracle_index_grid_sweep(self._h, _ptr(out)):
+            raise MemoryError
+        return out
+
+    def hash_bin(self, p: float) -> int:
+        return lib().oracle_hash_bin(self._h, p)
+
+    def hash_entry(self, b: int, n: int) -> int:
+        return lib().oracle_hash_entry(self._h, b, n)
+
+    def hash_bracket(self, b: int, n: int, p: float) -> int:
+        return lib().oracle_hash_bracket(self._h, b, n, p)
+
+    def micro_xs(self, n: int, k: int, p: float) -> np.ndarray:
+        xs = np.zeros(5, np.float64)
+        lib().oracle_micro_xs(self._h, n, k, p, _ptr(xs))
+        return xs
+
+    def macro_xs(self, p: float, mat: int, mode: int = UNIONIZED):
+        M = np.zeros(5, np.float64)
+        gi = C.c_int64(0)
+        lib().oracle_macro_xs(self._h, p, mat, mode, _ptr(M), C.byref(gi))
+        return M, gi.value
+
+    def lookup(self, i: int, mode: int = UNIONIZED):
+        p, m, gi, v = C.c_double(), C.c_int32(), C.c_int64(), C.c_int32()
+        M = np.zeros(5, np.float64)
+        lib().oracle_lookup(self._h, i, mode, C.byref(p), C.byref(m), C.byref(gi), _ptr(M),
+                            C.byref(v))
+        return dict(p=p.value, mat=m.value, grid_index=gi.value, M=M, v=v.value)
+
+    def run(self, first: int, count: int, mode: int = UNIONIZED, nthreads: int = 1,
+            outputs: bool = False):
+        """Lookups [first, first+count).  Returns S (= sum v) or (S, dict of arrays)."""
+        if not outputs:
+            return lib().oracle_run(self._h, first, count, mode, nthreads, None, None, None,
+                                    None, None)
+        p = np.empty(count, np.float64)
+        mat = np.empty(count, np.int32)
+        gi = np.empty(count, np.int64)
+        M = np.empty((count, 5), np.float64)
+        v = np.empty(count, np.int32)
+        S = lib().oracle_run(self._h, first, count, mode, nthreads, _ptr(p), _ptr(mat), _ptr(gi),
+                             _ptr(M), _ptr(v))
+        return S, dict(p=p, mat=mat, grid_index=gi, M=M, v=v)
+
+    def run_explicit(self, p: np.ndarray, mat: np.ndarray, mode: int = UNIONIZED,
+                     nthreads: int = 1):
+        p = np.ascontiguousarray(p, np.float64)
+        mat = np.ascontiguousarray(mat, np.int32)
+        M = np.empty((len(p), 5), np.float64)
+        v = np.empty(len(p), np.int32)
+        S = lib().oracle_run_explicit(self._h, _ptr(p), _ptr(mat), len(p), mode, nthreads,
+                                      _ptr(M), _ptr(v))
+        return S, M, v

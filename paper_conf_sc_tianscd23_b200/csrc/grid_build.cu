@@ -1,0 +1,123 @@
+// grid_build.cu — device construction of the acceleration tables (run once
+// per grid at xs_init_grid; not part of the timed lookup step).
+//
+//   K0a  U  = sorted multiset of all I*N energies      (in-house LSD radix sort)
+//   K0b  IG[e][n] = clamp(ub(E_n, U[e]) - 1, 0, N-2)   (chunked search + sweep)
+//   K0c  HG[b][n] = clamp(ub(E_n, b du) - 1, 0, N-2)   (one search per entry)
+// Definitions: DESIGN.md R6, R7 (north_star: "the unionized (or
+// hash-accelerated) energy grid").
+#include "common.cuh"
+#include "radix_sort.cuh"
+#include "search.cuh"
+#include "xs_internal.h"
+
+namespace xs {
+
+// order-preserving map fp64 bits -> u64 (total order of non-NaN doubles)
+__device__ __forceinline__ uint64_t f2key(double x) {
+  uint64_t b = static_cast<uint64_t>(__double_as_longlong(x));
+  return (b >> 63) ? ~b : (b | 0x8000000000000000ULL);
+}
+__device__ __forceinline__ double key2f(uint64_t k) {
+  uint64_t b = (k >> 63) ? (k & 0x7fffffffffffffffULL) : ~k;
+  return __longlong_as_double(static_cast<long long>(b));
+}
+
+__global__ void k_extract_energy_keys(const double* __restrict__ grid, uint64_t n,
+                                      uint64_t* __restrict__ keys) {
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < n;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x)
+    keys[i] = f2key(grid[i * 6]);
+}
+
+__global__ void k_keys_to_energy(const uint64_t* __restrict__ keys, uint64_t n,
+                                 double* __restrict__ U) {
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < n;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x)
+    U[i] = key2f(keys[i]);
+}
+
+static int grid_for(uint64_t n, int threads, int sm) {
+  uint64_t b = (n + threads - 1) / threads;
+  uint64_t cap = static_cast<uint64_t>(sm) * 32;
+  return static_cast<int>(b < cap ? (b ? b : 1) : cap);
+}
+
+cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st) {
+  const uint64_t n = static_cast<uint64_t>(g.NU);
+  uint64_t* k0 = nullptr;
+  uint64_t* k1 = nullptr;
+  void* work = nullptr;
+  cudaError_t e = cudaMallocAsync(&k0, n * 8, st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&k1, n * 8, st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&work, rs::hist_bytes(n), st);
+  if (e == cudaSuccess) {
+    k_extract_energy_keys<<<grid_for(n, 256, g.sm_count), 256, 0, st>>>(g.grid, n, k0);
+    bool in1 = false;
+    e = rs::sort_pairs<uint64_t, false>(k0, nullptr, k1, nullptr, n, 64, work, st, &in1);
+    if (e == cudaSuccess) {
+      k_keys_to_energy<<<grid_for(n, 256, g.sm_count), 256, 0, st>>>(in1 ? k1 : k0, n, U);
+      e = cudaGetLastError();
+    }
+  }
+  if (k0) cudaFreeAsync(k0, st);
+  if (k1) cudaFreeAsync(k1, st);
+  if (work) cudaFreeAsync(work, st);
+  return e;
+}
+
+// K0b: block b owns rows [b R, (b+1) R); thread t owns nuclides t, t+T, ...
+// One binary search per (block, nuclide), then a monotone sweep: writes of a
+// row are consecutive in n (coalesced), reads of E_n advance monotonically.
+constexpr int kIgRows = 256;
+
+__global__ void __launch_bounds__(384) k_build_index_grid(const double* __restrict__ grid,
+                                                          int32_t I, int64_t N,
+                                                          const double* __restrict__ U,
+                                                          int64_t NU, int32_t* __restrict__ IG) {
+  const int64_t e0 = static_cast<int64_t>(blockIdx.x) * kIgRows;
+  const int64_t e1 = e0 + kIgRows < NU ? e0 + kIgRows : NU;
+  for (int32_t n = threadIdx.x; n < I; n += blockDim.x) {
+    const double* rec = grid + static_cast<int64_t>(n) * N * 6;
+    int64_t k = bracket_search_rec(rec, 0, N - 1, __ldg(U + e0));
+    double e_next = rec_energy(rec, k + 1);
+    for (int64_t e = e0; e < e1; ++e) {
+      const double q = __ldg(U + e);
+      while (k < N - 2 && e_next <= q) {
+        ++k;
+        e_next = rec_energy(rec, k + 1);
+      }
+      IG[e * I + n] = static_cast<int32_t>(k);
+    }
+  }
+}
+
+cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st) {
+  const int64_t blocks = (g.NU + kIgRows - 1) / kIgRows;
+  const int threads = g.I >= 384 ? 384 : ((g.I + 31) / 32) * 32;
+  k_build_index_grid<<<static_cast<unsigned>(blocks), threads, 0, st>>>(g.grid, g.I, g.N, g.U,
+                                                                         g.NU, g.index);
+  return cudaGetLastError();
+}
+
+__global__ void k_build_hash_grid(const double* __restrict__ grid, int32_t I, int64_t N, int32_t B,
+                                  double du, int32_t* __restrict__ HG) {
+  const uint64_t total = static_cast<uint64_t>(B) * I;
+  for (uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; t < total;
+       t += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    const int64_t b = static_cast<int64_t>(t / I);
+    const int32_t n = static_cast<int32_t>(t % I);
+    const double energy = static_cast<double>(b) * du;
+    HG[t] = static_cast<int32_t>(
+        bracket_search_rec(grid + static_cast<int64_t>(n) * N * 6, 0, N - 1, energy));
+  }
+}
+
+cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st) {
+  const uint64_t total = static_cast<uint64_t>(g.B) * g.I;
+  k_build_hash_grid<<<grid_for(total, 256, g.sm_count), 256, 0, st>>>(g.grid, g.I, g.N, g.B,
+                                                                        g.du, g.index);
+  return cudaGetLastError();
+}
+
+}  // namespace xs

@@ -1,0 +1,671 @@
+// lookup.cu — the timed hot path: A1 sample, A2 (optional) sort, A3 search,
+// A4 index gather, A5 record-pair gather, A6 interpolate, A7 accumulate,
+// A8 verify (BASELINE.json north_star).
+//
+// Pipeline of one xs_lookup_batch call (all on the caller's stream):
+//   k_count     A1: per-material histogram of the batch (materials only)
+//   k_bucket    A1+A3: sample (p, m) again, search p on U (or hash bin),
+//               write a 16-B LookupRec into the material bucket
+//               (unsorted) or in id order plus a (material, energy) key
+//               (sorted; then the in-house radix sort produces the
+//               permutation — A2)
+//   k_gather    A4-A8: warp-per-task over material buckets; each group of
+//               G=3 lanes owns one lookup and walks the material's nuclides
+//               in list order; per nuclide the 3 lanes gather the 96-B
+//               record pair as 2x3 128-bit loads (lane r takes 16-B chunk r
+//               of the low and of the high record), lane 0 computes the
+//               interpolation weight f and broadcasts it, each lane
+//               interpolates its two channels and accumulates them in list
+//               order (exact binary64, no FMA), so every M_c is bit-identical
+//               to the serial definition.
+//   verification: v = 1 + argmax; per-block reduction, one atomic per block.
+#include <cfloat>
+
+#include "common.cuh"
+#include "radix_sort.cuh"
+#include "search.cuh"
+#include "xs_internal.h"
+
+namespace xs {
+
+__constant__ JumpTable c_jump;
+
+cudaError_t init_constants() {
+  JumpTable t = make_jump_table();
+  return cudaMemcpyToSymbol(c_jump, &t, sizeof(t));
+}
+
+// ------------------------------------------------------------------ A1 ----
+// LCG^n(s) through the constant-memory jump table (powers of one affine map
+// commute, so the bits can be applied in any order).
+__device__ __forceinline__ uint64_t fast_forward(uint64_t s, uint64_t n) {
+  s &= kMask63;
+  int b = 0;
+  while (n) {
+    if (n & 1ULL) s = (c_jump.A[b] * s + c_jump.C[b]) & kMask63;
+    n >>= 1;
+    ++b;
+  }
+  return s;
+}
+
+struct Sample {
+  double p;
+  int32_t mat;
+};
+
+// lookup id -> (p, mat): s = FF(seed, 2 id); p = draw; roll = draw (R4)
+__device__ __forceinline__ Sample sample_lookup(uint64_t seed, uint64_t id) {
+  uint64_t s = fast_forward(seed, 2 * id);
+  s = lcg_next(s);
+  const double p = lcg_double(s);
+  s = lcg_next(s);
+  return Sample{p, pick_material(lcg_double(s))};
+}
+
+struct Params {
+  // grid
+  const double* grid;
+  int32_t I;
+  int64_t N;
+  const double* U;
+  int64_t NU;
+  const int32_t* index;
+  int32_t B;
+  double du;
+  const int32_t* num_nucs;
+  const int32_t* mats;
+  const double* concs;
+  int32_t n_mats, max_nucs;
+  // batch
+  uint64_t seed, first_id;
+  uint32_t count;
+  const double* in_energy;
+  const int32_t* in_mat;
+  // workspace
+  uint32_t* counts;
+  uint32_t* cursor;
+  LookupRec* recs;
+  uint32_t* keys;
+  uint32_t* vals;
+  const uint32_t* perm;
+  // outputs
+  double* out_M;
+  double* out_E;
+  int32_t* out_mat;
+  int64_t* out_gidx;
+  int32_t* out_v;
+  unsigned long long* vsum;
+};
+
+__device__ __forceinline__ Sample get_lookup(const Params& P, uint32_t i) {
+  if (P.in_energy) {
+    int32_t m = P.in_mat[i];
+    if (m < 0 || m >= P.n_mats) m = P.n_mats;  // invalid bucket
+    return Sample{P.in_energy[i], m};
+  }
+  return sample_lookup(P.seed, P.first_id + i);
+}
+
+template <int GT>
+__device__ __forceinline__ int32_t grid_index_of(const Params& P, double p) {
+  if (GT == XS_GRID_UNIONIZED) return static_cast<int32_t>(union_search(P.U, P.NU, p));
+  if (GT == XS_GRID_HASH) return hash_bin(p, P.du, P.B);
+  return -1;
+}
+
+// k_count: histogram of materials over the batch (bucket n_mats = invalid)
+__global__ void __launch_bounds__(256) k_count(Params P) {
+  __shared__ uint32_t s_h[kMaxMats + 1];
+  for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x) s_h[t] = 0;
+  __syncthreads();
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < P.count;
+       i += gridDim.x * blockDim.x) {
+    int32_t m;
+    if (P.in_energy) {
+      m = P.in_mat[i];
+      if (m < 0 || m >= P.n_mats) m = P.n_mats;
+    } else {
+      m = sample_lookup(P.seed, P.first_id + i).mat;
+    }
+    atomicAdd(&s_h[m], 1u);
+  }
+  __syncthreads();
+  for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x)
+    if (s_h[t]) atomicAdd(&P.counts[t], s_h[t]);
+}
+
+constexpr int kBucketThreads = 256;
+constexpr int kBucketItems = 4;
+
+__device__ __forceinline__ void write_invalid(const Params& P, uint32_t i) {
+  if (P.out_M)
+    for (int c = 0; c < 5; ++c) P.out_M[static_cast<uint64_t>(i) * 5 + c] = __longlong_as_double(0x7ff8000000000000LL);
+  if (P.out_v) P.out_v[i] = 0;
+}
+
+// k_bucket: A1 + A3.  SORTED=false: scatter into material buckets with
+// block-aggregated cursors; SORTED=true: records in id order + sort keys.
+template <int GT, bool SORTED>
+__global__ void __launch_bounds__(kBucketThreads) k_bucket(Params P) {
+  __shared__ uint32_t s_off[kMaxMats + 2];
+  __shared__ uint32_t s_cnt[kMaxMats + 1];
+  __shared__ uint32_t s_base[kMaxMats + 1];
+  const int nm1 = P.n_mats + 1;
+  if (threadIdx.x == 0) {
+    uint32_t run = 0;
+    for (int m = 0; m < nm1; ++m) {
+      s_off[m] = run;
+      run += P.counts[m];
+    }
+    s_off[nm1] = run;
+  }
+  __syncthreads();
+  // material-field width of the sort key
+  int mat_bits = 1;
+  while ((1 << mat_bits) < nm1) ++mat_bits;
+  const int p_bits = 32 - mat_bits;
+  const uint32_t chunk = kBucketThreads * kBucketItems;
+  for (uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * chunk; c0 < P.count;
+       c0 += static_cast<uint64_t>(gridDim.x) * chunk) {
+    if (!SORTED) {
+      for (int t = threadIdx.x; t < nm1; t += blockDim.x) s_cnt[t] = 0;
+      __syncthreads();
+    }
+    Sample smp[kBucketItems];
+    int32_t gi[kBucketItems];
+    uint32_t rank[kBucketItems];
+#pragma unroll
+    for (int it = 0; it < kBucketItems; ++it) {
+      const uint64_t i = c0 + static_cast<uint64_t>(it) * kBucketThreads + threadIdx.x;
+      const bool ok = i < P.count;
+      smp[it] = ok ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
+      gi[it] = 0;
+      if (ok && smp[it].mat < P.n_mats) gi[it] = grid_index_of<GT>(P, smp[it].p);
+      rank[it] = 0;
+      if (!SORTED) {
+        // warp-aggregated shared-memory rank within the block
+        const int key = ok ? smp[it].mat : kMaxMats + 7;
+        const uint32_t peers = __match_any_sync(0xffffffffu, key);
+        const int lane = threadIdx.x & 31;
+        const int leader = __ffs(peers) - 1;
+        uint32_t b = 0;
+        if (ok && lane == leader) b = atomicAdd(&s_cnt[key], __popc(peers));
+        b = __shfl_sync(0xffffffffu, b, leader);
+        rank[it] = b + __popc(peers & ((1u << lane) - 1u));
+      }
+    }
+    if (!SORTED) {
+      __syncthreads();
+      for (int t = threadIdx.x; t < nm1; t += blockDim.x)
+        s_base[t] = s_cnt[t] ? s_off[t] + atomicAdd(&P.cursor[t], s_cnt[t]) : 0u;
+      __syncthreads();
+    }
+#pragma unroll
+    for (int it = 0; it < kBucketItems; ++it) {
+      const uint64_t i64 = c0 + static_cast<uint64_t>(it) * kBucketThreads + threadIdx.x;
+      if (i64 >= P.count) continue;
+      const uint32_t i = static_cast<uint32_t>(i64);
+      const int32_t m = smp[it].mat;
+      const double p = smp[it].p;
+      LookupRec r;
+      r.p = p;
+      r.idx = i;
+      r.gidx = gi[it];
+      if (SORTED) {
+        P.recs[i] = r;
+        double q = p * static_cast<double>(1u << p_bits);
+        uint32_t pk = q > 0.0 ? (q < static_cast<double>((1u << p_bits) - 1u)
+                                     ? static_cast<uint32_t>(q)
+                                     : (1u << p_bits) - 1u)
+                              : 0u;
+        P.keys[i] = (static_cast<uint32_t>(m) << p_bits) | pk;
+        P.vals[i] = i;
+      } else {
+        P.recs[s_base[m] + rank[it]] = r;
+      }
+      if (P.out_E) P.out_E[i] = p;
+      if (P.out_mat) P.out_mat[i] = m < P.n_mats ? m : (P.in_mat ? P.in_mat[i] : -1);
+      if (P.out_gidx) P.out_gidx[i] = (m < P.n_mats && GT != XS_GRID_NUCLIDE) ? gi[it] : -1;
+      if (m >= P.n_mats) write_invalid(P, i);
+    }
+    if (!SORTED) __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------- A4 -- A8 ---
+// Bracket index k_n for the lookup's energy through the grid's structure.
+template <int GT>
+__device__ __forceinline__ int32_t bracket_of(const Params& P, int32_t gidx, int32_t n, double p) {
+  if (GT == XS_GRID_UNIONIZED)
+    return __ldg(P.index + static_cast<int64_t>(gidx) * P.I + n);
+  const double* rec = P.grid + static_cast<int64_t>(n) * P.N * 6;
+  if (GT == XS_GRID_HASH) return hash_bracket(P.index, P.I, P.B, gidx, n, rec, P.N, p);
+  return nuclide_bracket(rec, P.N, p);
+}
+
+constexpr int kGatherThreads = 256;
+constexpr int kG = 3;                 // lanes per lookup
+constexpr int kLPT = 32 / kG;         // lookups per warp task (10)
+
+struct GatherSmem {
+  int32_t num[kMaxMats];
+  uint32_t off[kMaxMats + 1];   // bucket start of material m
+  uint32_t cnt[kMaxMats];
+  uint32_t toff[kMaxMats + 1];  // first task of material m
+};
+
+// U = nuclides per round per group (multiple of kG)
+template <int GT, bool SORTED, int U>
+__global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
+  static_assert(U % kG == 0, "U must be a multiple of the group size");
+  constexpr int Q = U / kG;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  double* s_concs = reinterpret_cast<double*>(smem_raw + sizeof(GatherSmem));
+  int32_t* s_mats = reinterpret_cast<int32_t*>(s_concs + tab);
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    s_concs[t] = P.concs[t];
+    s_mats[t] = P.mats[t];
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kLPT - 1) / kLPT;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const int g = lane / kG;
+  const int r = lane - g * kG;
+  const int base = g * kG;
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t warps_per_block = blockDim.x >> 5;
+  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
+  const uint32_t nw = gridDim.x * warps_per_block;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nw) {
+    while (task >= S.toff[m + 1]) ++m;  // tasks are visited in increasing order
+    const uint32_t slot = (task - S.toff[m]) * kLPT + g;
+    const bool valid = (g < kLPT) && (slot < S.cnt[m]);
+    LookupRec rec{0.5, 0u, 0};
+    if (valid) {
+      uint32_t pos = S.off[m] + slot;
+      if (SORTED) pos = __ldg(P.perm + pos);
+      rec = P.recs[pos];
+    }
+    const double p = rec.p;
+    const int nn = S.num[m];
+    const int32_t* mrow = s_mats + m * P.max_nucs;
+    const double* crow = s_concs + m * P.max_nucs;
+
+    double acc_a = 0.0, acc_b = 0.0;
+    int32_t knext[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const int j = r + q * kG;
+      knext[q] = (valid && j < nn) ? bracket_of<GT>(P, rec.gidx, mrow[j], p) : 0;
+    }
+    for (int j0 = 0; j0 < nn; j0 += U) {
+      int32_t kcur[Q];
+#pragma unroll
+      for (int q = 0; q < Q; ++q) kcur[q] = knext[q];
+      // A4 for the next round (overlaps this round's pair gathers)
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {
+        const int j = j0 + U + r + q * kG;
+        knext[q] = (valid && j < nn) ? bracket_of<GT>(P, rec.gidx, mrow[j], p) : 0;
+      }
+      // A5: 96-B record pairs, lane r loads chunk r of the low and high record
+      double2 lo[U], hi[U];
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + t;
+        const int32_t kt = __shfl_sync(0xffffffffu, kcur[t / kG], base + (t % kG));
+        lo[t] = make_double2(0.0, 0.0);
+        hi[t] = make_double2(1.0, 0.0);
+        if (valid && j < nn) {
+          const int32_t n = mrow[j];
+          const double2* pr = grid2 + (static_cast<int64_t>(n) * P.N + kt) * 3;
+          lo[t] = __ldg(pr + r);
+          hi[t] = __ldg(pr + 3 + r);
+        }
+      }
+      // A6 + A7 in list order
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + t;
+        if (j < nn) {  // warp-uniform
+          double f = 0.0;
+          if (r == 0) f = ddiv(dsub(hi[t].x, p), dsub(hi[t].x, lo[t].x));
+          f = __shfl_sync(0xffffffffu, f, base);
+          const double xa = dsub(hi[t].x, dmul(f, dsub(hi[t].x, lo[t].x)));
+          const double xb = dsub(hi[t].y, dmul(f, dsub(hi[t].y, lo[t].y)));
+          const double c = crow[j];
+          acc_a = dadd(acc_a, dmul(xa, c));
+          acc_b = dadd(acc_b, dmul(xb, c));
+        }
+      }
+    }
+    // A8: channels (t, s, a, f, nf) = (b@r0, a@r1, b@r1, a@r2, b@r2)
+    double M[5];
+    M[0] = __shfl_sync(0xffffffffu, acc_b, base);
+    M[1] = __shfl_sync(0xffffffffu, acc_a, base + 1);
+    M[2] = __shfl_sync(0xffffffffu, acc_b, base + 1);
+    M[3] = __shfl_sync(0xffffffffu, acc_a, base + 2);
+    M[4] = __shfl_sync(0xffffffffu, acc_b, base + 2);
+    if (valid && r == 0) {
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[c] > mx) {
+          mx = M[c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[rec.idx] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(rec.idx) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[c];
+      }
+    }
+  }
+  // block reduction of the verification sums; one atomic pair per block
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
+  if (lane == 0) {
+    s_red[0][threadIdx.x >> 5] = acc_v;
+    s_red[1][threadIdx.x >> 5] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (uint32_t w = 0; w < warps_per_block; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
+// --------------------------------------------------- XSBench-shape baseline
+// One thread per lookup, no bucketing, serial nuclide loop (the shape of the
+// CUDA kernels the paper measured).  Same exact
+// arithmetic.  For comparison only (XS_FLAG_BASELINE).
+template <int GT>
+__global__ void __launch_bounds__(256) k_baseline(Params P) {
+  unsigned long long acc_v = 0, acc_n = 0;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < P.count;
+       i += gridDim.x * blockDim.x) {
+    const Sample s = get_lookup(P, i);
+    if (s.mat >= P.n_mats) {
+      write_invalid(P, i);
+      if (P.out_mat) P.out_mat[i] = P.in_mat ? P.in_mat[i] : -1;
+      if (P.out_gidx) P.out_gidx[i] = -1;
+      if (P.out_E) P.out_E[i] = s.p;
+      continue;
+    }
+    const int32_t gidx = grid_index_of<GT>(P, s.p);
+    double M[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
+    const int nn = P.num_nucs[s.mat];
+    for (int j = 0; j < nn; ++j) {
+      const int32_t n = __ldg(P.mats + s.mat * P.max_nucs + j);
+      const double c = __ldg(P.concs + s.mat * P.max_nucs + j);
+      const int32_t k = bracket_of<GT>(P, gidx, n, s.p);
+      const double2* pr =
+          reinterpret_cast<const double2*>(P.grid) + (static_cast<int64_t>(n) * P.N + k) * 3;
+      const double2 l0 = __ldg(pr), l1 = __ldg(pr + 1), l2 = __ldg(pr + 2);
+      const double2 h0 = __ldg(pr + 3), h1 = __ldg(pr + 4), h2 = __ldg(pr + 5);
+      const double f = ddiv(dsub(h0.x, s.p), dsub(h0.x, l0.x));
+      const double lo[5] = {l0.y, l1.x, l1.y, l2.x, l2.y};
+      const double hi[5] = {h0.y, h1.x, h1.y, h2.x, h2.y};
+#pragma unroll
+      for (int ch = 0; ch < 5; ++ch) {
+        const double x = dsub(hi[ch], dmul(f, dsub(hi[ch], lo[ch])));
+        M[ch] = dadd(M[ch], dmul(x, c));
+      }
+    }
+    double mx = -1.0;
+    int vi = 0;
+#pragma unroll
+    for (int ch = 0; ch < 5; ++ch)
+      if (M[ch] > mx) {
+        mx = M[ch];
+        vi = ch;
+      }
+    acc_v += static_cast<unsigned long long>(vi + 1);
+    acc_n += 1;
+    if (P.out_v) P.out_v[i] = vi + 1;
+    if (P.out_M)
+      for (int ch = 0; ch < 5; ++ch) P.out_M[static_cast<uint64_t>(i) * 5 + ch] = M[ch];
+    if (P.out_E) P.out_E[i] = s.p;
+    if (P.out_mat) P.out_mat[i] = s.mat;
+    if (P.out_gidx) P.out_gidx[i] = GT == XS_GRID_NUCLIDE ? -1 : gidx;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  if ((threadIdx.x & 31) == 0 && acc_n) {
+    atomicAdd(P.vsum, acc_v);
+    atomicAdd(P.vsum + 1, acc_n);
+  }
+}
+
+// ------------------------------------------------------------ A8 alone ----
+__global__ void k_verify(const double* __restrict__ M, uint64_t count,
+                         unsigned long long* __restrict__ vsum) {
+  unsigned long long acc_v = 0, acc_n = 0;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < count;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    double mx = -1.0;
+    int vi = 0;
+    for (int c = 0; c < 5; ++c) {
+      const double x = M[i * 5 + c];
+      if (x > mx) {
+        mx = x;
+        vi = c;
+      }
+    }
+    acc_v += static_cast<unsigned long long>(vi + 1);
+    acc_n += 1;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  if ((threadIdx.x & 31) == 0 && acc_n) {
+    atomicAdd(vsum, acc_v);
+    atomicAdd(vsum + 1, acc_n);
+  }
+}
+
+template <int GT>
+__global__ void k_nuclide_index(Params P, const double* __restrict__ energy,
+                                const int32_t* __restrict__ nuc, uint64_t count,
+                                int32_t* __restrict__ k_out) {
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < count;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    const double p = energy[i];
+    const int32_t n = nuc[i];
+    const int32_t gidx = grid_index_of<GT>(P, p);
+    k_out[i] = bracket_of<GT>(P, gidx, n, p);
+  }
+}
+
+// ----------------------------------------------------------------- host ----
+static Params make_params(const DeviceGrid& g) {
+  Params P{};
+  P.grid = g.grid;
+  P.I = g.I;
+  P.N = g.N;
+  P.U = g.U;
+  P.NU = g.NU;
+  P.index = g.index;
+  P.B = g.B;
+  P.du = g.du;
+  P.num_nucs = g.num_nucs;
+  P.mats = g.mats;
+  P.concs = g.concs;
+  P.n_mats = g.n_mats;
+  P.max_nucs = g.max_nucs;
+  P.seed = g.lookup_seed;
+  return P;
+}
+
+static unsigned grid_cap(uint64_t work, int threads, int sm, int per_sm) {
+  uint64_t b = (work + threads - 1) / threads;
+  uint64_t cap = static_cast<uint64_t>(sm) * per_sm;
+  if (b == 0) b = 1;
+  return static_cast<unsigned>(b < cap ? b : cap);
+}
+
+template <int GT, bool SORTED, int U>
+static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t smem = sizeof(GatherSmem) +
+                      static_cast<size_t>(g.n_mats) * g.max_nucs * (sizeof(double) + sizeof(int32_t));
+  auto kern = k_gather<GT, SORTED, U>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
+template <int GT, bool SORTED>
+static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  switch (g.unroll) {
+    case 3: return launch_gather<GT, SORTED, 3>(g, P, st);
+    case 9: return launch_gather<GT, SORTED, 9>(g, P, st);
+    default: return launch_gather<GT, SORTED, 6>(g, P, st);
+  }
+}
+
+template <int GT>
+static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
+                                cudaStream_t st) {
+  Params P = make_params(g);
+  P.first_id = a.first_id;
+  P.count = a.count;
+  P.in_energy = a.in_energy;
+  P.in_mat = a.in_mat;
+  P.counts = ws.counts;
+  P.cursor = ws.cursor;
+  P.recs = ws.recs;
+  P.out_M = a.out.macro_xs;
+  P.out_E = a.out.energy;
+  P.out_mat = a.out.mat;
+  P.out_gidx = a.out.grid_index;
+  P.out_v = a.out.verification;
+  P.vsum = reinterpret_cast<unsigned long long*>(a.out.vsum);
+  auto mark = [&](int i) {
+    if (a.ev) cudaEventRecord(a.ev[i], st);
+  };
+  auto launched = [&](uint64_t n) {
+    if (a.launches) *a.launches += n;
+  };
+  cudaError_t e;
+  mark(0);
+  if (a.flags & XS_FLAG_BASELINE) {
+    mark(1);
+    mark(2);
+    k_baseline<GT><<<grid_cap(a.count, 256, g.sm_count, 16), 256, 0, st>>>(P);
+    launched(1);
+    mark(3);
+    return cudaGetLastError();
+  }
+  e = cudaMemsetAsync(ws.counts, 0, 2 * (kMaxMats + 1) * sizeof(uint32_t), st);
+  if (e != cudaSuccess) return e;
+  k_count<<<grid_cap(a.count, 256, g.sm_count, 8), 256, 0, st>>>(P);
+  const unsigned nb = grid_cap(a.count, kBucketThreads * kBucketItems, g.sm_count, 16);
+  const bool sorted = a.flags & XS_FLAG_SORT;
+  if (sorted) {
+    P.keys = ws.keys0;
+    P.vals = ws.vals0;
+    k_bucket<GT, true><<<nb, kBucketThreads, 0, st>>>(P);
+  } else {
+    k_bucket<GT, false><<<nb, kBucketThreads, 0, st>>>(P);
+  }
+  launched(2);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  mark(1);
+  if (sorted) {
+    bool in1 = false;
+    e = rs::sort_pairs<uint32_t, true>(ws.keys0, ws.vals0, ws.keys1, ws.vals1, a.count, 32,
+                                       ws.sort_work, st, &in1);
+    if (e != cudaSuccess) return e;
+    launched(12);
+    P.perm = in1 ? ws.vals1 : ws.vals0;
+  }
+  mark(2);
+  e = sorted ? launch_gather_u<GT, true>(g, P, st) : launch_gather_u<GT, false>(g, P, st);
+  launched(1);
+  mark(3);
+  return e;
+}
+
+cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
+                       cudaStream_t st) {
+  switch (g.grid_type) {
+    case XS_GRID_UNIONIZED: return run_lookup_t<XS_GRID_UNIONIZED>(g, a, ws, st);
+    case XS_GRID_HASH: return run_lookup_t<XS_GRID_HASH>(g, a, ws, st);
+    default: return run_lookup_t<XS_GRID_NUCLIDE>(g, a, ws, st);
+  }
+}
+
+cudaError_t run_verify(const DeviceGrid& g, const double* M, uint64_t count, uint64_t* vsum,
+                       cudaStream_t st) {
+  k_verify<<<grid_cap(count, 256, g.sm_count, 8), 256, 0, st>>>(
+      M, count, reinterpret_cast<unsigned long long*>(vsum));
+  return cudaGetLastError();
+}
+
+cudaError_t run_nuclide_index(const DeviceGrid& g, const double* energy, const int32_t* nuc,
+                              uint64_t count, int32_t* k_out, cudaStream_t st) {
+  Params P = make_params(g);
+  const unsigned nb = grid_cap(count, 256, g.sm_count, 8);
+  switch (g.grid_type) {
+    case XS_GRID_UNIONIZED:
+      k_nuclide_index<XS_GRID_UNIONIZED><<<nb, 256, 0, st>>>(P, energy, nuc, count, k_out);
+      break;
+    case XS_GRID_HASH:
+      k_nuclide_index<XS_GRID_HASH><<<nb, 256, 0, st>>>(P, energy, nuc, count, k_out);
+      break;
+    default:
+      k_nuclide_index<XS_GRID_NUCLIDE><<<nb, 256, 0, st>>>(P, energy, nuc, count, k_out);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace xs

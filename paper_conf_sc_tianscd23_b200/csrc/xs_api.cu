@@ -1,0 +1,535 @@
+// xs_api.cu — the C-ABI (include/xs.h): argument checking, ownership,
+// device selection, workspace layout and staging.  All compute is in
+// grid_build.cu / lookup.cu; there is no host compute path and no fallback.
+#include <cuda_runtime.h>
+
+#include <array>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <new>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../gen/xs_gen.h"
+#include "common.cuh"
+#include "radix_sort.cuh"
+#include "xs_internal.h"
+
+struct xs_grid {
+  xs::DeviceGrid d;
+  // per-phase event timing (xs_timing_enable / xs_timing_read)
+  bool timing = false;
+  std::vector<std::array<cudaEvent_t, 4>> ev;
+  size_t ev_used = 0;
+  uint64_t calls = 0;
+  uint64_t launches_read = 0;
+};
+
+namespace xs {
+
+static thread_local std::string g_err;
+
+static xs_status fail(xs_status code, const std::string& msg, cudaError_t ce = cudaSuccess) {
+  g_err = msg;
+  if (ce != cudaSuccess) {
+    g_err += ": ";
+    g_err += cudaGetErrorName(ce);
+    g_err += " (";
+    g_err += cudaGetErrorString(ce);
+    g_err += ")";
+    if (ce == cudaErrorMemoryAllocation) code = XS_ERR_OUT_OF_MEMORY;
+    cudaGetLastError();  // clear sticky-free errors
+  }
+  return code;
+}
+
+#define XS_TRY(expr, what)                                   \
+  do {                                                       \
+    cudaError_t _e = (expr);                                 \
+    if (_e != cudaSuccess) return fail(XS_ERR_CUDA, what, _e); \
+  } while (0)
+
+// Switch to the grid's device for the duration of a call.
+struct DeviceGuard {
+  int prev = -1;
+  bool ok = false;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    ok = cudaSetDevice(dev) == cudaSuccess;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+static size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
+
+size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws) {
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off += align256(bytes);
+    return o;
+  };
+  const size_t o_counts = take(2 * (kMaxMats + 1) * sizeof(uint32_t));
+  const size_t o_recs = take(count * sizeof(LookupRec));
+  size_t o_k0 = 0, o_k1 = 0, o_v0 = 0, o_v1 = 0, o_work = 0;
+  if (flags & XS_FLAG_SORT) {
+    o_k0 = take(count * 4);
+    o_k1 = take(count * 4);
+    o_v0 = take(count * 4);
+    o_v1 = take(count * 4);
+    o_work = take(rs::hist_bytes(count));
+  }
+  if (ws) {
+    char* b = static_cast<char*>(base);
+    ws->counts = reinterpret_cast<uint32_t*>(b + o_counts);
+    ws->cursor = ws->counts + (kMaxMats + 1);
+    ws->recs = reinterpret_cast<LookupRec*>(b + o_recs);
+    ws->keys0 = reinterpret_cast<uint32_t*>(b + o_k0);
+    ws->keys1 = reinterpret_cast<uint32_t*>(b + o_k1);
+    ws->vals0 = reinterpret_cast<uint32_t*>(b + o_v0);
+    ws->vals1 = reinterpret_cast<uint32_t*>(b + o_v1);
+    ws->sort_work = b + o_work;
+    ws->total = off;
+  }
+  return off;
+}
+
+// staging area for XS_FLAG_HOST_IO (after the compute workspace)
+struct Staging {
+  double* energy;
+  int32_t* mat;
+  double* M;
+  double* E;
+  int32_t* omat;
+  int64_t* gidx;
+  int32_t* v;
+  uint64_t* vsum;
+};
+
+static size_t staging_layout(uint64_t count, void* base, Staging* s) {
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off += align256(bytes);
+    return o;
+  };
+  const size_t o_e = take(count * 8), o_m = take(count * 4), o_M = take(count * 40),
+               o_E = take(count * 8), o_om = take(count * 4), o_g = take(count * 8),
+               o_v = take(count * 4), o_s = take(16);
+  if (s) {
+    char* b = static_cast<char*>(base);
+    s->energy = reinterpret_cast<double*>(b + o_e);
+    s->mat = reinterpret_cast<int32_t*>(b + o_m);
+    s->M = reinterpret_cast<double*>(b + o_M);
+    s->E = reinterpret_cast<double*>(b + o_E);
+    s->omat = reinterpret_cast<int32_t*>(b + o_om);
+    s->gidx = reinterpret_cast<int64_t*>(b + o_g);
+    s->v = reinterpret_cast<int32_t*>(b + o_v);
+    s->vsum = reinterpret_cast<uint64_t*>(b + o_s);
+  }
+  return off;
+}
+
+static size_t total_workspace(uint64_t count, uint32_t flags) {
+  size_t w = workspace_layout(count, flags, nullptr, nullptr);
+  if (flags & XS_FLAG_HOST_IO) w += staging_layout(count, nullptr, nullptr);
+  return w;
+}
+
+static xs_status check_device(int device, int* sm_count) {
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess || n == 0) return fail(XS_ERR_CUDA, "no CUDA device available", e);
+  if (device < 0 || device >= n) return fail(XS_ERR_INVALID_ARG, "device index out of range");
+  cudaDeviceProp prop;
+  XS_TRY(cudaGetDeviceProperties(&prop, device), "cudaGetDeviceProperties");
+  if (prop.major != 10)
+    return fail(XS_ERR_UNSUPPORTED, "libxs is built for sm_100a (B200); device is sm_" +
+                                        std::to_string(prop.major * 10 + prop.minor));
+  *sm_count = prop.multiProcessorCount;
+  return XS_OK;
+}
+
+static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st, xs_grid** out) {
+  const int32_t I = d->n_isotopes;
+  const int64_t N = d->n_gridpoints;
+  if (I < 1 || N < 2 || !d->nuclide_grid || d->n_mats < 1 || d->max_num_nucs < 1 ||
+      !d->num_nucs || !d->mats || !d->concs)
+    return fail(XS_ERR_INVALID_ARG, "xs_grid_data: missing array or bad size");
+  if (N > 0x7fffffffLL || static_cast<int64_t>(I) * N >= 0x7fffffffLL)
+    return fail(XS_ERR_UNSUPPORTED, "I*N must be < 2^31 (32-bit grid indices)");
+  if (d->n_mats > kMaxMats)
+    return fail(XS_ERR_UNSUPPORTED, "more than 64 materials");
+  if (d->grid_type < 0 || d->grid_type > 2) return fail(XS_ERR_INVALID_ARG, "bad grid_type");
+  if (d->grid_type == XS_GRID_HASH && d->hash_bins < 1)
+    return fail(XS_ERR_INVALID_ARG, "hash grid needs hash_bins >= 1");
+  const size_t tab = static_cast<size_t>(d->n_mats) * d->max_num_nucs;
+  if (tab * 12 > 160 * 1024)
+    return fail(XS_ERR_UNSUPPORTED, "material tables exceed the 160 KB shared-memory stage");
+  for (int32_t m = 0; m < d->n_mats; ++m) {
+    if (d->num_nucs[m] < 0 || d->num_nucs[m] > d->max_num_nucs)
+      return fail(XS_ERR_INVALID_ARG, "num_nucs out of range");
+    for (int32_t j = 0; j < d->num_nucs[m]; ++j) {
+      const int32_t n = d->mats[static_cast<size_t>(m) * d->max_num_nucs + j];
+      if (n < 0 || n >= I) return fail(XS_ERR_INVALID_ARG, "mats: nuclide id out of range");
+    }
+  }
+  for (int32_t n = 0; n < I; ++n) {
+    const double* E = d->nuclide_grid + static_cast<size_t>(n) * N * 6;
+    if (d->grid_type == XS_GRID_HASH && !(E[0] >= 0.0))
+      return fail(XS_ERR_INVALID_ARG, "hash grid needs non-negative energies");
+    for (int64_t k = 1; k < N; ++k)
+      if (!(E[(k - 1) * 6] < E[k * 6]))
+        return fail(XS_ERR_DATA, "nuclide " + std::to_string(n) +
+                                     ": energies not strictly increasing");
+  }
+  int sm = 0;
+  xs_status s = check_device(device, &sm);
+  if (s != XS_OK) return s;
+  DeviceGuard guard(device);
+  if (!guard.ok) return fail(XS_ERR_CUDA, "cudaSetDevice failed");
+  XS_TRY(init_constants(), "init_constants");
+
+  std::unique_ptr<xs_grid> g(new (std::nothrow) xs_grid());
+  if (!g) return fail(XS_ERR_OUT_OF_MEMORY, "host allocation");
+  DeviceGrid& G = g->d;
+  G.device = device;
+  G.sm_count = sm;
+  G.I = I;
+  G.N = N;
+  G.n_mats = d->n_mats;
+  G.max_nucs = d->max_num_nucs;
+  G.grid_type = d->grid_type;
+  G.B = d->grid_type == XS_GRID_HASH ? d->hash_bins : 0;
+  G.du = G.B ? 1.0 / static_cast<double>(G.B) : 0.0;
+  G.lookup_seed = d->lookup_seed;
+  G.NU = d->grid_type == XS_GRID_UNIONIZED ? static_cast<int64_t>(I) * N : 0;
+  G.index_len = d->grid_type == XS_GRID_UNIONIZED ? G.NU * I
+                : d->grid_type == XS_GRID_HASH    ? static_cast<int64_t>(G.B) * I
+                                                  : 0;
+  auto cleanup = [&]() {
+    cudaFree(G.grid);
+    cudaFree(G.U);
+    cudaFree(G.index);
+    cudaFree(G.num_nucs);
+    cudaFree(G.mats);
+    cudaFree(G.concs);
+  };
+  const size_t grid_bytes = static_cast<size_t>(I) * N * 6 * sizeof(double);
+  cudaError_t e = cudaMalloc(&G.grid, grid_bytes);
+  if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
+  if (e == cudaSuccess && G.index_len) e = cudaMalloc(&G.index, G.index_len * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&G.num_nucs, d->n_mats * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&G.mats, tab * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&G.concs, tab * sizeof(double));
+  if (e != cudaSuccess) {
+    cleanup();
+    return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
+  }
+  G.device_bytes = grid_bytes + G.NU * 8 + G.index_len * 4 + d->n_mats * 4 + tab * 12;
+  e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(G.mats, d->mats, tab * 4, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(G.concs, d->concs, tab * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
+    e = build_union_grid(G, G.U, st);
+    if (e == cudaSuccess) e = build_index_grid(G, st);
+  }
+  if (e == cudaSuccess && G.grid_type == XS_GRID_HASH) e = build_hash_grid(G, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) {
+    cleanup();
+    return fail(XS_ERR_CUDA, "grid upload / build", e);
+  }
+  *out = g.release();
+  return XS_OK;
+}
+
+}  // namespace xs
+
+using namespace xs;
+
+extern "C" {
+
+uint32_t xs_abi_version(void) { return XS_ABI_VERSION; }
+
+const char* xs_last_error(void) { return g_err.c_str(); }
+
+uint64_t xs_hash_finalize(uint64_t global_sum) { return global_sum % 999983ULL; }
+
+xs_status xs_init_grid(const xs_grid_spec* spec, int device, void* cuda_stream, xs_grid** out) {
+  if (!spec || !out) return fail(XS_ERR_INVALID_ARG, "NULL spec/out");
+  *out = nullptr;
+  if (spec->abi_version != XS_ABI_VERSION) return fail(XS_ERR_INVALID_ARG, "abi_version mismatch");
+  if (spec->reserved0 != 0) return fail(XS_ERR_INVALID_ARG, "reserved0 must be 0");
+  const int32_t I = spec->n_isotopes;
+  const int64_t N = spec->n_gridpoints;
+  const int32_t mx = xsgen_max_num_nucs(I, spec->material_rule);
+  if (I < 1 || N < 2 || mx < 1)
+    return fail(XS_ERR_INVALID_ARG, "bad spec (I, N or material_rule; rule 0 needs I in {68,355})");
+  if (static_cast<int64_t>(I) * N >= 0x7fffffffLL)
+    return fail(XS_ERR_UNSUPPORTED, "I*N must be < 2^31");
+  std::vector<int32_t> num(XSGEN_N_MATS), mats(static_cast<size_t>(XSGEN_N_MATS) * mx);
+  std::vector<double> concs(static_cast<size_t>(XSGEN_N_MATS) * mx);
+  if (xsgen_num_nucs(I, spec->material_rule, num.data()) ||
+      xsgen_mats(I, spec->material_rule, mx, mats.data()) ||
+      xsgen_concs(spec->conc_seed, num.data(), mx, concs.data()))
+    return fail(XS_ERR_INVALID_ARG, "material generation failed");
+  std::unique_ptr<double[]> grid(new (std::nothrow) double[static_cast<size_t>(I) * N * 6]);
+  if (!grid) return fail(XS_ERR_OUT_OF_MEMORY, "host grid buffer");
+  const int ge = xsgen_nuclide_grid(I, N, spec->grid_seed, grid.get(), 0);
+  if (ge == XSGEN_ERR_DUP_ENERGY)
+    return fail(XS_ERR_DATA, "generated grid has a duplicate energy within a nuclide (seed)");
+  if (ge) return fail(XS_ERR_INVALID_ARG, "grid generation failed");
+  xs_grid_data d{};
+  d.abi_version = XS_ABI_VERSION;
+  d.n_isotopes = I;
+  d.n_gridpoints = N;
+  d.nuclide_grid = grid.get();
+  d.n_mats = XSGEN_N_MATS;
+  d.max_num_nucs = mx;
+  d.num_nucs = num.data();
+  d.mats = mats.data();
+  d.concs = concs.data();
+  d.grid_type = spec->grid_type;
+  d.hash_bins = spec->hash_bins;
+  d.lookup_seed = spec->lookup_seed;
+  return init_common(&d, device, static_cast<cudaStream_t>(cuda_stream), out);
+}
+
+xs_status xs_init_grid_data(const xs_grid_data* data, int device, void* cuda_stream,
+                            xs_grid** out) {
+  if (!data || !out) return fail(XS_ERR_INVALID_ARG, "NULL data/out");
+  *out = nullptr;
+  if (data->abi_version != XS_ABI_VERSION) return fail(XS_ERR_INVALID_ARG, "abi_version mismatch");
+  return init_common(data, device, static_cast<cudaStream_t>(cuda_stream), out);
+}
+
+xs_status xs_grid_get_info(const xs_grid* g, xs_grid_info* info) {
+  if (!g || !info) return fail(XS_ERR_INVALID_ARG, "NULL grid/info");
+  const DeviceGrid& G = g->d;
+  info->n_isotopes = G.I;
+  info->n_mats = G.n_mats;
+  info->max_num_nucs = G.max_nucs;
+  info->grid_type = G.grid_type;
+  info->hash_bins = G.B;
+  info->device = G.device;
+  info->n_gridpoints = G.N;
+  info->n_union = G.NU;
+  info->index_grid_len = G.index_len;
+  info->device_bytes = G.device_bytes;
+  info->lookup_seed = G.lookup_seed;
+  return XS_OK;
+}
+
+xs_status xs_workspace_size(const xs_grid* g, uint64_t count, uint32_t flags, size_t* bytes) {
+  if (!g || !bytes) return fail(XS_ERR_INVALID_ARG, "NULL grid/bytes");
+  if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
+  *bytes = total_workspace(count, flags);
+  return XS_OK;
+}
+
+static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* energy,
+                               const int32_t* mat, uint64_t count, uint32_t flags,
+                               const xs_outputs* out, void* workspace, size_t ws_bytes,
+                               void* cuda_stream) {
+  if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
+  if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
+  if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
+  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE))
+    return fail(XS_ERR_INVALID_ARG, "unknown flag bits");
+  if (count == 0) return XS_OK;
+  const size_t need = total_workspace(count, flags);
+  if (!workspace || ws_bytes < need)
+    return fail(XS_ERR_INVALID_ARG, "workspace too small: need " + std::to_string(need) + " bytes");
+  if (reinterpret_cast<uintptr_t>(workspace) & 255)
+    return fail(XS_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
+  DeviceGuard guard(g->d.device);
+  if (!guard.ok) return fail(XS_ERR_CUDA, "cudaSetDevice failed");
+  cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+  Workspace ws;
+  const size_t wbytes = workspace_layout(count, flags, workspace, &ws);
+  LookupArgs a;
+  a.first_id = first_id;
+  a.count = static_cast<uint32_t>(count);
+  a.flags = flags;
+  a.in_energy = energy;
+  a.in_mat = mat;
+  a.out = *out;
+  a.launches = &g->d.launches;
+  if (g->timing) {
+    if (g->ev_used == g->ev.size()) {
+      std::array<cudaEvent_t, 4> evs{};
+      for (auto& x : evs) XS_TRY(cudaEventCreate(&x), "cudaEventCreate");
+      g->ev.push_back(evs);
+    }
+    a.ev = g->ev[g->ev_used++].data();
+  }
+  ++g->calls;
+  Staging sg{};
+  const bool host_io = flags & XS_FLAG_HOST_IO;
+  if (host_io) {
+    staging_layout(count, static_cast<char*>(workspace) + wbytes, &sg);
+    if (energy) {
+      XS_TRY(cudaMemcpyAsync(sg.energy, energy, count * 8, cudaMemcpyHostToDevice, st), "H2D energy");
+      XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * 4, cudaMemcpyHostToDevice, st), "H2D mat");
+      a.in_energy = sg.energy;
+      a.in_mat = sg.mat;
+    }
+    XS_TRY(cudaMemcpyAsync(sg.vsum, out->vsum, 16, cudaMemcpyHostToDevice, st), "H2D vsum");
+    a.out.vsum = sg.vsum;
+    a.out.macro_xs = out->macro_xs ? sg.M : nullptr;
+    a.out.energy = out->energy ? sg.E : nullptr;
+    a.out.mat = out->mat ? sg.omat : nullptr;
+    a.out.grid_index = out->grid_index ? sg.gidx : nullptr;
+    a.out.verification = out->verification ? sg.v : nullptr;
+  }
+  cudaError_t e = run_lookup(g->d, a, ws, st);
+  if (e != cudaSuccess) return fail(XS_ERR_CUDA, "lookup launch", e);
+  if (host_io) {
+    struct {
+      void* dst;
+      const void* src;
+      size_t n;
+    } cp[] = {{out->macro_xs, sg.M, count * 40}, {out->energy, sg.E, count * 8},
+              {out->mat, sg.omat, count * 4},    {out->grid_index, sg.gidx, count * 8},
+              {out->verification, sg.v, count * 4}, {out->vsum, sg.vsum, 16}};
+    for (auto& c : cp)
+      if (c.dst) XS_TRY(cudaMemcpyAsync(c.dst, c.src, c.n, cudaMemcpyDeviceToHost, st), "D2H output");
+    XS_TRY(cudaStreamSynchronize(st), "lookup (host io) completion");
+  }
+  return XS_OK;
+}
+
+xs_status xs_lookup_batch(xs_grid* g, uint64_t first_id, uint64_t count, uint32_t flags,
+                          const xs_outputs* out, void* workspace, size_t workspace_bytes,
+                          void* cuda_stream) {
+  if (g && g->d.n_mats != XSGEN_N_MATS)
+    return fail(XS_ERR_UNSUPPORTED, "sampled batches need the 12 XSBench materials");
+  return lookup_common(g, first_id, nullptr, nullptr, count, flags, out, workspace,
+                       workspace_bytes, cuda_stream);
+}
+
+xs_status xs_lookup_explicit(xs_grid* g, const double* energy, const int32_t* mat, uint64_t count,
+                             uint32_t flags, const xs_outputs* out, void* workspace,
+                             size_t workspace_bytes, void* cuda_stream) {
+  if (count && (!energy || !mat)) return fail(XS_ERR_INVALID_ARG, "NULL energy/mat");
+  return lookup_common(g, 0, energy, mat, count, flags, out, workspace, workspace_bytes,
+                       cuda_stream);
+}
+
+xs_status xs_verify(const xs_grid* g, const double* macro_xs, uint64_t count, uint64_t* vsum,
+                    void* cuda_stream) {
+  if (!g || !vsum || (count && !macro_xs)) return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  if (count == 0) return XS_OK;
+  DeviceGuard guard(g->d.device);
+  cudaError_t e = run_verify(g->d, macro_xs, count, vsum, static_cast<cudaStream_t>(cuda_stream));
+  if (e != cudaSuccess) return fail(XS_ERR_CUDA, "verify launch", e);
+  return XS_OK;
+}
+
+xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t* nuclide,
+                           uint64_t count, int32_t* k_out, void* cuda_stream) {
+  if (!g || (count && (!energy || !nuclide || !k_out)))
+    return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  if (count == 0) return XS_OK;
+  DeviceGuard guard(g->d.device);
+  cudaError_t e = run_nuclide_index(g->d, energy, nuclide, count, k_out,
+                                    static_cast<cudaStream_t>(cuda_stream));
+  if (e != cudaSuccess) return fail(XS_ERR_CUDA, "nuclide_index launch", e);
+  return XS_OK;
+}
+
+xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
+                       void* host_dst) {
+  if (!g || (count && !host_dst)) return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  const DeviceGrid& G = g->d;
+  const void* src = nullptr;
+  uint64_t len = 0;
+  size_t es = 8;
+  switch (table) {
+    case XS_TABLE_NUCLIDE_GRID: src = G.grid; len = static_cast<uint64_t>(G.I) * G.N * 6; break;
+    case XS_TABLE_UNION_ENERGY: src = G.U; len = G.NU; break;
+    case XS_TABLE_INDEX_GRID: src = G.index; len = G.index_len; es = 4; break;
+    case XS_TABLE_NUM_NUCS: src = G.num_nucs; len = G.n_mats; es = 4; break;
+    case XS_TABLE_MATS: src = G.mats; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; es = 4; break;
+    case XS_TABLE_CONCS: src = G.concs; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; break;
+    default: return fail(XS_ERR_INVALID_ARG, "unknown table id");
+  }
+  if (offset > len || count > len - offset) return fail(XS_ERR_INVALID_ARG, "table range out of bounds");
+  if (count == 0) return XS_OK;
+  DeviceGuard guard(G.device);
+  XS_TRY(cudaMemcpy(host_dst, static_cast<const char*>(src) + offset * es, count * es,
+                    cudaMemcpyDeviceToHost),
+         "table copy");
+  return XS_OK;
+}
+
+xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
+  if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  DeviceGrid& G = g->d;
+  if (!std::strcmp(name, "unroll")) {
+    if (value != 3 && value != 6 && value != 9) return fail(XS_ERR_INVALID_ARG, "unroll in {3,6,9}");
+    G.unroll = static_cast<int>(value);
+  } else if (!std::strcmp(name, "blocks_per_sm")) {
+    if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");
+    G.blocks_per_sm = static_cast<int>(value);
+  } else {
+    return fail(XS_ERR_INVALID_ARG, std::string("unknown parameter ") + name);
+  }
+  return XS_OK;
+}
+
+xs_status xs_timing_enable(xs_grid* g, int enable) {
+  if (!g) return fail(XS_ERR_INVALID_ARG, "NULL grid");
+  g->timing = enable != 0;
+  g->ev_used = 0;
+  g->calls = 0;
+  g->launches_read = g->d.launches;
+  return XS_OK;
+}
+
+xs_status xs_timing_read(xs_grid* g, xs_timing* out) {
+  if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  DeviceGuard guard(g->d.device);
+  std::memset(out, 0, sizeof(*out));
+  out->calls = g->calls;
+  out->kernel_launches = g->d.launches - g->launches_read;
+  for (size_t i = 0; i < g->ev_used; ++i) {
+    auto& e = g->ev[i];
+    XS_TRY(cudaEventSynchronize(e[3]), "cudaEventSynchronize");
+    float t[3];
+    XS_TRY(cudaEventElapsedTime(&t[0], e[0], e[1]), "cudaEventElapsedTime");
+    XS_TRY(cudaEventElapsedTime(&t[1], e[1], e[2]), "cudaEventElapsedTime");
+    XS_TRY(cudaEventElapsedTime(&t[2], e[2], e[3]), "cudaEventElapsedTime");
+    out->ms_prepare += t[0];
+    out->ms_sort += t[1];
+    out->ms_gather += t[2];
+  }
+  out->ms_total = out->ms_prepare + out->ms_sort + out->ms_gather;
+  g->ev_used = 0;
+  g->calls = 0;
+  g->launches_read = g->d.launches;
+  return XS_OK;
+}
+
+void xs_free_grid(xs_grid* g) {
+  if (!g) return;
+  DeviceGuard guard(g->d.device);
+  for (auto& e : g->ev)
+    for (auto x : e) cudaEventDestroy(x);
+  cudaFree(g->d.grid);
+  cudaFree(g->d.U);
+  cudaFree(g->d.index);
+  cudaFree(g->d.num_nucs);
+  cudaFree(g->d.mats);
+  cudaFree(g->d.concs);
+  delete g;
+}
+
+}  // extern "C"

@@ -1,0 +1,86 @@
+// xs_internal.h — internal (C++) interface between the C-ABI layer
+// (xs_api.cu) and the kernels (grid_build.cu, lookup.cu).  Not installed.
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include "../../include/xs.h"
+
+namespace xs {
+
+// one lookup after A1/A3: energy, position in the batch, grid index (u or b)
+struct alignas(16) LookupRec {
+  double p;
+  uint32_t idx;
+  int32_t gidx;
+};
+
+constexpr int kMaxMats = 64;  // materials supported by the bucketed kernels
+
+struct DeviceGrid {
+  int device = 0;
+  int sm_count = 0;
+  int32_t I = 0;
+  int64_t N = 0;
+  int32_t n_mats = 0, max_nucs = 0;
+  int32_t grid_type = 0, B = 0;
+  double du = 0.0;
+  uint64_t lookup_seed = 0;
+  int64_t NU = 0, index_len = 0;
+  double* grid = nullptr;    // [I][N][6]
+  double* U = nullptr;       // [NU]
+  int32_t* index = nullptr;  // IG [NU][I] or HG [B][I]
+  int32_t* num_nucs = nullptr;
+  int32_t* mats = nullptr;   // [n_mats][max_nucs]
+  double* concs = nullptr;   // [n_mats][max_nucs]
+  uint64_t device_bytes = 0;
+  // tuning
+  int group_lanes = 3;
+  int unroll = 6;          // nuclides per round per group
+  int blocks_per_sm = 0;   // 0 = occupancy calculator
+  // instrumentation (host side)
+  uint64_t launches = 0;   // kernels launched by lookup calls
+};
+
+// Per-call parameters of the lookup pipeline.
+struct LookupArgs {
+  uint64_t first_id = 0;
+  uint32_t count = 0;
+  uint32_t flags = 0;
+  const double* in_energy = nullptr;  // explicit mode (device)
+  const int32_t* in_mat = nullptr;
+  xs_outputs out{};                    // device pointers
+  cudaEvent_t* ev = nullptr;           // [4] phase events (optional)
+  uint64_t* launches = nullptr;        // incremented per kernel launch
+};
+
+// workspace layout for a batch
+struct Workspace {
+  uint32_t* counts;   // [kMaxMats + 1]
+  uint32_t* cursor;   // [kMaxMats + 1]
+  LookupRec* recs;    // [count]
+  uint32_t* keys0;    // sort
+  uint32_t* keys1;
+  uint32_t* vals0;
+  uint32_t* vals1;
+  void* sort_work;
+  size_t total;
+};
+size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws);
+
+// grid_build.cu
+cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st);
+cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st);
+cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st);
+cudaError_t init_constants();
+
+// lookup.cu
+cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
+                       cudaStream_t st);
+cudaError_t run_verify(const DeviceGrid& g, const double* M, uint64_t count, uint64_t* vsum,
+                       cudaStream_t st);
+cudaError_t run_nuclide_index(const DeviceGrid& g, const double* energy, const int32_t* nuc,
+                              uint64_t count, int32_t* k_out, cudaStream_t st);
+
+}  // namespace xs

@@ -1,0 +1,344 @@
+"""GPU parity: the CUDA path (through the C-ABI, libxs.so) against the CPU
+oracle, element by element on the same seeded inputs.
+
+Bars (BASELINE.json north_star):
+  * energy p, material, grid index u/b, bracket k, verification v and the
+    hash: bit-exact;
+  * macro XS M_c: the kernels accumulate in the oracle's order with no FMA,
+    so they are required bit-exact here too (stronger than the 1e-12
+    relative bound the north_star allows).
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+NT = max(1, min(16, os.cpu_count() or 1))
+CONC_SEED = 1070 * 1070
+
+with open(os.path.join(HERE, "golden", "oracle_hashes.json")) as f:
+    GOLDEN = json.load(f)
+
+
+@pytest.fixture(scope="module")
+def X():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_tianscd23_b200.xs as xs
+    return xs
+
+
+_ORACLES = {}
+
+
+def oracle_for(name, hash_bins=0):
+    key = (name, hash_bins)
+    if key not in _ORACLES:
+        g = GOLDEN[name]
+        _ORACLES[key] = oracle.Oracle.from_spec(g["n_isotopes"], g["n_gridpoints"],
+                                                conc_seed=CONC_SEED,
+                                                material_rule=g["material_rule"],
+                                                hash_bins=hash_bins, nthreads=NT)
+    return _ORACLES[key]
+
+
+def _full_outputs(grid, first, count, **kw):
+    want = ("macro_xs", "energy", "mat", "grid_index", "verification")
+    vsum, res = grid.lookup(first, count, want=want, **kw)
+    torch.cuda.synchronize()
+    out = {k: v.cpu().numpy() for k, v in res.items()}
+    return [int(x) for x in vsum.cpu()], out
+
+
+def _compare(out, ref, mode_index=True):
+    assert np.array_equal(out["energy"], ref["p"])
+    assert np.array_equal(out["mat"], ref["mat"])
+    if mode_index:
+        assert np.array_equal(out["grid_index"], ref["grid_index"])
+    bad = np.nonzero(~np.all(out["macro_xs"] == ref["M"], axis=1))[0]
+    assert bad.size == 0, (bad[:10], out["macro_xs"][bad[:3]], ref["M"][bad[:3]])
+    assert np.array_equal(out["verification"], ref["v"])
+
+
+# ------------------------------------------------------------------- tiny --
+@pytest.mark.parametrize("variant", ["default", "sort", "baseline", "unroll3", "unroll9"])
+def test_tiny_full_parity(X, variant):
+    g = X.Grid.from_preset("tiny")
+    kw = {}
+    if variant == "sort":
+        kw["sort"] = True
+    if variant == "baseline":
+        kw["baseline"] = True
+    if variant.startswith("unroll"):
+        g.set_param("unroll", int(variant[-1]))
+    S, ref = oracle_for("tiny").run(0, 100_000, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
+    vs, out = _full_outputs(g, 0, 100_000, **kw)
+    _compare(out, ref)
+    assert vs == [S, 100_000]
+    assert X.hash_of(vs) == GOLDEN["tiny"]["hash"]
+
+
+@pytest.mark.parametrize("grid_type,bins", [("hash", 97), ("hash", 8192), ("nuclide", 0)])
+@pytest.mark.parametrize("sort", [False, True])
+def test_tiny_other_grids(X, grid_type, bins, sort):
+    g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
+    mode = oracle.HASH if grid_type == "hash" else oracle.NUCLIDE
+    o = oracle_for("tiny", hash_bins=bins)
+    S, ref = o.run(0, 100_000, mode=mode, nthreads=NT, outputs=True)
+    vs, out = _full_outputs(g, 0, 100_000, sort=sort)
+    _compare(out, ref)
+    assert vs == [S, 100_000]
+
+
+@pytest.mark.parametrize("first,count", [(0, 1), (5, 7), (123, 31), (999_999, 1001),
+                                         (2**31 + 5, 333), (7, 4097), (0, 65_537)])
+def test_ragged_batches(X, first, count):
+    g = X.Grid.from_preset("tiny")
+    S, ref = oracle_for("tiny").run(first, count, mode=oracle.UNIONIZED, nthreads=NT,
+                                    outputs=True)
+    for sort in (False, True):
+        vs, out = _full_outputs(g, first, count, sort=sort)
+        _compare(out, ref)
+        assert vs == [S, count]
+
+
+def test_empty_batch_and_accumulation(X):
+    g = X.Grid.from_preset("tiny")
+    vsum = torch.tensor([5, 6], dtype=torch.int64, device="cuda")
+    g.lookup(0, 0, vsum=vsum)
+    g.lookup(0, 1000, vsum=vsum)
+    g.lookup(1000, 1000, vsum=vsum)
+    torch.cuda.synchronize()
+    S = oracle_for("tiny").run(0, 2000, nthreads=NT)
+    assert vsum.cpu().tolist() == [S + 5, 2006]
+
+
+def test_tables_tiny(X):
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    assert np.array_equal(g.table(X.XS_TABLE_NUCLIDE_GRID), o.grid().ravel())
+    U = g.table(X.XS_TABLE_UNION_ENERGY)
+    assert np.array_equal(U, o.union())
+    IG = g.table(X.XS_TABLE_INDEX_GRID).reshape(o.NU, o.I)
+    assert np.array_equal(IG, o.index_grid_sweep())
+    assert np.array_equal(g.table(X.XS_TABLE_MATS).reshape(12, -1), o.mats())
+    assert np.array_equal(g.table(X.XS_TABLE_CONCS).reshape(12, -1), o.concs())
+    assert np.array_equal(g.table(X.XS_TABLE_NUM_NUCS), o.num_nucs())
+    gh = X.Grid.from_preset("tiny", grid_type="hash", hash_bins=257)
+    oh = oracle_for("tiny", hash_bins=257)
+    HG = gh.table(X.XS_TABLE_INDEX_GRID).reshape(257, 12)
+    ref = np.array([[oh.hash_entry(b, n) for n in range(12)] for b in range(257)])
+    assert np.array_equal(HG, ref)
+
+
+@pytest.mark.parametrize("grid_type,bins", [("unionized", 0), ("hash", 64), ("nuclide", 0)])
+def test_nuclide_index_edges(X, grid_type, bins):
+    g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
+    o = oracle_for("tiny", hash_bins=bins)
+    grid = o.grid()
+    E = grid[:, :, 0].ravel()
+    rng = np.random.default_rng(5)
+    probes = np.concatenate([[0.0, 1.0, np.nextafter(1.0, 0), 1e-300], E, np.nextafter(E, 0),
+                             np.nextafter(E, 2), np.arange(65) / 64.0, rng.random(5000)])
+    nucs = rng.integers(0, 12, probes.size).astype(np.int32)
+    k = g.nuclide_index(torch.tensor(probes, device="cuda"),
+                        torch.tensor(nucs, device="cuda")).cpu().numpy()
+    ref = np.array([o.nuclide_bracket(int(n), float(p)) for p, n in zip(probes, nucs)])
+    assert np.array_equal(k, ref)
+
+
+# ----------------------------------------------------------- explicit API --
+def test_explicit_lookups(X):
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    rng = np.random.default_rng(11)
+    E = o.grid()[:, :, 0].ravel()
+    p = np.concatenate([rng.random(20000), E[:500], [0.0, 1.0, -0.25, 1.5, 1e-300]])
+    m = rng.integers(0, 12, p.size).astype(np.int32)
+    m[7] = 12          # invalid material
+    m[11] = -1
+    S, M, v = o.run_explicit(np.where((m >= 0) & (m < 12), p, 0.5),
+                             np.clip(m, 0, 11), mode=oracle.UNIONIZED, nthreads=NT)
+    ok = (m >= 0) & (m < 12)
+    for sort in (False, True):
+        vs, res = g.lookup_explicit(torch.tensor(p, device="cuda"), torch.tensor(m, device="cuda"),
+                                    sort=sort, want=("macro_xs", "verification", "mat"))
+        torch.cuda.synchronize()
+        Mg = res["macro_xs"].cpu().numpy()
+        vg = res["verification"].cpu().numpy()
+        assert np.array_equal(Mg[ok], M[ok])
+        assert np.array_equal(vg[ok], v[ok])
+        assert np.all(vg[~ok] == 0) and np.all(np.isnan(Mg[~ok]))
+        assert np.array_equal(res["mat"].cpu().numpy(), m)
+        assert vs.cpu().tolist() == [int(v[ok].sum()), int(ok.sum())]
+    # host buffers (XS_FLAG_HOST_IO): same results, outputs on the host
+    vs, res = g.lookup_explicit(torch.tensor(p), torch.tensor(m), want=("macro_xs",))
+    assert np.array_equal(res["macro_xs"].numpy()[ok], M[ok])
+    assert vs.tolist() == [int(v[ok].sum()), int(ok.sum())]
+
+
+def test_verify_entry_point(X):
+    g = X.Grid.from_preset("tiny")
+    vs, res = g.lookup(0, 5000, want=("macro_xs",))
+    v2 = g.verify(res["macro_xs"])
+    torch.cuda.synchronize()
+    assert vs.cpu().tolist() == v2.cpu().tolist()
+    M = torch.tensor([[0.5, 0.5, 0.1, 0.2, 0.3], [-2.0, -3.0, -1.5, -1.0, -4.0],
+                      [0.0, 0.0, 0.0, 0.0, 0.0], [1.0, 2.0, 3.0, 4.0, 5.0]], device="cuda",
+                     dtype=torch.float64)
+    assert g.verify(M).cpu().tolist() == [1 + 1 + 1 + 5, 4]
+
+
+# --------------------------------------------------- caller-supplied data --
+def test_worked_example_through_gpu(X):
+    with open(os.path.join(HERE, "golden", "worked_two_nuclide.json")) as f:
+        w = json.load(f)
+    grid = np.zeros((2, 3, 6))
+    for i, name in enumerate(("A", "B")):
+        grid[i, :, 0] = w["nuclides"][name]["E"]
+        grid[i, :, 1:] = np.array(w["nuclides"][name]["xs"], np.float64)
+    for gt, bins in (("unionized", 0), ("hash", 4), ("nuclide", 0)):
+        g = X.Grid.from_arrays(grid, [2], [w["material"]["nuclides"]], [w["material"]["concs"]],
+                               grid_type=gt, hash_bins=bins)
+        p = torch.tensor([c["p"] for c in w["cases"]], device="cuda", dtype=torch.float64)
+        m = torch.zeros(len(w["cases"]), dtype=torch.int32, device="cuda")
+        vs, res = g.lookup_explicit(p, m, want=("macro_xs", "verification", "grid_index"))
+        torch.cuda.synchronize()
+        for i, c in enumerate(w["cases"]):
+            assert res["macro_xs"][i].cpu().tolist() == c["M"]
+            assert int(res["verification"][i]) == c["v"]
+            if gt == "unionized":
+                assert int(res["grid_index"][i]) == c["u"]
+
+
+def test_linear_closed_form_at_scale(X):
+    # P7 on the GPU with no oracle: dyadic linear channels are interpolated
+    # exactly, so M_c = sum_j conc_j (alpha_jc p + beta_jc) for dyadic p.
+    rng = np.random.default_rng(2)
+    I, N = 40, 200
+    E = np.array([np.sort(rng.choice(np.arange(1, 4096), N, replace=False)) for _ in range(I)])
+    E = E / 4096.0
+    alpha = rng.integers(-8, 9, (I, 5)) / 8.0
+    beta = rng.integers(-8, 9, (I, 5)) / 4.0
+    grid = np.zeros((I, N, 6))
+    grid[:, :, 0] = E
+    grid[:, :, 1:] = alpha[:, None, :] * E[:, :, None] + beta[:, None, :]
+    mats = np.stack([rng.permutation(I)[:30] for _ in range(3)]).astype(np.int32)
+    concs = rng.integers(1, 16, (3, 30)) / 16.0
+    g = X.Grid.from_arrays(grid, [30, 30, 30], mats, concs)
+    p = rng.integers(0, 4097, 200_000) / 4096.0
+    m = rng.integers(0, 3, p.size).astype(np.int32)
+    vs, res = g.lookup_explicit(torch.tensor(p, device="cuda"), torch.tensor(m, device="cuda"),
+                                want=("macro_xs",))
+    got = res["macro_xs"].cpu().numpy()
+    ref = np.zeros((p.size, 5))
+    for j in range(30):
+        n = mats[m, j]
+        ref = ref + concs[m, j][:, None] * (alpha[n] * p[:, None] + beta[n])
+    assert np.array_equal(got, ref)
+
+
+def test_invalid_arguments(X):
+    with pytest.raises(X.XSError) as e:
+        X.Grid.from_spec(n_isotopes=100, n_gridpoints=100, material_rule=0)
+    assert e.value.status == 1
+    with pytest.raises(X.XSError):
+        X.Grid.from_spec(n_isotopes=12, n_gridpoints=1, material_rule=1)
+    g = X.Grid.from_preset("tiny")
+    vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+    o = X.xs_outputs(None, None, None, None, None, vsum.data_ptr())
+    with pytest.raises(X.XSError):  # workspace too small
+        X.xs_lookup_batch(g._h, 0, 1000, 0, o, g.workspace(10).data_ptr(), 16,
+                          torch.cuda.current_stream().cuda_stream)
+    with pytest.raises(X.XSError):  # unknown flag
+        X.xs_lookup_batch(g._h, 0, 10, 0x80, o, g.workspace(10).data_ptr(), 1 << 20,
+                          torch.cuda.current_stream().cuda_stream)
+    bad = np.zeros((1, 3, 6))
+    bad[0, :, 0] = [0.1, 0.1, 0.2]   # duplicate energy
+    with pytest.raises(X.XSError) as e:
+        X.Grid.from_arrays(bad, [1], [[0]], [[1.0]])
+    assert e.value.status == 6
+
+
+# ------------------------------------------------------ full-size configs --
+def _sample_ids(L, k=3000, seed=0):
+    rng = np.random.default_rng(seed)
+    ids = np.concatenate([[0, 1, L - 1, L // 2], rng.integers(0, L, k)])
+    return np.unique(ids)
+
+
+@pytest.mark.parametrize("name", ["small", "large", "large-hash", "xl"])
+def test_full_config_hash_and_samples(X, name):
+    gold = GOLDEN[name]
+    if name == "xl":
+        free, _ = torch.cuda.mem_get_info()
+        if free < 140e9:
+            pytest.skip("XL needs ~130 GB of device memory")
+    g = X.Grid.from_preset(name)
+    pre = X.PRESETS[name]
+    L = pre["lookups"]
+    sort = pre.get("sort", False)
+    # the launch configuration bench.py times: one batch of all L lookups
+    if L <= 20_000_000:
+        want = ("energy", "mat", "grid_index", "verification")
+        vs, res = g.lookup(0, L, sort=sort, want=want)
+        torch.cuda.synchronize()
+        assert [int(x) for x in vs.cpu()] == [gold["sum_v"], L]
+        ids = _sample_ids(L)
+        o = oracle_for(name, hash_bins=pre.get("hash_bins", 0))
+        mode = oracle.HASH if pre["grid_type"] == "hash" else oracle.UNIONIZED
+        ids_t = torch.tensor(ids, device="cuda")
+        E = res["energy"][ids_t].cpu().numpy()
+        mt = res["mat"][ids_t].cpu().numpy()
+        gi = res["grid_index"][ids_t].cpu().numpy()
+        v = res["verification"][ids_t].cpu().numpy()
+        # macro XS for the sampled ids through the explicit entry point
+        _, rex = g.lookup_explicit(torch.tensor(E, device="cuda"), torch.tensor(mt, device="cuda"),
+                                   want=("macro_xs",))
+        Mx = rex["macro_xs"].cpu().numpy()
+        for j, i in enumerate(ids):
+            r = o.lookup(int(i), mode)
+            assert (E[j], mt[j], gi[j], v[j]) == (r["p"], r["mat"], r["grid_index"], r["v"]), i
+            assert np.array_equal(Mx[j], r["M"]), i
+    else:
+        # XL: 170M lookups in 10 shards of 17M (the bench's per-GPU batch size)
+        vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+        step = 17_000_000
+        for first in range(0, L, step):
+            g.lookup(first, min(step, L - first), vsum=vsum)
+        torch.cuda.synchronize()
+        assert [int(x) for x in vsum.cpu()] == [gold["sum_v"], L]
+        ids = _sample_ids(L, k=400)
+        o = oracle_for("xl", hash_bins=131072)
+        for i in ids:
+            i = int(i)
+            vs, res = g.lookup(i, 1, want=("energy", "mat", "grid_index", "macro_xs",
+                                           "verification"))
+            r = o.lookup(i, oracle.HASH)
+            assert float(res["energy"][0]) == r["p"] and int(res["mat"][0]) == r["mat"]
+            assert int(res["grid_index"][0]) == o.union_index(r["p"])
+            assert res["macro_xs"][0].cpu().tolist() == r["M"].tolist()
+            assert int(res["verification"][0]) == r["v"]
+    assert X.hash_of([gold["sum_v"]]) == gold["hash"]
+
+
+def test_shard_invariance_small(X):
+    # P10: sum over contiguous shards == one batch, for R in {1,2,3,4,7,8}
+    g = X.Grid.from_preset("small")
+    L = 17_000_000
+    sums = []
+    for R in (1, 2, 3, 4, 7, 8):
+        vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+        for r in range(R):
+            a, b = r * L // R, (r + 1) * L // R
+            g.lookup(a, b - a, vsum=vsum, sort=(R % 2 == 0))
+        torch.cuda.synchronize()
+        sums.append(vsum.cpu().tolist())
+    assert all(s == [GOLDEN["small"]["sum_v"], L] for s in sums)
