@@ -191,8 +191,9 @@ xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t
 xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
                        void* host_dst);
 
-/* Tuning knobs: "unroll" (nuclides per round per lookup group: 3, 6 or 9)
- * and "blocks_per_sm" (0 = occupancy calculator).  INVALID_ARG for an
+/* Tuning knobs: "variant" (gather kernel shape: 0 = default, 1-4 = (nuclides
+ * per round, min resident blocks) in {(3,3), (3,4), (6,2), (6,3)}) and
+ * "blocks_per_sm" (0 = occupancy calculator).  INVALID_ARG for an
  * unknown name or value.  Never changes results. */
 xs_status xs_set_param(xs_grid* g, const char* name, int64_t value);
 

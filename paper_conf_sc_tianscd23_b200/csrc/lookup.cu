@@ -20,6 +20,7 @@
 //               to the serial definition.
 //   verification: v = 1 + argmax; per-block reduction, one atomic per block.
 #include <cfloat>
+#include <type_traits>
 
 #include "common.cuh"
 #include "radix_sort.cuh"
@@ -255,9 +256,57 @@ struct GatherSmem {
   uint32_t toff[kMaxMats + 1];  // first task of material m
 };
 
-// U = nuclides per round per group (multiple of kG)
-template <int GT, bool SORTED, int U>
-__global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
+// Per-lookup view of the acceleration structure for A4: the unionized index
+// row IG[u], or the two hash rows HG[b], HG[b+1].
+template <int GT>
+struct RowView {
+  const int32_t* r0;
+  const int32_t* r1;
+  __device__ __forceinline__ RowView(const Params& P, int32_t gidx) {
+    if (GT == XS_GRID_UNIONIZED) {
+      r0 = P.index + static_cast<int64_t>(gidx) * P.I;
+      r1 = r0;
+    } else if (GT == XS_GRID_HASH) {
+      r0 = P.index + static_cast<int64_t>(gidx) * P.I;
+      r1 = gidx == P.B - 1 ? nullptr : r0 + P.I;
+    } else {
+      r0 = r1 = nullptr;
+    }
+  }
+  // bracket k_n(p) of nuclide n whose records start at record index noff
+  __device__ __forceinline__ int32_t bracket(const Params& P, int32_t n, uint32_t noff,
+                                             double p) const {
+    if (GT == XS_GRID_UNIONIZED) return __ldg(r0 + n);
+    const double* rec = P.grid + static_cast<uint64_t>(noff) * 6;
+    if (GT == XS_GRID_NUCLIDE) return nuclide_bracket(rec, P.N, p);
+    const int64_t N = P.N;
+    const int64_t u_lo = __ldg(r0 + n);
+    const int64_t u_hi = r1 ? static_cast<int64_t>(__ldg(r1 + n)) + 1 : N - 1;
+    int64_t lower;
+    if (p <= rec_energy(rec, u_lo))
+      lower = u_lo;
+    else if (p >= rec_energy(rec, u_hi))
+      lower = N - 1;
+    else
+      lower = bracket_search_rec(rec, u_lo, u_hi, p);
+    return static_cast<int32_t>(lower == N - 1 ? N - 2 : lower);
+  }
+};
+
+// U = nuclides per round per group (multiple of kG).
+//
+// Control flow is warp-uniform by construction (all 10 groups of a warp
+// serve the same material, so they walk the same nuclide list); lanes that
+// have no lookup (tail of a bucket, lanes 30-31) run the same instructions
+// with their loads predicated off.  Every shuffle is executed by all 32
+// lanes, outside any branch, and the interpolation weight is computed by
+// every lane from its own chunk (only lane r = 0's value, from the energy
+// chunk, is used) so the U divisions of a round are independent and
+// branch-free.  Record addresses are 32-bit record indices (I*N < 2^31,
+// checked at init) scaled once: n*N is precomputed per material slot in
+// shared memory.
+template <int GT, bool SORTED, int U, int MINB, bool CHECK>
+__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
   static_assert(U % kG == 0, "U must be a multiple of the group size");
   constexpr int Q = U / kG;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -265,9 +314,12 @@ __global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
   const int tab = P.n_mats * P.max_nucs;
   double* s_concs = reinterpret_cast<double*>(smem_raw + sizeof(GatherSmem));
   int32_t* s_mats = reinterpret_cast<int32_t*>(s_concs + tab);
+  uint32_t* s_noff = reinterpret_cast<uint32_t*>(s_mats + tab);
   for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
     s_concs[t] = P.concs[t];
-    s_mats[t] = P.mats[t];
+    s_mats[t] = n;
+    s_noff[t] = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
   }
   if (threadIdx.x == 0) {
     uint32_t run = 0, trun = 0;
@@ -293,7 +345,7 @@ __global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
   const uint32_t warps_per_block = blockDim.x >> 5;
   const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
   const uint32_t nw = gridDim.x * warps_per_block;
-  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid) + r;
 
   unsigned long long acc_v = 0, acc_n = 0;
   int m = 0;
@@ -308,18 +360,25 @@ __global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
       rec = P.recs[pos];
     }
     const double p = rec.p;
-    const int nn = S.num[m];
+    const int nn = valid ? S.num[m] : 0;   // invalid lanes load nothing
+    const int nw_loop = S.num[m];           // warp-uniform trip count
     const int32_t* mrow = s_mats + m * P.max_nucs;
+    const uint32_t* orow = s_noff + m * P.max_nucs;
     const double* crow = s_concs + m * P.max_nucs;
+    const RowView<GT> rv(P, valid ? rec.gidx : 0);
 
     double acc_a = 0.0, acc_b = 0.0;
     int32_t knext[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       const int j = r + q * kG;
-      knext[q] = (valid && j < nn) ? bracket_of<GT>(P, rec.gidx, mrow[j], p) : 0;
+      knext[q] = j < nn ? rv.bracket(P, mrow[j], orow[j], p) : 0;
     }
-    for (int j0 = 0; j0 < nn; j0 += U) {
+    // One round = U consecutive nuclides of the list.  Full rounds run
+    // without any per-nuclide predicate; the (at most one) partial round at
+    // the end of the list runs the TAIL instantiation.
+    auto round = [&](const int j0, auto tail_tag) {
+      constexpr bool TAIL = decltype(tail_tag)::value;
       int32_t kcur[Q];
 #pragma unroll
       for (int q = 0; q < Q; ++q) kcur[q] = knext[q];
@@ -327,39 +386,55 @@ __global__ void __launch_bounds__(kGatherThreads) k_gather(Params P) {
 #pragma unroll
       for (int q = 0; q < Q; ++q) {
         const int j = j0 + U + r + q * kG;
-        knext[q] = (valid && j < nn) ? bracket_of<GT>(P, rec.gidx, mrow[j], p) : 0;
+        knext[q] = j < nn ? rv.bracket(P, mrow[j], orow[j], p) : 0;
       }
-      // A5: 96-B record pairs, lane r loads chunk r of the low and high record
+      // A5: 96-B record pairs; lane r loads chunk r of the low and high
+      // record.  (Past the end of the list, or without a lookup, a lane
+      // reads the grid's first record pair instead: always valid memory,
+      // the value is never accumulated.)
       double2 lo[U], hi[U];
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + t;
         const int32_t kt = __shfl_sync(0xffffffffu, kcur[t / kG], base + (t % kG));
-        lo[t] = make_double2(0.0, 0.0);
-        hi[t] = make_double2(1.0, 0.0);
-        if (valid && j < nn) {
-          const int32_t n = mrow[j];
-          const double2* pr = grid2 + (static_cast<int64_t>(n) * P.N + kt) * 3;
-          lo[t] = __ldg(pr + r);
-          hi[t] = __ldg(pr + 3 + r);
-        }
+        uint32_t off = orow[j] + static_cast<uint32_t>(kt);
+        if (TAIL || !valid) off = j < nn ? off : 0u;
+        const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
+        lo[t] = __ldg(pr);
+        hi[t] = __ldg(pr + 3);
+      }
+      // A6: f = (hi.E - p) / (hi.E - lo.E), correctly rounded, every lane
+      // (lane r = 0 holds the energies; the other lanes' values are unused)
+      double fl[U];
+      bool fast = true;
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const double an = dsub(hi[t].x, p), bd = dsub(hi[t].x, lo[t].x);
+        fl[t] = div_nr(an, bd);
+        if (CHECK) fast &= (r != 0) || div_in_range(an, bd);
+      }
+      if (CHECK && !__all_sync(0xffffffffu, fast)) {  // rare: extreme data
+#pragma unroll
+        for (int t = 0; t < U; ++t)
+          if (r == 0) fl[t] = ddiv(dsub(hi[t].x, p), dsub(hi[t].x, lo[t].x));
       }
       // A6 + A7 in list order
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + t;
-        if (j < nn) {  // warp-uniform
-          double f = 0.0;
-          if (r == 0) f = ddiv(dsub(hi[t].x, p), dsub(hi[t].x, lo[t].x));
-          f = __shfl_sync(0xffffffffu, f, base);
-          const double xa = dsub(hi[t].x, dmul(f, dsub(hi[t].x, lo[t].x)));
-          const double xb = dsub(hi[t].y, dmul(f, dsub(hi[t].y, lo[t].y)));
+        const double f = __shfl_sync(0xffffffffu, fl[t], base);
+        const double xa = dsub(hi[t].x, dmul(f, dsub(hi[t].x, lo[t].x)));
+        const double xb = dsub(hi[t].y, dmul(f, dsub(hi[t].y, lo[t].y)));
+        if (!TAIL || j < nw_loop) {  // warp-uniform
           const double c = crow[j];
           acc_a = dadd(acc_a, dmul(xa, c));
           acc_b = dadd(acc_b, dmul(xb, c));
         }
       }
-    }
+    };
+    int j0 = 0;
+    for (; j0 + U <= nw_loop; j0 += U) round(j0, std::false_type{});
+    if (j0 < nw_loop) round(j0, std::true_type{});
     // A8: channels (t, s, a, f, nf) = (b@r0, a@r1, b@r1, a@r2, b@r2)
     double M[5];
     M[0] = __shfl_sync(0xffffffffu, acc_b, base);
@@ -545,11 +620,11 @@ static unsigned grid_cap(uint64_t work, int threads, int sm, int per_sm) {
   return static_cast<unsigned>(b < cap ? b : cap);
 }
 
-template <int GT, bool SORTED, int U>
+template <int GT, bool SORTED, int U, int MINB, bool CHECK>
 static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  const size_t smem = sizeof(GatherSmem) +
-                      static_cast<size_t>(g.n_mats) * g.max_nucs * (sizeof(double) + sizeof(int32_t));
-  auto kern = k_gather<GT, SORTED, U>;
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs *
+                                               (sizeof(double) + 2 * sizeof(int32_t));
+  auto kern = k_gather<GT, SORTED, U, MINB, CHECK>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -563,13 +638,26 @@ static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStrea
   return cudaGetLastError();
 }
 
+// gather variants: (nuclides per round U, min resident blocks of 256 threads)
+// CHECK: the division fast path is exact without a range check when every
+// energy (grid and lookups) is a multiple of 2^-63 in [0, 1] (DESIGN.md §4:
+// then |hi.E - p| and |hi.E - lo.E| are 0 or >= 2^-63), which holds for
+// generated grids with sampled lookups; otherwise the checked kernel runs.
+template <int GT, bool SORTED, bool CHECK>
+static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  switch (g.unroll) {
+    case 1: return launch_gather<GT, SORTED, 3, 3, CHECK>(g, P, st);
+    case 2: return launch_gather<GT, SORTED, 3, 4, CHECK>(g, P, st);
+    case 4: return launch_gather<GT, SORTED, 6, 3, CHECK>(g, P, st);
+    default: return launch_gather<GT, SORTED, 6, 2, CHECK>(g, P, st);
+  }
+}
+
 template <int GT, bool SORTED>
 static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  switch (g.unroll) {
-    case 3: return launch_gather<GT, SORTED, 3>(g, P, st);
-    case 9: return launch_gather<GT, SORTED, 9>(g, P, st);
-    default: return launch_gather<GT, SORTED, 6>(g, P, st);
-  }
+  const bool check = P.in_energy != nullptr || !g.dyadic63;
+  return check ? launch_gather_v<GT, SORTED, true>(g, P, st)
+               : launch_gather_v<GT, SORTED, false>(g, P, st);
 }
 
 template <int GT>

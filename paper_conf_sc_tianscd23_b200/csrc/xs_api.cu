@@ -168,7 +168,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   if (d->grid_type == XS_GRID_HASH && d->hash_bins < 1)
     return fail(XS_ERR_INVALID_ARG, "hash grid needs hash_bins >= 1");
   const size_t tab = static_cast<size_t>(d->n_mats) * d->max_num_nucs;
-  if (tab * 12 > 160 * 1024)
+  if (tab * 16 > 160 * 1024)
     return fail(XS_ERR_UNSUPPORTED, "material tables exceed the 160 KB shared-memory stage");
   for (int32_t m = 0; m < d->n_mats; ++m) {
     if (d->num_nucs[m] < 0 || d->num_nucs[m] > d->max_num_nucs)
@@ -186,6 +186,14 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
       if (!(E[(k - 1) * 6] < E[k * 6]))
         return fail(XS_ERR_DATA, "nuclide " + std::to_string(n) +
                                      ": energies not strictly increasing");
+  }
+  // energies on the 2^-63 lattice of [0, 1] (all generated grids): lets the
+  // gather kernel skip the division range check for sampled lookups
+  bool dyadic = true;
+  for (int64_t i = 0; i < static_cast<int64_t>(I) * N && dyadic; ++i) {
+    const double e = d->nuclide_grid[i * 6];
+    const double k = e * 0x1p63;  // exact scaling by a power of two
+    dyadic = e >= 0.0 && e <= 1.0 && k == static_cast<double>(static_cast<uint64_t>(k));
   }
   int sm = 0;
   xs_status s = check_device(device, &sm);
@@ -207,6 +215,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   G.B = d->grid_type == XS_GRID_HASH ? d->hash_bins : 0;
   G.du = G.B ? 1.0 / static_cast<double>(G.B) : 0.0;
   G.lookup_seed = d->lookup_seed;
+  G.dyadic63 = dyadic;
   G.NU = d->grid_type == XS_GRID_UNIONIZED ? static_cast<int64_t>(I) * N : 0;
   G.index_len = d->grid_type == XS_GRID_UNIONIZED ? G.NU * I
                 : d->grid_type == XS_GRID_HASH    ? static_cast<int64_t>(G.B) * I
@@ -473,8 +482,8 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
 xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
   DeviceGrid& G = g->d;
-  if (!std::strcmp(name, "unroll")) {
-    if (value != 3 && value != 6 && value != 9) return fail(XS_ERR_INVALID_ARG, "unroll in {3,6,9}");
+  if (!std::strcmp(name, "variant")) {
+    if (value < 0 || value > 4) return fail(XS_ERR_INVALID_ARG, "variant in [0,4]");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "blocks_per_sm")) {
     if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");

@@ -35,9 +35,9 @@ struct DeviceGrid {
   int32_t* mats = nullptr;   // [n_mats][max_nucs]
   double* concs = nullptr;   // [n_mats][max_nucs]
   uint64_t device_bytes = 0;
+  bool dyadic63 = false;     // every grid energy is k * 2^-63 in [0, 1]
   // tuning
-  int group_lanes = 3;
-  int unroll = 6;          // nuclides per round per group
+  int unroll = 0;          // gather variant (0 = default; see launch_gather_u)
   int blocks_per_sm = 0;   // 0 = occupancy calculator
   // instrumentation (host side)
   uint64_t launches = 0;   // kernels launched by lookup calls

@@ -68,7 +68,7 @@ def _compare(out, ref, mode_index=True):
 
 
 # ------------------------------------------------------------------- tiny --
-@pytest.mark.parametrize("variant", ["default", "sort", "baseline", "unroll3", "unroll9"])
+@pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -76,8 +76,8 @@ def test_tiny_full_parity(X, variant):
         kw["sort"] = True
     if variant == "baseline":
         kw["baseline"] = True
-    if variant.startswith("unroll"):
-        g.set_param("unroll", int(variant[-1]))
+    if variant.startswith("v"):
+        g.set_param("variant", int(variant[-1]))
     S, ref = oracle_for("tiny").run(0, 100_000, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
     vs, out = _full_outputs(g, 0, 100_000, **kw)
     _compare(out, ref)

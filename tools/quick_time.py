@@ -18,7 +18,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="large")
     ap.add_argument("--reps", type=int, default=5)
-    ap.add_argument("--variants", default="u6,u3,u9,sort,baseline")
+    ap.add_argument("--variants", default="v1,v2,v3,v4,sort,baseline")
     a = ap.parse_args()
     gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")))
     pre = dict(X.PRESETS[a.config])
@@ -30,13 +30,13 @@ def main():
     L = min(pre["lookups"], 17_000_000)
     for var in a.variants.split(","):
         kw = {}
-        if var.startswith("u"):
-            g.set_param("unroll", int(var[1:]))
+        if var.startswith("v"):
+            g.set_param("variant", int(var[1:]))
         if var == "sort":
             kw["sort"] = True
         if var == "baseline":
             kw["baseline"] = True
-        for bps in ([0] if var != "u6" else [0, 1, 2, 3]):
+        for bps in [0]:
             g.set_param("blocks_per_sm", bps)
             vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
             g.lookup(0, L, vsum=vsum, **kw)
@@ -58,7 +58,7 @@ def main():
             print(f"{var:9s} bps={bps} {ms:8.3f} ms/step  {L / ms / 1e6:8.3f} G lookups/s  "
                   f"prep {t['ms_prepare']/n:.3f} sort {t['ms_sort']/n:.3f} gather {t['ms_gather']/n:.3f}"
                   f"  launches/step {t['kernel_launches']/n:.0f} hash_ok={ok}", flush=True)
-        g.set_param("unroll", 6)
+        g.set_param("variant", 0)
         g.set_param("blocks_per_sm", 0)
 
 
