@@ -127,7 +127,8 @@ typedef struct {
 } xs_outputs;
 
 /* flags */
-#define XS_FLAG_SORT 0x1u     /* A2: radix-sort the batch by (material, energy)  */
+#define XS_FLAG_SORT 0x1u     /* A2: order the batch by (material, energy bin):
+                                 one in-house counting-sort radix pass       */
 #define XS_FLAG_HOST_IO 0x2u  /* inputs/outputs are host pointers               */
 #define XS_FLAG_BASELINE 0x4u /* thread-per-lookup, unbucketed kernel (XSBench's
                                  CUDA baseline shape; for comparison only)     */
@@ -204,8 +205,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value);
 typedef struct {
   uint64_t calls;           /* lookup calls since the last read              */
   uint64_t kernel_launches; /* kernels those calls launched                  */
-  double ms_prepare;        /* A1+A3: material count, sample+search, bucket  */
-  double ms_sort;           /* A2: radix sort (0 without XS_FLAG_SORT)       */
+  double ms_count;          /* A1: material (and energy-bin) histogram       */
+  double ms_bucket;         /* A1+A3 (+A2): sample, search, scatter to bins  */
   double ms_gather;         /* A4-A8: the gather/interpolate/verify kernel   */
   double ms_total;          /* sum of the above                              */
 } xs_timing;

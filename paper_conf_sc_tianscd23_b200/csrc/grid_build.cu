@@ -120,4 +120,32 @@ cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// UB[b] = ub(U, b / UBn) = #{U <= b / UBn}, b = 0..UBn: equal-width energy
+// bins over the unionized grid, so the A3 search for p in bin b only has to
+// run inside [UB[b] - 1, UB[b + 1]] (same result as the full search; DESIGN.md
+// §4 "A3").
+__global__ void k_union_table(const double* __restrict__ U, int64_t NU, int32_t UBn,
+                              int32_t* __restrict__ UB) {
+  const double inv = 1.0 / static_cast<double>(UBn);
+  for (int64_t b = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; b <= UBn;
+       b += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+    const double e = static_cast<double>(b) * inv;
+    int64_t lo = 0, hi = NU;
+    while (lo < hi) {
+      const int64_t mid = lo + ((hi - lo) >> 1);
+      if (U[mid] <= e)
+        lo = mid + 1;
+      else
+        hi = mid;
+    }
+    UB[b] = static_cast<int32_t>(lo);
+  }
+}
+
+cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st) {
+  k_union_table<<<grid_for(static_cast<uint64_t>(g.UBn) + 1, 256, g.sm_count), 256, 0, st>>>(
+      g.U, g.NU, g.UBn, g.UB);
+  return cudaGetLastError();
+}
+
 }  // namespace xs

@@ -5,10 +5,13 @@
 // Pipeline of one xs_lookup_batch call (all on the caller's stream):
 //   k_count     A1: per-material histogram of the batch (materials only)
 //   k_bucket    A1+A3: sample (p, m) again, search p on U (or hash bin),
-//               write a 16-B LookupRec into the material bucket
-//               (unsorted) or in id order plus a (material, energy) key
-//               (sorted; then the in-house radix sort produces the
-//               permutation — A2)
+//               write a 16-B LookupRec into the material bucket.  With
+//               XS_FLAG_SORT (A2) the bucket key is (material, energy bin)
+//               with 4096 energy bins per material: one in-house radix
+//               pass (k_count histogram, k_scan_bins scan, k_bucket
+//               scatter) that leaves each material's lookups ordered by
+//               energy to 2^-12, so the lookups sharing a warp touch the
+//               same record pairs.
 //   k_gather    A4-A8: warp-per-task over material buckets; each group of
 //               G=3 lanes owns one lookup and walks the material's nuclides
 //               in list order; per nuclide the 3 lanes gather the 96-B
@@ -56,6 +59,13 @@ struct Sample {
 };
 
 // lookup id -> (p, mat): s = FF(seed, 2 id); p = draw; roll = draw (R4)
+__device__ __forceinline__ Sample sample_from_state(uint64_t s) {
+  s = lcg_next(s);
+  const double p = lcg_double(s);
+  s = lcg_next(s);
+  return Sample{p, pick_material(lcg_double(s))};
+}
+
 __device__ __forceinline__ Sample sample_lookup(uint64_t seed, uint64_t id) {
   uint64_t s = fast_forward(seed, 2 * id);
   s = lcg_next(s);
@@ -71,6 +81,8 @@ struct Params {
   int64_t N;
   const double* U;
   int64_t NU;
+  const int32_t* UB;
+  int32_t UBn;
   const int32_t* index;
   int32_t B;
   double du;
@@ -87,9 +99,10 @@ struct Params {
   uint32_t* counts;
   uint32_t* cursor;
   LookupRec* recs;
-  uint32_t* keys;
-  uint32_t* vals;
-  const uint32_t* perm;
+  uint32_t* bins;   // [(n_mats + 1) * kEnergyBins] histogram -> cursors (A2)
+  LookupRec* tmp;   // [count] records in batch order
+  uint8_t* mat8;    // [count] material (n_mats = invalid)
+  uint32_t* partials;  // A2 scan: per-chunk sums -> offsets
   // outputs
   double* out_M;
   double* out_E;
@@ -115,45 +128,230 @@ __device__ __forceinline__ int32_t grid_index_of(const Params& P, double p) {
   return -1;
 }
 
-// k_count: histogram of materials over the batch (bucket n_mats = invalid)
-__global__ void __launch_bounds__(256) k_count(Params P) {
-  __shared__ uint32_t s_h[kMaxMats + 1];
-  for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x) s_h[t] = 0;
-  __syncthreads();
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < P.count;
-       i += gridDim.x * blockDim.x) {
-    int32_t m;
-    if (P.in_energy) {
-      m = P.in_mat[i];
-      if (m < 0 || m >= P.n_mats) m = P.n_mats;
-    } else {
-      m = sample_lookup(P.seed, P.first_id + i).mat;
-    }
-    atomicAdd(&s_h[m], 1u);
-  }
-  __syncthreads();
-  for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x)
-    if (s_h[t]) atomicAdd(&P.counts[t], s_h[t]);
+__device__ __forceinline__ uint32_t energy_bin(double p) {
+  const double q = p * static_cast<double>(kEnergyBins);
+  if (!(q > 0.0)) return 0u;
+  return q < static_cast<double>(kEnergyBins - 1) ? static_cast<uint32_t>(q) : kEnergyBins - 1u;
 }
 
-constexpr int kBucketThreads = 256;
-constexpr int kBucketItems = 4;
+constexpr int kPrepThreads = 256;
+constexpr int kPrepItems = 4;  // lookups per thread, searched in lockstep
 
 __device__ __forceinline__ void write_invalid(const Params& P, uint32_t i) {
   if (P.out_M)
-    for (int c = 0; c < 5; ++c) P.out_M[static_cast<uint64_t>(i) * 5 + c] = __longlong_as_double(0x7ff8000000000000LL);
+    for (int c = 0; c < 5; ++c)
+      P.out_M[static_cast<uint64_t>(i) * 5 + c] = __longlong_as_double(0x7ff8000000000000LL);
   if (P.out_v) P.out_v[i] = 0;
 }
 
-// k_bucket: A1 + A3.  SORTED=false: scatter into material buckets with
-// block-aggregated cursors; SORTED=true: records in id order + sort keys.
-template <int GT, bool SORTED>
-__global__ void __launch_bounds__(kBucketThreads) k_bucket(Params P) {
+// k_sample: A1 + A3 in batch order.  Thread t of a block handles lookups
+// c0 + it*256 + t, it < kPrepItems; their unionized searches run in
+// lockstep (kPrepItems independent probes in flight per thread).  Writes
+// the 16-B record tmp[i] = {p, i, u|b}, the material mat8[i] and the
+// histogram: per material (plain) or per (material, energy bin) (A2).
+template <int GT, bool BINNED>
+__global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
+  __shared__ uint32_t s_h[kMaxMats + 1];
+  if (!BINNED) {
+    for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x) s_h[t] = 0;
+    __syncthreads();
+  }
+  const uint32_t chunk = kPrepThreads * kPrepItems;
+  for (uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * chunk; c0 < P.count;
+       c0 += static_cast<uint64_t>(gridDim.x) * chunk) {
+    // A1: stream state at this chunk's first lookup, then short jumps
+    __shared__ uint64_t s_state;
+    if (!P.in_energy) {
+      if (threadIdx.x == 0) s_state = fast_forward(P.seed, 2 * (P.first_id + c0));
+      __syncthreads();
+    }
+    Sample smp[kPrepItems];
+    bool ok[kPrepItems];
+    int64_t lo[kPrepItems], hi[kPrepItems];
+#pragma unroll
+    for (int it = 0; it < kPrepItems; ++it) {
+      const uint64_t k = static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
+      const uint64_t i = c0 + k;
+      ok[it] = i < P.count;
+      if (P.in_energy)
+        smp[it] = ok[it] ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
+      else
+        smp[it] = sample_from_state(fast_forward(s_state, 2 * k));
+      lo[it] = 0;
+      hi[it] = P.NU - 1;
+      if (GT == XS_GRID_UNIONIZED) {
+        // A3 search range from the equal-width table: u in [UB[b]-1, UB[b+1]]
+        const double q = smp[it].p * static_cast<double>(P.UBn);
+        const int32_t b = q > 0.0 ? (q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q)
+                                                                    : P.UBn - 1)
+                                  : 0;
+        const int64_t l = static_cast<int64_t>(__ldg(P.UB + b)) - 1;
+        lo[it] = l < 0 ? 0 : (l > P.NU - 2 ? P.NU - 2 : l);
+        if (q < static_cast<double>(P.UBn)) {  // p < 1: U[UB[b+1]] > p
+          const int64_t h = __ldg(P.UB + b + 1);
+          hi[it] = h < P.NU - 1 ? h : P.NU - 1;
+        }
+      }
+    }
+    if (!P.in_energy) __syncthreads();  // s_state is rewritten next chunk
+    if (GT == XS_GRID_UNIONIZED) {
+      // XSBench grid_search loop on [lo, hi] (invariant U[lo] <= p < U[hi]),
+      // the kPrepItems searches interleaved
+      bool busy = true;
+      while (busy) {
+        busy = false;
+#pragma unroll
+        for (int it = 0; it < kPrepItems; ++it) {
+          const int64_t len = hi[it] - lo[it];
+          if (len > 1) {
+            const int64_t mid = lo[it] + (len >> 1);
+            if (__ldg(P.U + mid) > smp[it].p)
+              hi[it] = mid;
+            else
+              lo[it] = mid;
+            busy |= (hi[it] - lo[it]) > 1;
+          }
+        }
+      }
+    }
+    if (!BINNED) {
+#pragma unroll
+      for (int it = 0; it < kPrepItems; ++it) {
+        const int key = ok[it] ? smp[it].mat : kMaxMats + 7;
+        const uint32_t peers = __match_any_sync(0xffffffffu, key);
+        if (ok[it] && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&s_h[key], __popc(peers));
+      }
+    }
+#pragma unroll
+    for (int it = 0; it < kPrepItems; ++it) {
+      if (!ok[it]) continue;
+      const uint32_t i = static_cast<uint32_t>(c0 + static_cast<uint64_t>(it) * kPrepThreads +
+                                               threadIdx.x);
+      const int32_t m = smp[it].mat;
+      const double p = smp[it].p;
+      const bool valid = m < P.n_mats;
+      int32_t gi = -1;
+      if (GT == XS_GRID_UNIONIZED) gi = static_cast<int32_t>(lo[it]);
+      if (GT == XS_GRID_HASH) gi = hash_bin(p, P.du, P.B);
+      LookupRec r;
+      r.p = p;
+      r.idx = i;
+      r.gidx = valid ? gi : 0;
+      P.tmp[i] = r;
+      P.mat8[i] = static_cast<uint8_t>(m);
+      if (BINNED) {
+        atomicAdd(&P.bins[static_cast<uint32_t>(m) * kEnergyBins + energy_bin(p)], 1u);
+      }
+      if (P.out_E) P.out_E[i] = p;
+      if (P.out_mat) P.out_mat[i] = valid ? m : (P.in_mat ? P.in_mat[i] : -1);
+      if (P.out_gidx) P.out_gidx[i] = valid ? gi : -1;
+      if (!valid) write_invalid(P, i);
+    }
+  }
+  if (!BINNED) {
+    __syncthreads();
+    for (int t = threadIdx.x; t <= P.n_mats; t += blockDim.x)
+      if (s_h[t]) atomicAdd(&P.counts[t], s_h[t]);
+  }
+}
+
+// A2 scan of the (material, energy bin) histogram: exclusive prefix sums in
+// place (they become the scatter cursors) and the per-material totals.
+// Three kernels over chunks of kScanChunk bins (kEnergyBins is a multiple).
+constexpr int kScanChunk = 4096;
+
+// block-wide exclusive scan of v (1024 threads); returns the block total
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* excl) {
+  __shared__ uint32_t s_w[32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t t = s_w[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, t, o);
+      if (lane >= o) t += y;
+    }
+    s_w[lane] = t;
+  }
+  __syncthreads();
+  *excl = (w ? s_w[w - 1] : 0u) + x - v;
+  const uint32_t total = s_w[31];
+  __syncthreads();
+  return total;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_partial(Params P) {
+  const uint32_t* c = P.bins + static_cast<uint64_t>(blockIdx.x) * kScanChunk;
+  uint32_t v = 0;
+  for (int t = threadIdx.x; t < kScanChunk; t += blockDim.x) v += c[t];
+  uint32_t ex;
+  const uint32_t tot = block_excl_scan(v, &ex);
+  if (threadIdx.x == 0) P.partials[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_top(Params P, uint32_t nchunks) {
+  constexpr uint32_t kPer = kEnergyBins / kScanChunk;
+  // nchunks <= 1024 * 4 is guaranteed by the workspace layout
+  uint32_t v[4];
+  uint32_t sum = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t i = threadIdx.x * 4 + q;
+    v[q] = i < nchunks ? P.partials[i] : 0u;
+    sum += v[q];
+  }
+  uint32_t ex;
+  block_excl_scan(sum, &ex);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t i = threadIdx.x * 4 + q;
+    if (i < nchunks) {
+      P.partials[i] = ex;
+      if (v[q]) atomicAdd(&P.counts[i / kPer], v[q]);
+      ex += v[q];
+    }
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_scan_apply(Params P) {
+  uint32_t* c = P.bins + static_cast<uint64_t>(blockIdx.x) * kScanChunk;
+  constexpr int kPerThread = kScanChunk / 1024;
+  uint32_t v[kPerThread];
+  uint32_t sum = 0;
+#pragma unroll
+  for (int q = 0; q < kPerThread; ++q) {
+    v[q] = c[threadIdx.x * kPerThread + q];
+    sum += v[q];
+  }
+  uint32_t ex;
+  block_excl_scan(sum, &ex);
+  ex += P.partials[blockIdx.x];
+#pragma unroll
+  for (int q = 0; q < kPerThread; ++q) {
+    c[threadIdx.x * kPerThread + q] = ex;
+    ex += v[q];
+  }
+}
+
+// k_scatter: place each record in its material bucket (plain: block-
+// aggregated per-material cursors) or (material, energy bin) slot (A2: one
+// atomic per lookup on the scanned histogram).  Order inside a bucket or
+// bin is arbitrary: results never depend on it.
+template <bool BINNED>
+__global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
   __shared__ uint32_t s_off[kMaxMats + 2];
   __shared__ uint32_t s_cnt[kMaxMats + 1];
   __shared__ uint32_t s_base[kMaxMats + 1];
   const int nm1 = P.n_mats + 1;
-  if (threadIdx.x == 0) {
+  if (!BINNED && threadIdx.x == 0) {
     uint32_t run = 0;
     for (int m = 0; m < nm1; ++m) {
       s_off[m] = run;
@@ -162,75 +360,53 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket(Params P) {
     s_off[nm1] = run;
   }
   __syncthreads();
-  // material-field width of the sort key
-  int mat_bits = 1;
-  while ((1 << mat_bits) < nm1) ++mat_bits;
-  const int p_bits = 32 - mat_bits;
-  const uint32_t chunk = kBucketThreads * kBucketItems;
+  const int lane = threadIdx.x & 31;
+  const uint32_t chunk = kPrepThreads * kPrepItems;
   for (uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * chunk; c0 < P.count;
        c0 += static_cast<uint64_t>(gridDim.x) * chunk) {
-    if (!SORTED) {
+    if (!BINNED) {
       for (int t = threadIdx.x; t < nm1; t += blockDim.x) s_cnt[t] = 0;
       __syncthreads();
     }
-    Sample smp[kBucketItems];
-    int32_t gi[kBucketItems];
-    uint32_t rank[kBucketItems];
+    LookupRec rec[kPrepItems];
+    int32_t mm[kPrepItems];
+    uint32_t rank[kPrepItems];
 #pragma unroll
-    for (int it = 0; it < kBucketItems; ++it) {
-      const uint64_t i = c0 + static_cast<uint64_t>(it) * kBucketThreads + threadIdx.x;
+    for (int it = 0; it < kPrepItems; ++it) {
+      const uint64_t i = c0 + static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
       const bool ok = i < P.count;
-      smp[it] = ok ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
-      gi[it] = 0;
-      if (ok && smp[it].mat < P.n_mats) gi[it] = grid_index_of<GT>(P, smp[it].p);
+      if (ok) {
+        rec[it] = P.tmp[i];
+        mm[it] = P.mat8[i];
+      } else {
+        mm[it] = kMaxMats + 7;
+      }
       rank[it] = 0;
-      if (!SORTED) {
-        // warp-aggregated shared-memory rank within the block
-        const int key = ok ? smp[it].mat : kMaxMats + 7;
-        const uint32_t peers = __match_any_sync(0xffffffffu, key);
-        const int lane = threadIdx.x & 31;
+      if (BINNED) {
+        if (ok)
+          rank[it] = atomicAdd(
+              &P.bins[static_cast<uint32_t>(mm[it]) * kEnergyBins + energy_bin(rec[it].p)], 1u);
+      } else {
+        const uint32_t peers = __match_any_sync(0xffffffffu, mm[it]);
         const int leader = __ffs(peers) - 1;
         uint32_t b = 0;
-        if (ok && lane == leader) b = atomicAdd(&s_cnt[key], __popc(peers));
+        if (ok && lane == leader) b = atomicAdd(&s_cnt[mm[it]], __popc(peers));
         b = __shfl_sync(0xffffffffu, b, leader);
         rank[it] = b + __popc(peers & ((1u << lane) - 1u));
       }
     }
-    if (!SORTED) {
+    if (!BINNED) {
       __syncthreads();
       for (int t = threadIdx.x; t < nm1; t += blockDim.x)
         s_base[t] = s_cnt[t] ? s_off[t] + atomicAdd(&P.cursor[t], s_cnt[t]) : 0u;
       __syncthreads();
     }
 #pragma unroll
-    for (int it = 0; it < kBucketItems; ++it) {
-      const uint64_t i64 = c0 + static_cast<uint64_t>(it) * kBucketThreads + threadIdx.x;
-      if (i64 >= P.count) continue;
-      const uint32_t i = static_cast<uint32_t>(i64);
-      const int32_t m = smp[it].mat;
-      const double p = smp[it].p;
-      LookupRec r;
-      r.p = p;
-      r.idx = i;
-      r.gidx = gi[it];
-      if (SORTED) {
-        P.recs[i] = r;
-        double q = p * static_cast<double>(1u << p_bits);
-        uint32_t pk = q > 0.0 ? (q < static_cast<double>((1u << p_bits) - 1u)
-                                     ? static_cast<uint32_t>(q)
-                                     : (1u << p_bits) - 1u)
-                              : 0u;
-        P.keys[i] = (static_cast<uint32_t>(m) << p_bits) | pk;
-        P.vals[i] = i;
-      } else {
-        P.recs[s_base[m] + rank[it]] = r;
-      }
-      if (P.out_E) P.out_E[i] = p;
-      if (P.out_mat) P.out_mat[i] = m < P.n_mats ? m : (P.in_mat ? P.in_mat[i] : -1);
-      if (P.out_gidx) P.out_gidx[i] = (m < P.n_mats && GT != XS_GRID_NUCLIDE) ? gi[it] : -1;
-      if (m >= P.n_mats) write_invalid(P, i);
+    for (int it = 0; it < kPrepItems; ++it) {
+      const uint64_t i = c0 + static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
+      if (i < P.count) P.recs[BINNED ? rank[it] : s_base[mm[it]] + rank[it]] = rec[it];
     }
-    if (!SORTED) __syncthreads();
+    if (!BINNED) __syncthreads();
   }
 }
 
@@ -249,7 +425,13 @@ constexpr int kGatherThreads = 256;
 constexpr int kG = 3;                 // lanes per lookup
 constexpr int kLPT = 32 / kG;         // lookups per warp task (10)
 
-struct GatherSmem {
+struct alignas(16) MatEntry {
+  double conc;
+  uint32_t noff;  // n * N: first record of nuclide n
+  int32_t n;
+};
+
+struct alignas(16) GatherSmem {
   int32_t num[kMaxMats];
   uint32_t off[kMaxMats + 1];   // bucket start of material m
   uint32_t cnt[kMaxMats];
@@ -305,21 +487,23 @@ struct RowView {
 // branch-free.  Record addresses are 32-bit record indices (I*N < 2^31,
 // checked at init) scaled once: n*N is precomputed per material slot in
 // shared memory.
-template <int GT, bool SORTED, int U, int MINB, bool CHECK>
+template <int GT, int U, int MINB, bool CHECK>
 __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
   static_assert(U % kG == 0, "U must be a multiple of the group size");
   constexpr int Q = U / kG;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
   const int tab = P.n_mats * P.max_nucs;
-  double* s_concs = reinterpret_cast<double*>(smem_raw + sizeof(GatherSmem));
-  int32_t* s_mats = reinterpret_cast<int32_t*>(s_concs + tab);
-  uint32_t* s_noff = reinterpret_cast<uint32_t*>(s_mats + tab);
+  // material slot j of material m: {conc, record offset n*N, nuclide n},
+  // one 16-B shared-memory entry (a single broadcast load per nuclide step)
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
   for (int t = threadIdx.x; t < tab; t += blockDim.x) {
     const int32_t n = P.mats[t];
-    s_concs[t] = P.concs[t];
-    s_mats[t] = n;
-    s_noff[t] = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
   }
   if (threadIdx.x == 0) {
     uint32_t run = 0, trun = 0;
@@ -355,16 +539,12 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
     const bool valid = (g < kLPT) && (slot < S.cnt[m]);
     LookupRec rec{0.5, 0u, 0};
     if (valid) {
-      uint32_t pos = S.off[m] + slot;
-      if (SORTED) pos = __ldg(P.perm + pos);
-      rec = P.recs[pos];
+      rec = P.recs[S.off[m] + slot];
     }
     const double p = rec.p;
     const int nn = valid ? S.num[m] : 0;   // invalid lanes load nothing
     const int nw_loop = S.num[m];           // warp-uniform trip count
-    const int32_t* mrow = s_mats + m * P.max_nucs;
-    const uint32_t* orow = s_noff + m * P.max_nucs;
-    const double* crow = s_concs + m * P.max_nucs;
+    const MatEntry* row = s_tab + m * P.max_nucs;
     const RowView<GT> rv(P, valid ? rec.gidx : 0);
 
     double acc_a = 0.0, acc_b = 0.0;
@@ -372,7 +552,12 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       const int j = r + q * kG;
-      knext[q] = j < nn ? rv.bracket(P, mrow[j], orow[j], p) : 0;
+      int32_t kq = 0;
+      if (j < nn) {
+        const MatEntry me = row[j];
+        kq = rv.bracket(P, me.n, me.noff, p);
+      }
+      knext[q] = kq;
     }
     // One round = U consecutive nuclides of the list.  Full rounds run
     // without any per-nuclide predicate; the (at most one) partial round at
@@ -386,19 +571,27 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
 #pragma unroll
       for (int q = 0; q < Q; ++q) {
         const int j = j0 + U + r + q * kG;
-        knext[q] = j < nn ? rv.bracket(P, mrow[j], orow[j], p) : 0;
+        int32_t kq = 0;
+        if (j < nn) {
+          const MatEntry me = row[j];
+          kq = rv.bracket(P, me.n, me.noff, p);
+        }
+        knext[q] = kq;
       }
       // A5: 96-B record pairs; lane r loads chunk r of the low and high
-      // record.  (Past the end of the list, or without a lookup, a lane
-      // reads the grid's first record pair instead: always valid memory,
-      // the value is never accumulated.)
+      // record.  A lane without a lookup has k = 0 and reads the nuclide's
+      // first pair; in the tail round, slots past the end of the list read
+      // the grid's first pair: always valid memory, never accumulated.
       double2 lo[U], hi[U];
+      double cc[U];
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + t;
         const int32_t kt = __shfl_sync(0xffffffffu, kcur[t / kG], base + (t % kG));
-        uint32_t off = orow[j] + static_cast<uint32_t>(kt);
-        if (TAIL || !valid) off = j < nn ? off : 0u;
+        const MatEntry me = row[TAIL ? (j < nw_loop ? j : 0) : j];
+        cc[t] = me.conc;
+        uint32_t off = me.noff + static_cast<uint32_t>(kt);
+        if (TAIL) off = j < nw_loop ? off : 0u;
         const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
         lo[t] = __ldg(pr);
         hi[t] = __ldg(pr + 3);
@@ -426,7 +619,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
         const double xa = dsub(hi[t].x, dmul(f, dsub(hi[t].x, lo[t].x)));
         const double xb = dsub(hi[t].y, dmul(f, dsub(hi[t].y, lo[t].y)));
         if (!TAIL || j < nw_loop) {  // warp-uniform
-          const double c = crow[j];
+          const double c = cc[t];
           acc_a = dadd(acc_a, dmul(xa, c));
           acc_b = dadd(acc_b, dmul(xb, c));
         }
@@ -601,6 +794,8 @@ static Params make_params(const DeviceGrid& g) {
   P.N = g.N;
   P.U = g.U;
   P.NU = g.NU;
+  P.UB = g.UB;
+  P.UBn = g.UBn;
   P.index = g.index;
   P.B = g.B;
   P.du = g.du;
@@ -620,11 +815,10 @@ static unsigned grid_cap(uint64_t work, int threads, int sm, int per_sm) {
   return static_cast<unsigned>(b < cap ? b : cap);
 }
 
-template <int GT, bool SORTED, int U, int MINB, bool CHECK>
+template <int GT, int U, int MINB, bool CHECK>
 static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs *
-                                               (sizeof(double) + 2 * sizeof(int32_t));
-  auto kern = k_gather<GT, SORTED, U, MINB, CHECK>;
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
+  auto kern = k_gather<GT, U, MINB, CHECK>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -643,21 +837,20 @@ static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStrea
 // energy (grid and lookups) is a multiple of 2^-63 in [0, 1] (DESIGN.md §4:
 // then |hi.E - p| and |hi.E - lo.E| are 0 or >= 2^-63), which holds for
 // generated grids with sampled lookups; otherwise the checked kernel runs.
-template <int GT, bool SORTED, bool CHECK>
+template <int GT, bool CHECK>
 static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   switch (g.unroll) {
-    case 1: return launch_gather<GT, SORTED, 3, 3, CHECK>(g, P, st);
-    case 2: return launch_gather<GT, SORTED, 3, 4, CHECK>(g, P, st);
-    case 4: return launch_gather<GT, SORTED, 6, 3, CHECK>(g, P, st);
-    default: return launch_gather<GT, SORTED, 6, 2, CHECK>(g, P, st);
+    case 1: return launch_gather<GT, 3, 3, CHECK>(g, P, st);
+    case 2: return launch_gather<GT, 3, 4, CHECK>(g, P, st);
+    case 4: return launch_gather<GT, 6, 3, CHECK>(g, P, st);
+    default: return launch_gather<GT, 6, 2, CHECK>(g, P, st);
   }
 }
 
-template <int GT, bool SORTED>
+template <int GT>
 static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   const bool check = P.in_energy != nullptr || !g.dyadic63;
-  return check ? launch_gather_v<GT, SORTED, true>(g, P, st)
-               : launch_gather_v<GT, SORTED, false>(g, P, st);
+  return check ? launch_gather_v<GT, true>(g, P, st) : launch_gather_v<GT, false>(g, P, st);
 }
 
 template <int GT>
@@ -695,29 +888,32 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   }
   e = cudaMemsetAsync(ws.counts, 0, 2 * (kMaxMats + 1) * sizeof(uint32_t), st);
   if (e != cudaSuccess) return e;
-  k_count<<<grid_cap(a.count, 256, g.sm_count, 8), 256, 0, st>>>(P);
-  const unsigned nb = grid_cap(a.count, kBucketThreads * kBucketItems, g.sm_count, 16);
-  const bool sorted = a.flags & XS_FLAG_SORT;
-  if (sorted) {
-    P.keys = ws.keys0;
-    P.vals = ws.vals0;
-    k_bucket<GT, true><<<nb, kBucketThreads, 0, st>>>(P);
-  } else {
-    k_bucket<GT, false><<<nb, kBucketThreads, 0, st>>>(P);
-  }
-  launched(2);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  mark(1);
-  if (sorted) {
-    bool in1 = false;
-    e = rs::sort_pairs<uint32_t, true>(ws.keys0, ws.vals0, ws.keys1, ws.vals1, a.count, 32,
-                                       ws.sort_work, st, &in1);
+  const bool binned = a.flags & XS_FLAG_SORT;
+  const unsigned nb = grid_cap(a.count, kPrepThreads * kPrepItems, g.sm_count, 16);
+  P.tmp = ws.tmp;
+  P.mat8 = ws.mat8;
+  if (binned) {
+    P.bins = ws.bins;
+    e = cudaMemsetAsync(ws.bins, 0, static_cast<size_t>(g.n_mats + 1) * kEnergyBins * 4, st);
     if (e != cudaSuccess) return e;
-    launched(12);
-    P.perm = in1 ? ws.vals1 : ws.vals0;
+    P.partials = ws.partials;
+    const uint32_t nchunks = static_cast<uint32_t>(g.n_mats + 1) * (kEnergyBins / kScanChunk);
+    k_sample<GT, true><<<nb, kPrepThreads, 0, st>>>(P);
+    mark(1);
+    k_scan_partial<<<nchunks, 1024, 0, st>>>(P);
+    k_scan_top<<<1, 1024, 0, st>>>(P, nchunks);
+    k_scan_apply<<<nchunks, 1024, 0, st>>>(P);
+    k_scatter<true><<<nb, kPrepThreads, 0, st>>>(P);
+    launched(5);
+  } else {
+    k_sample<GT, false><<<nb, kPrepThreads, 0, st>>>(P);
+    mark(1);
+    k_scatter<false><<<nb, kPrepThreads, 0, st>>>(P);
+    launched(2);
   }
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
   mark(2);
-  e = sorted ? launch_gather_u<GT, true>(g, P, st) : launch_gather_u<GT, false>(g, P, st);
+  e = launch_gather_u<GT>(g, P, st);
   launched(1);
   mark(3);
   return e;

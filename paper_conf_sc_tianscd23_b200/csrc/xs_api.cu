@@ -75,24 +75,22 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
   };
   const size_t o_counts = take(2 * (kMaxMats + 1) * sizeof(uint32_t));
   const size_t o_recs = take(count * sizeof(LookupRec));
-  size_t o_k0 = 0, o_k1 = 0, o_v0 = 0, o_v1 = 0, o_work = 0;
+  const size_t o_tmp = take(count * sizeof(LookupRec));
+  const size_t o_mat8 = take(count);
+  size_t o_bins = 0, o_part = 0;
   if (flags & XS_FLAG_SORT) {
-    o_k0 = take(count * 4);
-    o_k1 = take(count * 4);
-    o_v0 = take(count * 4);
-    o_v1 = take(count * 4);
-    o_work = take(rs::hist_bytes(count));
+    o_bins = take(static_cast<size_t>(kMaxMats + 1) * kEnergyBins * 4);
+    o_part = take(static_cast<size_t>(kMaxMats + 1) * (kEnergyBins / 4096) * 4);
   }
   if (ws) {
     char* b = static_cast<char*>(base);
     ws->counts = reinterpret_cast<uint32_t*>(b + o_counts);
     ws->cursor = ws->counts + (kMaxMats + 1);
     ws->recs = reinterpret_cast<LookupRec*>(b + o_recs);
-    ws->keys0 = reinterpret_cast<uint32_t*>(b + o_k0);
-    ws->keys1 = reinterpret_cast<uint32_t*>(b + o_k1);
-    ws->vals0 = reinterpret_cast<uint32_t*>(b + o_v0);
-    ws->vals1 = reinterpret_cast<uint32_t*>(b + o_v1);
-    ws->sort_work = b + o_work;
+    ws->bins = reinterpret_cast<uint32_t*>(b + o_bins);
+    ws->partials = reinterpret_cast<uint32_t*>(b + o_part);
+    ws->tmp = reinterpret_cast<LookupRec*>(b + o_tmp);
+    ws->mat8 = reinterpret_cast<uint8_t*>(b + o_mat8);
     ws->total = off;
   }
   return off;
@@ -220,9 +218,14 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   G.index_len = d->grid_type == XS_GRID_UNIONIZED ? G.NU * I
                 : d->grid_type == XS_GRID_HASH    ? static_cast<int64_t>(G.B) * I
                                                   : 0;
+  if (G.NU) {  // ~64 unionized energies per search-table bin
+    G.UBn = 1024;
+    while (G.UBn < (1 << 22) && static_cast<int64_t>(G.UBn) * 64 < G.NU) G.UBn <<= 1;
+  }
   auto cleanup = [&]() {
     cudaFree(G.grid);
     cudaFree(G.U);
+    cudaFree(G.UB);
     cudaFree(G.index);
     cudaFree(G.num_nucs);
     cudaFree(G.mats);
@@ -231,6 +234,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   const size_t grid_bytes = static_cast<size_t>(I) * N * 6 * sizeof(double);
   cudaError_t e = cudaMalloc(&G.grid, grid_bytes);
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
+  if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.UB, (static_cast<size_t>(G.UBn) + 1) * 4);
   if (e == cudaSuccess && G.index_len) e = cudaMalloc(&G.index, G.index_len * sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&G.num_nucs, d->n_mats * sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&G.mats, tab * sizeof(int32_t));
@@ -239,7 +243,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cleanup();
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
-  G.device_bytes = grid_bytes + G.NU * 8 + G.index_len * 4 + d->n_mats * 4 + tab * 12;
+  G.device_bytes = grid_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 + d->n_mats * 4 + tab * 12;
   e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
@@ -247,6 +251,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.concs, d->concs, tab * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
     e = build_union_grid(G, G.U, st);
+    if (e == cudaSuccess) e = build_union_table(G, st);
     if (e == cudaSuccess) e = build_index_grid(G, st);
   }
   if (e == cudaSuccess && G.grid_type == XS_GRID_HASH) e = build_hash_grid(G, st);
@@ -516,11 +521,11 @@ xs_status xs_timing_read(xs_grid* g, xs_timing* out) {
     XS_TRY(cudaEventElapsedTime(&t[0], e[0], e[1]), "cudaEventElapsedTime");
     XS_TRY(cudaEventElapsedTime(&t[1], e[1], e[2]), "cudaEventElapsedTime");
     XS_TRY(cudaEventElapsedTime(&t[2], e[2], e[3]), "cudaEventElapsedTime");
-    out->ms_prepare += t[0];
-    out->ms_sort += t[1];
+    out->ms_count += t[0];
+    out->ms_bucket += t[1];
     out->ms_gather += t[2];
   }
-  out->ms_total = out->ms_prepare + out->ms_sort + out->ms_gather;
+  out->ms_total = out->ms_count + out->ms_bucket + out->ms_gather;
   g->ev_used = 0;
   g->calls = 0;
   g->launches_read = g->d.launches;
@@ -534,6 +539,7 @@ void xs_free_grid(xs_grid* g) {
     for (auto x : e) cudaEventDestroy(x);
   cudaFree(g->d.grid);
   cudaFree(g->d.U);
+  cudaFree(g->d.UB);
   cudaFree(g->d.index);
   cudaFree(g->d.num_nucs);
   cudaFree(g->d.mats);

@@ -17,6 +17,7 @@ struct alignas(16) LookupRec {
 };
 
 constexpr int kMaxMats = 64;  // materials supported by the bucketed kernels
+constexpr uint32_t kEnergyBins = 65536;  // A2: energy bins per material
 
 struct DeviceGrid {
   int device = 0;
@@ -30,6 +31,8 @@ struct DeviceGrid {
   int64_t NU = 0, index_len = 0;
   double* grid = nullptr;    // [I][N][6]
   double* U = nullptr;       // [NU]
+  int32_t* UB = nullptr;     // [UBn + 1]: UB[b] = ub(U, b / UBn)  (A3 search table)
+  int32_t UBn = 0;           // power of two
   int32_t* index = nullptr;  // IG [NU][I] or HG [B][I]
   int32_t* num_nucs = nullptr;
   int32_t* mats = nullptr;   // [n_mats][max_nucs]
@@ -60,11 +63,10 @@ struct Workspace {
   uint32_t* counts;   // [kMaxMats + 1]
   uint32_t* cursor;   // [kMaxMats + 1]
   LookupRec* recs;    // [count]
-  uint32_t* keys0;    // sort
-  uint32_t* keys1;
-  uint32_t* vals0;
-  uint32_t* vals1;
-  void* sort_work;
+  uint32_t* bins;     // A2: [(kMaxMats + 1) * kEnergyBins]
+  LookupRec* tmp;     // [count] records in batch order
+  uint8_t* mat8;      // [count]
+  uint32_t* partials; // A2 scan: [(kMaxMats + 1) * kEnergyBins / 4096]
   size_t total;
 };
 size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws);
@@ -73,6 +75,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
 cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st);
 cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st);
+cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st);
 cudaError_t init_constants();
 
 // lookup.cu

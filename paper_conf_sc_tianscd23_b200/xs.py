@@ -59,7 +59,7 @@ class xs_grid_info(C.Structure):
 
 class xs_timing(C.Structure):
     _fields_ = [("calls", C.c_uint64), ("kernel_launches", C.c_uint64),
-                ("ms_prepare", C.c_double), ("ms_sort", C.c_double), ("ms_gather", C.c_double),
+                ("ms_count", C.c_double), ("ms_bucket", C.c_double), ("ms_gather", C.c_double),
                 ("ms_total", C.c_double)]
 
 

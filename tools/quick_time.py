@@ -56,7 +56,7 @@ def main():
             g.timing(False)
             n = t["calls"] or 1
             print(f"{var:9s} bps={bps} {ms:8.3f} ms/step  {L / ms / 1e6:8.3f} G lookups/s  "
-                  f"prep {t['ms_prepare']/n:.3f} sort {t['ms_sort']/n:.3f} gather {t['ms_gather']/n:.3f}"
+                  f"count {t['ms_count']/n:.3f} bucket {t['ms_bucket']/n:.3f} gather {t['ms_gather']/n:.3f}"
                   f"  launches/step {t['kernel_launches']/n:.0f} hash_ok={ok}", flush=True)
         g.set_param("variant", 0)
         g.set_param("blocks_per_sm", 0)
