@@ -1,0 +1,378 @@
+#!/usr/bin/env python
+"""bench.py — XSBench event-based macroscopic XS lookups/s on B200.
+
+Metric (BASELINE.json): XS lookups/sec at 1/2/4/8 B200 and the fraction of
+the HBM-gather roofline.  One step = one pass of the whole hot path (A1
+sample, A2 (material, energy) binning, A3 unionized/hash search, A4-A8
+gather, interpolate, accumulate, verify; A9 all-reduce when N > 1) over one
+batch of synthetic lookups whose tables are resident in HBM.  At N = 1 the
+workload is XSBench "large" (355 nuclides x 11,303 points, 17M lookups,
+unionized grid) — the configuration BASELINE.json's target is quoted on.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config large]
+                  [--impl ours|reference] [--scaling weak|strong] [--no-sort]
+  (N > 1: python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N)
+
+--impl reference times the CPU oracle (oracle/, plain serial C per lookup)
+on the host cores, as the reference arm of this tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+ORACLE_MODE = {"unionized": 0, "nuclide": 1, "hash": 2}
+MAT_PROB = [0.139, .052, .275, .134, .154, .064, .066, .055, .008, .015, .025, .013]
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="large",
+                    choices=["tiny", "small", "large", "large-hash", "xl"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--no-sort", action="store_true", help="skip A2 (material/energy binning)")
+    ap.add_argument("--lookups", type=int, default=0, help="override lookups per GPU (weak)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0,
+                    help="target CPU seconds of the oracle sample")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- clocks --
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+    def __init__(self, index: int, period: float = 0.02):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.period = period
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover - NVML missing
+            self._nv = None
+            self.error = str(e)
+
+    def _run(self):
+        nv = self._nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self._nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self._nv:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml_unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------- helpers ------
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def golden():
+    with open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")) as f:
+        return json.load(f)
+
+
+def ncu_traffic(config: str, sort: bool):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None, None
+    with open(p) as f:
+        d = json.load(f)
+    e = d.get(f"{config}{'-sorted' if sort else ''}")
+    if not e:
+        return None, None
+    return e.get("dram_bytes_per_lookup"), e.get("source")
+
+
+def cpu_info():
+    name = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    name = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return name
+
+
+def oracle_sample_rate(pre, target_s: float, first: int = 0):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload
+    on all host cores.  Returns (lookups/s, cores, description, sum_v)."""
+    import oracle
+    cores = os.cpu_count() or 1
+    mode = ORACLE_MODE[pre["grid_type"]]
+    o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"], conc_seed=1070 * 1070,
+                                material_rule=pre["material_rule"],
+                                hash_bins=pre.get("hash_bins", 0), nthreads=cores)
+    pilot = min(pre["lookups"], 20_000)
+    t0 = time.perf_counter()
+    o.run(first, pilot, mode=mode, nthreads=cores)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    n = int(min(pre["lookups"], max(pilot, pilot / dt * target_s)))
+    t0 = time.perf_counter()
+    S = o.run(first, n, mode=mode, nthreads=cores)
+    dt = time.perf_counter() - t0
+    desc = (f"lookup ids [{first}, {first + n}) of the {pre['lookups']:,}-lookup "
+            f"{pre['grid_type']} workload, oracle route '{pre['grid_type']}', {cores} threads, "
+            f"{dt:.1f} s")
+    return n / dt, cores, desc, S, n
+
+
+# ------------------------------------------------------------- reference ----
+def run_reference(a, pre, cfg):
+    rank = int(os.environ.get("RANK", 0))
+    if rank != 0:
+        return 0
+    t_start = time.time()
+    # size each step to a bounded sample so the whole run takes a few minutes
+    budget = 150.0
+    per_step = max(1.0, min(a.cpu_seconds, budget / max(1, a.steps + a.warmup)))
+    rate0, cores, _, _, _ = oracle_sample_rate(pre, per_step / 4)
+    n = int(min(pre["lookups"], max(10_000, rate0 * per_step)))
+    import oracle
+    mode = ORACLE_MODE[pre["grid_type"]]
+    o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"], conc_seed=1070 * 1070,
+                                material_rule=pre["material_rule"],
+                                hash_bins=pre.get("hash_bins", 0), nthreads=cores)
+    for w in range(a.warmup):
+        o.run((w * n) % max(1, pre["lookups"] - n + 1), n, mode=mode, nthreads=cores)
+    times = []
+    for k in range(a.steps):
+        first = (k * n) % max(1, pre["lookups"] - n + 1)
+        t0 = time.perf_counter()
+        o.run(first, n, mode=mode, nthreads=cores)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    value = n * a.steps / tot
+    line = {"impl": "reference", "metric": "XS lookups/sec", "value": value,
+            "unit": "lookups/s", "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
+            "ms_per_step": 1e3 * tot / a.steps, "higher_is_better": True,
+            "scaling": a.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": cfg,
+            "cpu_baseline": {"value": value, "unit": "lookups/s", "cores": cores,
+                             "kind": "oracle",
+                             "sample": f"{n:,} lookups per step ({pre['grid_type']} route), "
+                                       f"{cores} host threads, {cpu_info()}"},
+            "e2e": {"value": value, "unit": "lookups/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0},
+            "wall_s": round(time.time() - t_start, 1)}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ ours ----
+def run_ours(a, pre, cfg):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_tianscd23_b200 import dist as D
+    from paper_conf_sc_tianscd23_b200 import xs as X
+
+    rank, world, local = D.env_rank()
+    if world != a.gpus:
+        raise SystemExit(f"--gpus {a.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    sort = not a.no_sort
+    L_cfg = a.lookups or pre["lookups"]
+    first, L = D.shard_range(rank, world, L_cfg, a.scaling)
+
+    t0 = time.time()
+    g = X.Grid.from_preset(a.config, device=local)
+    torch.cuda.synchronize()
+    init_s = time.time() - t0
+    stream = torch.cuda.current_stream(dev)
+
+    # untimed: per-material counts of this shard (exact algorithmic bytes)
+    # and the inputs of the end-to-end leg
+    vs0, res0 = g.lookup(first, L, sort=sort, want=("mat", "energy"))
+    torch.cuda.synchronize()
+    mats = torch.bincount(res0["mat"].long(), minlength=g.info.n_mats).cpu().tolist()
+    num_nucs = g.table(X.XS_TABLE_NUM_NUCS).tolist()
+    nuc_lookups = sum(c * n for c, n in zip(mats, num_nucs))
+    idx_bytes = 4 if pre["grid_type"] == "unionized" else 8
+    gather_bytes = nuc_lookups * (idx_bytes + 96)            # A4 + A5 per launch
+    search_bytes = L * 8 * math.ceil(math.log2(max(2, g.info.n_union - 1))) \
+        if pre["grid_type"] == "unionized" else 0
+    balg_per_lookup = (gather_bytes + search_bytes) / L      # SURVEY §8(d) B_alg
+    gold = golden().get(a.config)
+    hash_check = None
+    if gold and first == 0 and L == gold["lookups"]:
+        hash_check = int(vs0[0]) == gold["sum_v"] and int(vs0[1]) == L
+
+    vsum = torch.zeros(2, dtype=torch.int64, device=dev)
+
+    def step():
+        vsum.zero_()
+        g.lookup(first, L, sort=sort, vsum=vsum)
+        if world > 1:
+            D.combine_vsum(vsum)          # A9
+
+    for _ in range(a.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    g.timing(True)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(a.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms_local = ev0.elapsed_time(ev1)
+    tm = g.timing_read()
+    g.timing(False)
+    ms = D.max_over_ranks(ms_local, device=dev)
+    total_lookups = L * world * a.steps if a.scaling == "weak" else L_cfg * a.steps
+    value = total_lookups / (ms / 1e3)
+    vglob = [int(x) for x in vsum.cpu()]
+
+    peak, peak_src = measured_peaks()
+    gather_ms = tm["ms_gather"] / max(1, tm["calls"])
+    achieved = gather_bytes / (gather_ms / 1e3) / 1e9
+    traffic_per_lookup, traffic_src = ncu_traffic(a.config, sort)
+    roofline = {"bound": "hbm", "kernel": "k_gather (A4-A8)", "achieved": achieved,
+                "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic_per_lookup * L if traffic_per_lookup else None,
+                "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": gather_bytes,
+                "gather_ms_per_launch": gather_ms,
+                "traffic_source": traffic_src,
+                "note": "algorithmic bytes = sum over lookups of n_nuclides(mat) x "
+                        f"({idx_bytes} B index + 96 B record pair); L2 hits let frac exceed 1"}
+    step_frac = balg_per_lookup * (value / world) / 8e12
+
+    line = {"metric": "XS lookups/sec", "value": value, "unit": "lookups/s", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps,
+            "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic", "config": cfg,
+            "roofline": roofline,
+            "hbm_gather_roofline_frac_8TBs": step_frac,
+            "balg_bytes_per_lookup": balg_per_lookup,
+            "phase_ms_per_step": {k: tm[k] / max(1, tm["calls"])
+                                  for k in ("ms_count", "ms_bucket", "ms_gather")},
+            "gpu_launches": int(tm["kernel_launches"]),
+            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash_matches_oracle": hash_check, "init_s": round(init_s, 2)}
+    # ------------------------------------------------------------- e2e leg
+    if not a.no_e2e:
+        e_host = res0["energy"].cpu().pin_memory()
+        m_host = res0["mat"].cpu().pin_memory()
+        vs_h = torch.zeros(2, dtype=torch.int64).pin_memory()
+        g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)      # warm-up
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(a.e2e_steps):
+            vs_h.zero_()
+            g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)  # H2D, lookup, D2H
+        dt = time.perf_counter() - t0
+        dt = D.max_over_ranks(dt, device=dev)
+        e2e_total = L * world * a.e2e_steps if a.scaling == "weak" else L_cfg * a.e2e_steps
+        line["e2e"] = {"value": e2e_total / dt, "unit": "lookups/s",
+                       "h2d_bytes_per_step": int(L * 12), "d2h_bytes_per_step": 16,
+                       "api": "xs_lookup_explicit(XS_FLAG_HOST_IO): pinned host energy+material "
+                              "in, vsum out; wall clock per call (the call synchronizes)",
+                       "steps": a.e2e_steps,
+                       "vsum_matches_batch": [int(x) for x in vs_h] == [int(x) for x in vs0]}
+    line["clocks"] = clk.summary()
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        try:
+            rate, cores, desc, S, n = oracle_sample_rate(pre, a.cpu_seconds)
+            line["cpu_baseline"] = {"value": rate, "unit": "lookups/s", "cores": cores,
+                                    "kind": "oracle", "sample": desc, "cpu": cpu_info()}
+        except Exception as e:  # the oracle is test infrastructure; report, don't fail
+            line["cpu_baseline"] = {"value": None, "unit": "lookups/s", "cores": None,
+                                    "kind": "oracle", "sample": f"failed: {e}"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    a = parse()
+    from paper_conf_sc_tianscd23_b200.xs_presets import PRESETS
+    pre = dict(PRESETS[a.config])
+    per_gpu = a.lookups or pre["lookups"]
+    cfg = {"workload": a.config, "n_isotopes": pre["n_isotopes"],
+           "n_gridpoints": pre["n_gridpoints"], "grid": pre["grid_type"],
+           "hash_bins": pre.get("hash_bins"), "lookups_per_gpu": per_gpu if a.scaling == "weak"
+           else None, "lookups_total": per_gpu if a.scaling == "strong" else per_gpu * a.gpus,
+           "sort": ("A2 material+energy binning (65536 energy bins per material)"
+                    if not a.no_sort else "none"),
+           "l2": "not flushed: tables (5.9 GB for large) far exceed the 126 MB L2",
+           "parallelism": f"dp{a.gpus} (lookup shards, grid replicated)"}
+    if a.impl == "reference":
+        return run_reference(a, pre, cfg)
+    return run_ours(a, pre, cfg)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

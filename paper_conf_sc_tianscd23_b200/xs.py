@@ -173,6 +173,10 @@ def xs_set_param(g, name: str, value: int):
     _check(lib.xs_set_param(g, name.encode(), value))
 
 
+def xs_last_error() -> str:
+    return lib.xs_last_error().decode(errors="replace")
+
+
 def xs_hash_finalize(s: int) -> int:
     return lib.xs_hash_finalize(s)
 
@@ -192,20 +196,7 @@ def xs_timing_read(g) -> xs_timing:
 
 
 # --------------------------------------------------------------- presets
-# BASELINE.json configs; seeds per DESIGN.md R1 (grid 42, conc 1070^2, lookups 1070)
-PRESETS = {
-    "tiny": dict(n_isotopes=12, n_gridpoints=1000, material_rule=1, lookups=100_000,
-                 grid_type="unionized"),
-    "small": dict(n_isotopes=68, n_gridpoints=11303, material_rule=0, lookups=17_000_000,
-                  grid_type="unionized"),
-    "large": dict(n_isotopes=355, n_gridpoints=11303, material_rule=0, lookups=17_000_000,
-                  grid_type="unionized"),
-    "large-hash": dict(n_isotopes=355, n_gridpoints=11303, material_rule=0, lookups=17_000_000,
-                       grid_type="hash", hash_bins=8192, sort=True),
-    "xl": dict(n_isotopes=355, n_gridpoints=238847, material_rule=0, lookups=170_000_000,
-               grid_type="unionized"),
-}
-GRID_SEED, CONC_SEED, LOOKUP_SEED = 42, 1070 * 1070, 1070
+from .xs_presets import CONC_SEED, GRID_SEED, LOOKUP_SEED, PRESETS  # noqa: E402
 
 
 def make_spec(n_isotopes, n_gridpoints, grid_type="unionized", hash_bins=0, material_rule=0,
