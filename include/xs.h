@@ -78,8 +78,20 @@ typedef struct {
   uint64_t conc_seed;     /* concentration draws                                */
   uint64_t lookup_seed;   /* lookup stream seed (A1)                            */
   int32_t material_rule;  /* 0 = XSBench H-M tables, 1 = ids mod I (tiny)       */
-  int32_t reserved0;      /* must be 0                                          */
+  int32_t index_layout;   /* XS_INDEX_*: unionized index-grid layout(s), 0 = auto */
 } xs_grid_spec;
+
+/* Unionized index grid layouts (same values, different memory order):
+ *   ROW  IG[u][n]  (u-major, row of I ints per unionized energy): one lookup
+ *        reads a contiguous row — best for unsorted batches;
+ *   COL  IGT[n][u] (nuclide-major): the lookups of an energy-sorted batch
+ *        read neighbouring entries of one column — best with XS_FLAG_SORT.
+ * AUTO builds both when they fit comfortably in device memory (large: 2 x
+ * 5.7 GB), else COL only (XL: 120 GB). */
+#define XS_INDEX_AUTO 0
+#define XS_INDEX_ROW 1
+#define XS_INDEX_COL 2
+#define XS_INDEX_BOTH 3
 
 /* Caller-supplied nuclear data (HOST pointers, copied during init).  The
  * nuclide grid is [I][N][6] doubles (E, total, elastic, absorption, fission,
@@ -100,6 +112,8 @@ typedef struct {
   int32_t grid_type;
   int32_t hash_bins;
   uint64_t lookup_seed;
+  int32_t index_layout;   /* XS_INDEX_* (unionized only), 0 = auto */
+  int32_t reserved0;      /* must be 0 */
 } xs_grid_data;
 
 typedef struct xs_grid xs_grid; /* opaque: one replica of the tables on one device */
@@ -111,6 +125,8 @@ typedef struct {
   int64_t index_grid_len; /* NU*I (UNIONIZED), B*I (HASH), 0 (NUCLIDE)          */
   uint64_t device_bytes;  /* bytes of device memory the grid holds              */
   uint64_t lookup_seed;
+  int32_t index_layout;   /* layouts actually built (XS_INDEX_ROW | XS_INDEX_COL) */
+  int32_t reserved0;
 } xs_grid_info;
 
 /* Per-lookup outputs, indexed by position i in the batch (lookup id
@@ -140,6 +156,7 @@ typedef struct {
 #define XS_TABLE_NUM_NUCS 3     /* [int32]  n_mats                              */
 #define XS_TABLE_MATS 4         /* [int32]  n_mats*max_num_nucs                 */
 #define XS_TABLE_CONCS 5        /* [double] n_mats*max_num_nucs                 */
+#define XS_TABLE_INDEX_GRID_T 6 /* [int32]  IGT (I*NU), nuclide-major            */
 
 uint32_t xs_abi_version(void);
 

@@ -100,6 +100,45 @@ cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// K0b' (column layout): IGT[n][e] = clamp(ub(E_n, U[e]) - 1, 0, N-2).
+// Block (x, n): warp w sweeps 256 consecutive unionized energies of nuclide
+// n in steps of 32 (one per lane, coalesced 128-B writes).  The bracket of
+// the first energy comes from one binary search; each later lane advances
+// from its warp's previous bracket (energies increase along e).
+constexpr int kIgtPerWarp = 256;
+
+__global__ void __launch_bounds__(256) k_build_index_grid_t(const double* __restrict__ grid,
+                                                           int64_t N,
+                                                           const double* __restrict__ U,
+                                                           int64_t NU, int32_t* __restrict__ IGT) {
+  const int32_t n = blockIdx.y;
+  const int lane = threadIdx.x & 31;
+  const int64_t e_begin = (static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) +
+                           (threadIdx.x >> 5)) * kIgtPerWarp;
+  if (e_begin >= NU) return;
+  const double* rec = grid + static_cast<int64_t>(n) * N * 6;
+  int64_t kw = bracket_search_rec(rec, 0, N - 1, __ldg(U + e_begin));  // warp-uniform
+  int32_t* col = IGT + static_cast<int64_t>(n) * NU;
+  for (int64_t e0 = e_begin; e0 < e_begin + kIgtPerWarp && e0 < NU; e0 += 32) {
+    const int64_t e = e0 + lane;
+    int64_t k = kw;
+    if (e < NU) {
+      const double q = __ldg(U + e);
+      while (k < N - 2 && rec_energy(rec, k + 1) <= q) ++k;
+      col[e] = static_cast<int32_t>(k);
+    }
+    kw = __shfl_sync(0xffffffffu, k, 31);  // last lane's bracket (monotone in e)
+    if (e0 + 32 > NU) break;
+  }
+}
+
+cudaError_t build_index_grid_t(const DeviceGrid& g, cudaStream_t st) {
+  const int64_t per_block = 8 * kIgtPerWarp;
+  dim3 grid(static_cast<unsigned>((g.NU + per_block - 1) / per_block), static_cast<unsigned>(g.I));
+  k_build_index_grid_t<<<grid, 256, 0, st>>>(g.grid, g.N, g.U, g.NU, g.index_t);
+  return cudaGetLastError();
+}
+
 __global__ void k_build_hash_grid(const double* __restrict__ grid, int32_t I, int64_t N, int32_t B,
                                   double du, int32_t* __restrict__ HG) {
   const uint64_t total = static_cast<uint64_t>(B) * I;

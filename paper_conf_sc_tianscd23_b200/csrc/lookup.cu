@@ -83,7 +83,8 @@ struct Params {
   int64_t NU;
   const int32_t* UB;
   int32_t UBn;
-  const int32_t* index;
+  const int32_t* index;     // IG (row layout) / HG, or null
+  const int32_t* index_t;   // IGT (column layout), or null
   int32_t B;
   double du;
   const int32_t* num_nucs;
@@ -415,7 +416,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
 template <int GT>
 __device__ __forceinline__ int32_t bracket_of(const Params& P, int32_t gidx, int32_t n, double p) {
   if (GT == XS_GRID_UNIONIZED)
-    return __ldg(P.index + static_cast<int64_t>(gidx) * P.I + n);
+    return P.index ? __ldg(P.index + static_cast<int64_t>(gidx) * P.I + n)
+                   : __ldg(P.index_t + static_cast<int64_t>(n) * P.NU + gidx);
   const double* rec = P.grid + static_cast<int64_t>(n) * P.N * 6;
   if (GT == XS_GRID_HASH) return hash_bracket(P.index, P.I, P.B, gidx, n, rec, P.N, p);
   return nuclide_bracket(rec, P.N, p);
@@ -446,7 +448,7 @@ struct RowView {
   const int32_t* r1;
   __device__ __forceinline__ RowView(const Params& P, int32_t gidx) {
     if (GT == XS_GRID_UNIONIZED) {
-      r0 = P.index + static_cast<int64_t>(gidx) * P.I;
+      r0 = P.index ? P.index + static_cast<int64_t>(gidx) * P.I : nullptr;
       r1 = r0;
     } else if (GT == XS_GRID_HASH) {
       r0 = P.index + static_cast<int64_t>(gidx) * P.I;
@@ -679,6 +681,167 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
   }
 }
 
+// --------------------------------------------- thread-per-lookup gather ---
+// k_gather_t: for energy-sorted batches (XS_FLAG_SORT).  A warp takes 32
+// consecutive lookups of one material bucket — after A2 they lie within a
+// few 1e-5 of each other in energy, so for each nuclide the 32 lanes read
+// the same or neighbouring record pairs (1-2 cache lines per 128-bit load
+// instruction) and, with the column-layout index grid IGT[n][u], neighbouring
+// index entries.  Each lane then owns its whole lookup: 6 x 128-bit loads of
+// the record pair, its own exact division, all five channels, list-order
+// accumulation — no shuffles, every lane's arithmetic useful.
+constexpr int kLPTt = 32;  // lookups per warp task
+
+template <int GT, int U, int MINB, bool CHECK>
+__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kLPTt - 1) / kLPTt;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t warps_per_block = blockDim.x >> 5;
+  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
+  const uint32_t nw = gridDim.x * warps_per_block;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nw) {
+    while (task >= S.toff[m + 1]) ++m;
+    const uint32_t slot = (task - S.toff[m]) * kLPTt + lane;
+    const bool valid = slot < S.cnt[m];
+    LookupRec rec{0.5, 0u, 0};
+    if (valid) rec = P.recs[S.off[m] + slot];
+    const double p = rec.p;
+    const int nn = S.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    // per-lane view of the index structure for this lookup's energy
+    const int32_t* colbase = nullptr;  // unionized, column layout: IGT + u
+    RowView<GT> rv(P, valid ? rec.gidx : 0);
+    if (GT == XS_GRID_UNIONIZED && !P.index) colbase = P.index_t + (valid ? rec.gidx : 0);
+
+    auto bracket = [&](const MatEntry& me) -> int32_t {
+      if (GT == XS_GRID_UNIONIZED) {
+        if (colbase) return __ldg(colbase + static_cast<int64_t>(me.n) * P.NU);
+        return __ldg(rv.r0 + me.n);
+      }
+      return rv.bracket(P, me.n, me.noff, p);
+    };
+
+    double M0 = 0.0, M1 = 0.0, M2 = 0.0, M3 = 0.0, M4 = 0.0;
+    int32_t knext[U];
+#pragma unroll
+    for (int t = 0; t < U; ++t) knext[t] = t < nn ? bracket(row[t]) : 0;
+    for (int j0 = 0; j0 < nn; j0 += U) {
+      int32_t kcur[U];
+#pragma unroll
+      for (int t = 0; t < U; ++t) kcur[t] = knext[t];
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + U + t;
+        knext[t] = j < nn ? bracket(row[j]) : 0;
+      }
+      double2 c[U][6];
+      double cc[U];
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + t;
+        const MatEntry me = row[j < nn ? j : 0];
+        cc[t] = me.conc;
+        const uint32_t off = j < nn ? me.noff + static_cast<uint32_t>(kcur[t]) : 0u;
+        const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
+#pragma unroll
+        for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
+      }
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        if (j0 + t < nn) {  // warp-uniform
+          // lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5]
+          const double an = dsub(c[t][3].x, p), bd = dsub(c[t][3].x, c[t][0].x);
+          double f = div_nr(an, bd);
+          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+          const double x0 = dsub(c[t][3].y, dmul(f, dsub(c[t][3].y, c[t][0].y)));
+          const double x1 = dsub(c[t][4].x, dmul(f, dsub(c[t][4].x, c[t][1].x)));
+          const double x2 = dsub(c[t][4].y, dmul(f, dsub(c[t][4].y, c[t][1].y)));
+          const double x3 = dsub(c[t][5].x, dmul(f, dsub(c[t][5].x, c[t][2].x)));
+          const double x4 = dsub(c[t][5].y, dmul(f, dsub(c[t][5].y, c[t][2].y)));
+          M0 = dadd(M0, dmul(x0, cc[t]));
+          M1 = dadd(M1, dmul(x1, cc[t]));
+          M2 = dadd(M2, dmul(x2, cc[t]));
+          M3 = dadd(M3, dmul(x3, cc[t]));
+          M4 = dadd(M4, dmul(x4, cc[t]));
+        }
+      }
+    }
+    if (valid) {
+      const double M[5] = {M0, M1, M2, M3, M4};
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[c] > mx) {
+          mx = M[c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[rec.idx] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(rec.idx) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
+  if (lane == 0) {
+    s_red[0][threadIdx.x >> 5] = acc_v;
+    s_red[1][threadIdx.x >> 5] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (uint32_t w = 0; w < warps_per_block; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -797,6 +960,7 @@ static Params make_params(const DeviceGrid& g) {
   P.UB = g.UB;
   P.UBn = g.UBn;
   P.index = g.index;
+  P.index_t = g.index_t;
   P.B = g.B;
   P.du = g.du;
   P.num_nucs = g.num_nucs;
@@ -847,9 +1011,44 @@ static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStr
   }
 }
 
+template <int GT, int U, int MINB, bool CHECK>
+static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
+  auto kern = k_gather_t<GT, U, MINB, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
+template <int GT, bool CHECK>
+static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  switch (g.unroll) {
+    case 1: return launch_gather_t<GT, 1, 3, CHECK>(g, P, st);
+    case 3: return launch_gather_t<GT, 2, 2, CHECK>(g, P, st);
+    case 4: return launch_gather_t<GT, 3, 2, CHECK>(g, P, st);
+    default: return launch_gather_t<GT, 2, 3, CHECK>(g, P, st);
+  }
+}
+
+// Kernel choice: energy-sorted batches use the thread-per-lookup kernel;
+// unsorted batches the 3-lanes-per-lookup kernel, which needs the row
+// layout of the unionized index grid (a column-only grid falls back to the
+// thread-per-lookup kernel).
 template <int GT>
-static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool sorted,
+                                   cudaStream_t st) {
   const bool check = P.in_energy != nullptr || !g.dyadic63;
+  const bool thread_kernel = sorted || (GT == XS_GRID_UNIONIZED && !g.index);
+  if (thread_kernel)
+    return check ? launch_gather_tv<GT, true>(g, P, st) : launch_gather_tv<GT, false>(g, P, st);
   return check ? launch_gather_v<GT, true>(g, P, st) : launch_gather_v<GT, false>(g, P, st);
 }
 
@@ -913,7 +1112,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   }
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   mark(2);
-  e = launch_gather_u<GT>(g, P, st);
+  e = launch_gather_u<GT>(g, P, binned, st);
   launched(1);
   mark(3);
   return e;

@@ -215,6 +215,20 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   G.lookup_seed = d->lookup_seed;
   G.dyadic63 = dyadic;
   G.NU = d->grid_type == XS_GRID_UNIONIZED ? static_cast<int64_t>(I) * N : 0;
+  if (d->index_layout < 0 || d->index_layout > 3)
+    return fail(XS_ERR_INVALID_ARG, "index_layout must be XS_INDEX_AUTO/ROW/COL/BOTH");
+  if (G.NU) {
+    int lay = d->index_layout;
+    if (lay == XS_INDEX_AUTO) {
+      size_t free_b = 0, total_b = 0;
+      cudaMemGetInfo(&free_b, &total_b);
+      const double one = static_cast<double>(G.NU) * I * 4.0;
+      lay = (2.0 * one <= 0.45 * static_cast<double>(free_b)) ? XS_INDEX_BOTH : XS_INDEX_COL;
+    }
+    G.index_layout = lay;
+  } else {
+    G.index_layout = d->grid_type == XS_GRID_HASH ? XS_INDEX_ROW : 0;
+  }
   G.index_len = d->grid_type == XS_GRID_UNIONIZED ? G.NU * I
                 : d->grid_type == XS_GRID_HASH    ? static_cast<int64_t>(G.B) * I
                                                   : 0;
@@ -227,6 +241,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cudaFree(G.U);
     cudaFree(G.UB);
     cudaFree(G.index);
+    cudaFree(G.index_t);
     cudaFree(G.num_nucs);
     cudaFree(G.mats);
     cudaFree(G.concs);
@@ -235,7 +250,10 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   cudaError_t e = cudaMalloc(&G.grid, grid_bytes);
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.UB, (static_cast<size_t>(G.UBn) + 1) * 4);
-  if (e == cudaSuccess && G.index_len) e = cudaMalloc(&G.index, G.index_len * sizeof(int32_t));
+  if (e == cudaSuccess && G.index_len && (G.index_layout & XS_INDEX_ROW))
+    e = cudaMalloc(&G.index, G.index_len * sizeof(int32_t));
+  if (e == cudaSuccess && G.NU && (G.index_layout & XS_INDEX_COL))
+    e = cudaMalloc(&G.index_t, G.index_len * sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&G.num_nucs, d->n_mats * sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&G.mats, tab * sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&G.concs, tab * sizeof(double));
@@ -243,7 +261,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cleanup();
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
-  G.device_bytes = grid_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 + d->n_mats * 4 + tab * 12;
+  G.device_bytes = grid_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
   e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
@@ -252,7 +270,8 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
     e = build_union_grid(G, G.U, st);
     if (e == cudaSuccess) e = build_union_table(G, st);
-    if (e == cudaSuccess) e = build_index_grid(G, st);
+    if (e == cudaSuccess && G.index) e = build_index_grid(G, st);
+    if (e == cudaSuccess && G.index_t) e = build_index_grid_t(G, st);
   }
   if (e == cudaSuccess && G.grid_type == XS_GRID_HASH) e = build_hash_grid(G, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -280,7 +299,7 @@ xs_status xs_init_grid(const xs_grid_spec* spec, int device, void* cuda_stream, 
   if (!spec || !out) return fail(XS_ERR_INVALID_ARG, "NULL spec/out");
   *out = nullptr;
   if (spec->abi_version != XS_ABI_VERSION) return fail(XS_ERR_INVALID_ARG, "abi_version mismatch");
-  if (spec->reserved0 != 0) return fail(XS_ERR_INVALID_ARG, "reserved0 must be 0");
+
   const int32_t I = spec->n_isotopes;
   const int64_t N = spec->n_gridpoints;
   const int32_t mx = xsgen_max_num_nucs(I, spec->material_rule);
@@ -313,6 +332,7 @@ xs_status xs_init_grid(const xs_grid_spec* spec, int device, void* cuda_stream, 
   d.grid_type = spec->grid_type;
   d.hash_bins = spec->hash_bins;
   d.lookup_seed = spec->lookup_seed;
+  d.index_layout = spec->index_layout;
   return init_common(&d, device, static_cast<cudaStream_t>(cuda_stream), out);
 }
 
@@ -321,6 +341,7 @@ xs_status xs_init_grid_data(const xs_grid_data* data, int device, void* cuda_str
   if (!data || !out) return fail(XS_ERR_INVALID_ARG, "NULL data/out");
   *out = nullptr;
   if (data->abi_version != XS_ABI_VERSION) return fail(XS_ERR_INVALID_ARG, "abi_version mismatch");
+  if (data->reserved0 != 0) return fail(XS_ERR_INVALID_ARG, "reserved0 must be 0");
   return init_common(data, device, static_cast<cudaStream_t>(cuda_stream), out);
 }
 
@@ -338,6 +359,8 @@ xs_status xs_grid_get_info(const xs_grid* g, xs_grid_info* info) {
   info->index_grid_len = G.index_len;
   info->device_bytes = G.device_bytes;
   info->lookup_seed = G.lookup_seed;
+  info->index_layout = G.index_layout;
+  info->reserved0 = 0;
   return XS_OK;
 }
 
@@ -469,7 +492,12 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
   switch (table) {
     case XS_TABLE_NUCLIDE_GRID: src = G.grid; len = static_cast<uint64_t>(G.I) * G.N * 6; break;
     case XS_TABLE_UNION_ENERGY: src = G.U; len = G.NU; break;
-    case XS_TABLE_INDEX_GRID: src = G.index; len = G.index_len; es = 4; break;
+    case XS_TABLE_INDEX_GRID:
+      if (!G.index) return fail(XS_ERR_UNSUPPORTED, "grid has no row-layout index grid");
+      src = G.index; len = G.index_len; es = 4; break;
+    case XS_TABLE_INDEX_GRID_T:
+      if (!G.index_t) return fail(XS_ERR_UNSUPPORTED, "grid has no column-layout index grid");
+      src = G.index_t; len = G.index_len; es = 4; break;
     case XS_TABLE_NUM_NUCS: src = G.num_nucs; len = G.n_mats; es = 4; break;
     case XS_TABLE_MATS: src = G.mats; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; es = 4; break;
     case XS_TABLE_CONCS: src = G.concs; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; break;
@@ -541,6 +569,7 @@ void xs_free_grid(xs_grid* g) {
   cudaFree(g->d.U);
   cudaFree(g->d.UB);
   cudaFree(g->d.index);
+  cudaFree(g->d.index_t);
   cudaFree(g->d.num_nucs);
   cudaFree(g->d.mats);
   cudaFree(g->d.concs);

@@ -33,7 +33,9 @@ struct DeviceGrid {
   double* U = nullptr;       // [NU]
   int32_t* UB = nullptr;     // [UBn + 1]: UB[b] = ub(U, b / UBn)  (A3 search table)
   int32_t UBn = 0;           // power of two
-  int32_t* index = nullptr;  // IG [NU][I] or HG [B][I]
+  int32_t* index = nullptr;  // IG [NU][I] (row layout) or HG [B][I]; null if no row IG
+  int32_t* index_t = nullptr;  // IGT [I][NU] (column layout), unionized only
+  int32_t index_layout = 0;    // XS_INDEX_ROW | XS_INDEX_COL actually built
   int32_t* num_nucs = nullptr;
   int32_t* mats = nullptr;   // [n_mats][max_nucs]
   double* concs = nullptr;   // [n_mats][max_nucs]
@@ -74,6 +76,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
 // grid_build.cu
 cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st);
 cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st);
+cudaError_t build_index_grid_t(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st);
 cudaError_t init_constants();

@@ -22,7 +22,9 @@ XS_ABI_VERSION = 1
 XS_GRID_UNIONIZED, XS_GRID_NUCLIDE, XS_GRID_HASH = 0, 1, 2
 XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE = 0x1, 0x2, 0x4
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
- XS_TABLE_MATS, XS_TABLE_CONCS) = range(6)
+ XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T) = range(7)
+XS_INDEX_AUTO, XS_INDEX_ROW, XS_INDEX_COL, XS_INDEX_BOTH = 0, 1, 2, 3
+INDEX_LAYOUTS = {"auto": 0, "row": 1, "col": 2, "both": 3}
 STATUS = {0: "XS_OK", 1: "XS_ERR_INVALID_ARG", 2: "XS_ERR_OUT_OF_MEMORY", 3: "XS_ERR_CUDA",
           4: "XS_ERR_UNSUPPORTED", 5: "XS_ERR_STATE", 6: "XS_ERR_DATA"}
 GRID_TYPES = {"unionized": XS_GRID_UNIONIZED, "nuclide": XS_GRID_NUCLIDE, "hash": XS_GRID_HASH}
@@ -38,7 +40,7 @@ class xs_grid_spec(C.Structure):
     _fields_ = [("abi_version", C.c_uint32), ("n_isotopes", C.c_int32),
                 ("n_gridpoints", C.c_int64), ("grid_type", C.c_int32), ("hash_bins", C.c_int32),
                 ("grid_seed", C.c_uint64), ("conc_seed", C.c_uint64), ("lookup_seed", C.c_uint64),
-                ("material_rule", C.c_int32), ("reserved0", C.c_int32)]
+                ("material_rule", C.c_int32), ("index_layout", C.c_int32)]
 
 
 class xs_grid_data(C.Structure):
@@ -46,7 +48,8 @@ class xs_grid_data(C.Structure):
                 ("n_gridpoints", C.c_int64), ("nuclide_grid", C.c_void_p),
                 ("n_mats", C.c_int32), ("max_num_nucs", C.c_int32), ("num_nucs", C.c_void_p),
                 ("mats", C.c_void_p), ("concs", C.c_void_p), ("grid_type", C.c_int32),
-                ("hash_bins", C.c_int32), ("lookup_seed", C.c_uint64)]
+                ("hash_bins", C.c_int32), ("lookup_seed", C.c_uint64),
+                ("index_layout", C.c_int32), ("reserved0", C.c_int32)]
 
 
 class xs_grid_info(C.Structure):
@@ -54,7 +57,8 @@ class xs_grid_info(C.Structure):
                 ("grid_type", C.c_int32), ("hash_bins", C.c_int32), ("device", C.c_int32),
                 ("n_gridpoints", C.c_int64), ("n_union", C.c_int64),
                 ("index_grid_len", C.c_int64), ("device_bytes", C.c_uint64),
-                ("lookup_seed", C.c_uint64)]
+                ("lookup_seed", C.c_uint64), ("index_layout", C.c_int32),
+                ("reserved0", C.c_int32)]
 
 
 class xs_timing(C.Structure):
@@ -200,11 +204,13 @@ from .xs_presets import CONC_SEED, GRID_SEED, LOOKUP_SEED, PRESETS  # noqa: E402
 
 
 def make_spec(n_isotopes, n_gridpoints, grid_type="unionized", hash_bins=0, material_rule=0,
-              grid_seed=GRID_SEED, conc_seed=CONC_SEED, lookup_seed=LOOKUP_SEED, **_):
+              grid_seed=GRID_SEED, conc_seed=CONC_SEED, lookup_seed=LOOKUP_SEED,
+              index_layout="auto", **_):
     gt = GRID_TYPES[grid_type] if isinstance(grid_type, str) else int(grid_type)
+    il = INDEX_LAYOUTS[index_layout] if isinstance(index_layout, str) else int(index_layout)
     return xs_grid_spec(XS_ABI_VERSION, n_isotopes, n_gridpoints, gt,
                         hash_bins if gt == XS_GRID_HASH else 0, grid_seed, conc_seed,
-                        lookup_seed, material_rule, 0)
+                        lookup_seed, material_rule, il)
 
 
 class Grid:
@@ -232,7 +238,7 @@ class Grid:
 
     @classmethod
     def from_arrays(cls, grid, num_nucs, mats, concs, grid_type="unionized", hash_bins=0,
-                    lookup_seed=LOOKUP_SEED, device: int = 0):
+                    lookup_seed=LOOKUP_SEED, device: int = 0, index_layout="auto"):
         import numpy as np
         import torch
         grid = np.ascontiguousarray(grid, np.float64)
@@ -244,7 +250,9 @@ class Grid:
         gt = GRID_TYPES[grid_type] if isinstance(grid_type, str) else int(grid_type)
         d = xs_grid_data(XS_ABI_VERSION, I, N, grid.ctypes.data, mats.shape[0], mats.shape[1],
                          num_nucs.ctypes.data, mats.ctypes.data, concs.ctypes.data, gt,
-                         hash_bins, lookup_seed)
+                         hash_bins, lookup_seed,
+                         INDEX_LAYOUTS[index_layout] if isinstance(index_layout, str)
+                         else int(index_layout), 0)
         with torch.cuda.device(device):
             st = torch.cuda.current_stream().cuda_stream
             return cls(xs_init_grid_data(d, device, st), device)
@@ -347,8 +355,10 @@ class Grid:
         lens = {XS_TABLE_NUCLIDE_GRID: i.n_isotopes * i.n_gridpoints * 6,
                 XS_TABLE_UNION_ENERGY: i.n_union, XS_TABLE_INDEX_GRID: i.index_grid_len,
                 XS_TABLE_NUM_NUCS: i.n_mats, XS_TABLE_MATS: i.n_mats * i.max_num_nucs,
-                XS_TABLE_CONCS: i.n_mats * i.max_num_nucs}
-        dt = np.int32 if which in (XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS, XS_TABLE_MATS) \
+                XS_TABLE_CONCS: i.n_mats * i.max_num_nucs,
+                XS_TABLE_INDEX_GRID_T: i.index_grid_len if i.index_layout & 2 else 0}
+        dt = np.int32 if which in (XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS, XS_TABLE_MATS,
+                                   XS_TABLE_INDEX_GRID_T) \
             else np.float64
         if count is None:
             count = lens[which] - offset

@@ -68,11 +68,12 @@ def _compare(out, ref, mode_index=True):
 
 
 # ------------------------------------------------------------------- tiny --
-@pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4"])
+@pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
+                                     "sort-v1", "sort-v3", "sort-v4"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
-    if variant == "sort":
+    if variant.startswith("sort"):
         kw["sort"] = True
     if variant == "baseline":
         kw["baseline"] = True
@@ -95,6 +96,17 @@ def test_tiny_other_grids(X, grid_type, bins, sort):
     vs, out = _full_outputs(g, 0, 100_000, sort=sort)
     _compare(out, ref)
     assert vs == [S, 100_000]
+
+
+@pytest.mark.parametrize("layout", ["row", "col", "both"])
+@pytest.mark.parametrize("sort", [False, True])
+def test_index_layouts(X, layout, sort):
+    g = X.Grid.from_preset("tiny", index_layout=layout)
+    assert g.info.index_layout == X.INDEX_LAYOUTS[layout]
+    S, ref = oracle_for("tiny").run(7, 50_001, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
+    vs, out = _full_outputs(g, 7, 50_001, sort=sort)
+    _compare(out, ref)
+    assert vs == [S, 50_001]
 
 
 @pytest.mark.parametrize("first,count", [(0, 1), (5, 7), (123, 31), (999_999, 1001),
@@ -127,7 +139,11 @@ def test_tables_tiny(X):
     U = g.table(X.XS_TABLE_UNION_ENERGY)
     assert np.array_equal(U, o.union())
     IG = g.table(X.XS_TABLE_INDEX_GRID).reshape(o.NU, o.I)
-    assert np.array_equal(IG, o.index_grid_sweep())
+    ref_ig = o.index_grid_sweep()
+    assert np.array_equal(IG, ref_ig)
+    assert g.info.index_layout == X.XS_INDEX_BOTH
+    IGT = g.table(X.XS_TABLE_INDEX_GRID_T).reshape(o.I, o.NU)
+    assert np.array_equal(IGT, ref_ig.T)
     assert np.array_equal(g.table(X.XS_TABLE_MATS).reshape(12, -1), o.mats())
     assert np.array_equal(g.table(X.XS_TABLE_CONCS).reshape(12, -1), o.concs())
     assert np.array_equal(g.table(X.XS_TABLE_NUM_NUCS), o.num_nucs())

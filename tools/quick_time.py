@@ -32,8 +32,10 @@ def main():
         kw = {}
         if var.startswith("v"):
             g.set_param("variant", int(var[1:]))
-        if var == "sort":
+        if var.startswith("sort"):
             kw["sort"] = True
+            if var != "sort":
+                g.set_param("variant", int(var[-1]))
         if var == "baseline":
             kw["baseline"] = True
         for bps in [0]:
