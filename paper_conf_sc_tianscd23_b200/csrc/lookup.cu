@@ -682,18 +682,22 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
 }
 
 // --------------------------------------------- thread-per-lookup gather ---
-// k_gather_t: for energy-sorted batches (XS_FLAG_SORT).  A warp takes 32
-// consecutive lookups of one material bucket — after A2 they lie within a
-// few 1e-5 of each other in energy, so for each nuclide the 32 lanes read
-// the same or neighbouring record pairs (1-2 cache lines per 128-bit load
-// instruction) and, with the column-layout index grid IGT[n][u], neighbouring
-// index entries.  Each lane then owns its whole lookup: 6 x 128-bit loads of
-// the record pair, its own exact division, all five channels, list-order
-// accumulation — no shuffles, every lane's arithmetic useful.
-constexpr int kLPTt = 32;  // lookups per warp task
-
-template <int GT, int U, int MINB, bool CHECK>
+// k_gather_t: for energy-sorted batches (XS_FLAG_SORT).  A warp takes 32*R
+// consecutive lookups of one material bucket; lane l owns the R adjacent
+// lookups R*l .. R*l+R-1.  After A2 they lie within ~1e-5 of each other in
+// energy, so
+//   * for each nuclide the lane's R lookups almost always share one record
+//     pair: the lane loads the pair once (6 x 128-bit loads) and reloads
+//     only when a later lookup's bracket differs (rare, divergent);
+//   * the 32 lanes read the same or neighbouring pairs (1-2 cache lines per
+//     load instruction) and, with the column-layout index grid IGT[n][u],
+//     neighbouring index entries.
+// Each lane does its own exact division and all five channels, and
+// accumulates each lookup in list order: no shuffles, every lane's
+// arithmetic useful.  R = 1 is plain thread-per-lookup.
+template <int GT, int R, int U, int MINB, bool CHECK>
 __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
+  constexpr int kTask = 32 * R;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
   const int tab = P.n_mats * P.max_nucs;
@@ -715,7 +719,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
       S.cnt[m] = c;
       S.toff[m] = trun;
       run += c;
-      trun += (c + kLPTt - 1) / kLPTt;
+      trun += (c + kTask - 1) / kTask;
     }
     S.off[P.n_mats] = run;
     S.toff[P.n_mats] = trun;
@@ -733,88 +737,117 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
   int m = 0;
   for (uint32_t task = gw; task < total_tasks; task += nw) {
     while (task >= S.toff[m + 1]) ++m;
-    const uint32_t slot = (task - S.toff[m]) * kLPTt + lane;
-    const bool valid = slot < S.cnt[m];
-    LookupRec rec{0.5, 0u, 0};
-    if (valid) rec = P.recs[S.off[m] + slot];
-    const double p = rec.p;
+    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < S.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = P.recs[S.off[m] + slot0 + r];
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
     const int nn = S.num[m];
     const MatEntry* row = s_tab + m * P.max_nucs;
-    // per-lane view of the index structure for this lookup's energy
-    const int32_t* colbase = nullptr;  // unionized, column layout: IGT + u
-    RowView<GT> rv(P, valid ? rec.gidx : 0);
-    if (GT == XS_GRID_UNIONIZED && !P.index) colbase = P.index_t + (valid ? rec.gidx : 0);
 
-    auto bracket = [&](const MatEntry& me) -> int32_t {
+    // bracket k_n of lookup r (A4) through the grid's index structure
+    auto bracket = [&](const MatEntry& me, int r) -> int32_t {
       if (GT == XS_GRID_UNIONIZED) {
-        if (colbase) return __ldg(colbase + static_cast<int64_t>(me.n) * P.NU);
-        return __ldg(rv.r0 + me.n);
+        if (!P.index) return __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + gidx[r]);
+        return __ldg(P.index + static_cast<int64_t>(gidx[r]) * P.I + me.n);
       }
-      return rv.bracket(P, me.n, me.noff, p);
+      const RowView<GT> rv(P, gidx[r]);
+      return rv.bracket(P, me.n, me.noff, p[r]);
     };
 
-    double M0 = 0.0, M1 = 0.0, M2 = 0.0, M3 = 0.0, M4 = 0.0;
-    int32_t knext[U];
+    double M[R][5];
 #pragma unroll
-    for (int t = 0; t < U; ++t) knext[t] = t < nn ? bracket(row[t]) : 0;
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    int32_t knext[U][R];
+#pragma unroll
+    for (int t = 0; t < U; ++t)
+#pragma unroll
+      for (int r = 0; r < R; ++r) knext[t][r] = t < nn ? bracket(row[t], r) : 0;
+
     for (int j0 = 0; j0 < nn; j0 += U) {
-      int32_t kcur[U];
+      int32_t kcur[U][R];
 #pragma unroll
-      for (int t = 0; t < U; ++t) kcur[t] = knext[t];
+      for (int t = 0; t < U; ++t)
+#pragma unroll
+        for (int r = 0; r < R; ++r) kcur[t][r] = knext[t][r];
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + U + t;
-        knext[t] = j < nn ? bracket(row[j]) : 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) knext[t][r] = j < nn ? bracket(row[j], r) : 0;
       }
+      // A5: the pair of each nuclide's first lookup
       double2 c[U][6];
       double cc[U];
+      uint32_t noff[U];
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + t;
         const MatEntry me = row[j < nn ? j : 0];
         cc[t] = me.conc;
-        const uint32_t off = j < nn ? me.noff + static_cast<uint32_t>(kcur[t]) : 0u;
-        const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
+        noff[t] = j < nn ? me.noff : 0u;
+        const double2* pr = grid2 + static_cast<uint64_t>(noff[t] + (j < nn ? kcur[t][0] : 0)) * 3;
 #pragma unroll
         for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
       }
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         if (j0 + t < nn) {  // warp-uniform
-          // lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5]
-          const double an = dsub(c[t][3].x, p), bd = dsub(c[t][3].x, c[t][0].x);
-          double f = div_nr(an, bd);
-          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
-          const double x0 = dsub(c[t][3].y, dmul(f, dsub(c[t][3].y, c[t][0].y)));
-          const double x1 = dsub(c[t][4].x, dmul(f, dsub(c[t][4].x, c[t][1].x)));
-          const double x2 = dsub(c[t][4].y, dmul(f, dsub(c[t][4].y, c[t][1].y)));
-          const double x3 = dsub(c[t][5].x, dmul(f, dsub(c[t][5].x, c[t][2].x)));
-          const double x4 = dsub(c[t][5].y, dmul(f, dsub(c[t][5].y, c[t][2].y)));
-          M0 = dadd(M0, dmul(x0, cc[t]));
-          M1 = dadd(M1, dmul(x1, cc[t]));
-          M2 = dadd(M2, dmul(x2, cc[t]));
-          M3 = dadd(M3, dmul(x3, cc[t]));
-          M4 = dadd(M4, dmul(x4, cc[t]));
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (r > 0 && kcur[t][r] != kcur[t][r - 1]) {  // rare: a different pair
+              const double2* pr = grid2 + static_cast<uint64_t>(noff[t] + kcur[t][r]) * 3;
+#pragma unroll
+              for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
+            }
+            // A6 + A7: lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5]
+            const double an = dsub(c[t][3].x, p[r]), bd = dsub(c[t][3].x, c[t][0].x);
+            double f = div_nr(an, bd);
+            if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+            const double x0 = dsub(c[t][3].y, dmul(f, dsub(c[t][3].y, c[t][0].y)));
+            const double x1 = dsub(c[t][4].x, dmul(f, dsub(c[t][4].x, c[t][1].x)));
+            const double x2 = dsub(c[t][4].y, dmul(f, dsub(c[t][4].y, c[t][1].y)));
+            const double x3 = dsub(c[t][5].x, dmul(f, dsub(c[t][5].x, c[t][2].x)));
+            const double x4 = dsub(c[t][5].y, dmul(f, dsub(c[t][5].y, c[t][2].y)));
+            M[r][0] = dadd(M[r][0], dmul(x0, cc[t]));
+            M[r][1] = dadd(M[r][1], dmul(x1, cc[t]));
+            M[r][2] = dadd(M[r][2], dmul(x2, cc[t]));
+            M[r][3] = dadd(M[r][3], dmul(x3, cc[t]));
+            M[r][4] = dadd(M[r][4], dmul(x4, cc[t]));
+          }
         }
       }
     }
-    if (valid) {
-      const double M[5] = {M0, M1, M2, M3, M4};
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
       double mx = -1.0;
       int vi = 0;
 #pragma unroll
       for (int c = 0; c < 5; ++c)
-        if (M[c] > mx) {
-          mx = M[c];
+        if (M[r][c] > mx) {
+          mx = M[r][c];
           vi = c;
         }
       acc_v += static_cast<unsigned long long>(vi + 1);
       acc_n += 1;
-      if (P.out_v) P.out_v[rec.idx] = vi + 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
       if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(rec.idx) * 5;
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
 #pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[c];
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
       }
     }
   }
@@ -1011,10 +1044,10 @@ static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStr
   }
 }
 
-template <int GT, int U, int MINB, bool CHECK>
+template <int GT, int R, int U, int MINB, bool CHECK>
 static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
-  auto kern = k_gather_t<GT, U, MINB, CHECK>;
+  auto kern = k_gather_t<GT, R, U, MINB, CHECK>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -1030,11 +1063,12 @@ static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStr
 
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  switch (g.unroll) {
-    case 1: return launch_gather_t<GT, 1, 3, CHECK>(g, P, st);
-    case 3: return launch_gather_t<GT, 2, 2, CHECK>(g, P, st);
-    case 4: return launch_gather_t<GT, 3, 2, CHECK>(g, P, st);
-    default: return launch_gather_t<GT, 2, 3, CHECK>(g, P, st);
+  switch (g.unroll) {  // (lookups per lane R, nuclides per round U, min blocks)
+    case 1: return launch_gather_t<GT, 1, 3, 2, CHECK>(g, P, st);
+    case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
+    case 3: return launch_gather_t<GT, 2, 1, 3, CHECK>(g, P, st);
+    case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
+    default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
 
