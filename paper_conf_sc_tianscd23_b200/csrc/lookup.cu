@@ -236,13 +236,12 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
       if (GT == XS_GRID_HASH) gi = hash_bin(p, P.du, P.B);
       LookupRec r;
       r.p = p;
-      r.idx = i;
+      r.idx = i;  // BINNED: the rank within the (material, energy) bin instead
       r.gidx = valid ? gi : 0;
+      if (BINNED)
+        r.idx = atomicAdd(&P.bins[static_cast<uint32_t>(m) * kEnergyBins + energy_bin(p)], 1u);
       P.tmp[i] = r;
       P.mat8[i] = static_cast<uint8_t>(m);
-      if (BINNED) {
-        atomicAdd(&P.bins[static_cast<uint32_t>(m) * kEnergyBins + energy_bin(p)], 1u);
-      }
       if (P.out_E) P.out_E[i] = p;
       if (P.out_mat) P.out_mat[i] = valid ? m : (P.in_mat ? P.in_mat[i] : -1);
       if (P.out_gidx) P.out_gidx[i] = valid ? gi : -1;
@@ -343,9 +342,10 @@ __global__ void __launch_bounds__(1024) k_scan_apply(Params P) {
 }
 
 // k_scatter: place each record in its material bucket (plain: block-
-// aggregated per-material cursors) or (material, energy bin) slot (A2: one
-// atomic per lookup on the scanned histogram).  Order inside a bucket or
-// bin is arbitrary: results never depend on it.
+// aggregated per-material cursors) or (material, energy bin) slot (A2: the
+// scanned histogram gives the bin start, k_sample's atomic the rank within
+// the bin).  Order inside a bucket or bin is arbitrary: results never
+// depend on it.
 template <bool BINNED>
 __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
   __shared__ uint32_t s_off[kMaxMats + 2];
@@ -384,9 +384,11 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
       }
       rank[it] = 0;
       if (BINNED) {
-        if (ok)
-          rank[it] = atomicAdd(
-              &P.bins[static_cast<uint32_t>(mm[it]) * kEnergyBins + energy_bin(rec[it].p)], 1u);
+        if (ok) {
+          rank[it] = __ldg(P.bins + static_cast<uint32_t>(mm[it]) * kEnergyBins +
+                           energy_bin(rec[it].p)) + rec[it].idx;
+          rec[it].idx = static_cast<uint32_t>(i);
+        }
       } else {
         const uint32_t peers = __match_any_sync(0xffffffffu, mm[it]);
         const int leader = __ffs(peers) - 1;
@@ -805,22 +807,38 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         if (j0 + t < nn) {  // warp-uniform
+          // per pair: lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5];
+          // bd, its reciprocal and the channel differences are shared by
+          // every lookup of the lane that falls in this pair
+          double bd, rc, d0, d1, d2, d3, d4;
+          auto pair_terms = [&]() {
+            bd = dsub(c[t][3].x, c[t][0].x);
+            rc = recip_nr(bd);
+            d0 = dsub(c[t][3].y, c[t][0].y);
+            d1 = dsub(c[t][4].x, c[t][1].x);
+            d2 = dsub(c[t][4].y, c[t][1].y);
+            d3 = dsub(c[t][5].x, c[t][2].x);
+            d4 = dsub(c[t][5].y, c[t][2].y);
+          };
+          pair_terms();
 #pragma unroll
           for (int r = 0; r < R; ++r) {
             if (r > 0 && kcur[t][r] != kcur[t][r - 1]) {  // rare: a different pair
               const double2* pr = grid2 + static_cast<uint64_t>(noff[t] + kcur[t][r]) * 3;
 #pragma unroll
               for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
+              pair_terms();
             }
-            // A6 + A7: lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5]
-            const double an = dsub(c[t][3].x, p[r]), bd = dsub(c[t][3].x, c[t][0].x);
-            double f = div_nr(an, bd);
+            // A6: f = (hi.E - p) / (hi.E - lo.E), correctly rounded
+            const double an = dsub(c[t][3].x, p[r]);
+            double f = div_by_recip(an, bd, rc);
             if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
-            const double x0 = dsub(c[t][3].y, dmul(f, dsub(c[t][3].y, c[t][0].y)));
-            const double x1 = dsub(c[t][4].x, dmul(f, dsub(c[t][4].x, c[t][1].x)));
-            const double x2 = dsub(c[t][4].y, dmul(f, dsub(c[t][4].y, c[t][1].y)));
-            const double x3 = dsub(c[t][5].x, dmul(f, dsub(c[t][5].x, c[t][2].x)));
-            const double x4 = dsub(c[t][5].y, dmul(f, dsub(c[t][5].y, c[t][2].y)));
+            // x_c = hi_c - f * (hi_c - lo_c); A7: M_c += x_c * conc
+            const double x0 = dsub(c[t][3].y, dmul(f, d0));
+            const double x1 = dsub(c[t][4].x, dmul(f, d1));
+            const double x2 = dsub(c[t][4].y, dmul(f, d2));
+            const double x3 = dsub(c[t][5].x, dmul(f, d3));
+            const double x4 = dsub(c[t][5].y, dmul(f, d4));
             M[r][0] = dadd(M[r][0], dmul(x0, cc[t]));
             M[r][1] = dadd(M[r][1], dmul(x1, cc[t]));
             M[r][2] = dadd(M[r][2], dmul(x2, cc[t]));
@@ -1063,11 +1081,14 @@ static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStr
 
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  switch (g.unroll) {  // (lookups per lane R, nuclides per round U, min blocks)
+  // (lookups per lane R, nuclides per round U, min blocks); default measured
+  // best on B200: unionized (4, 1, 2), hash / nuclide (2, 1, 3)
+  int v = g.unroll;
+  if (v == 0) v = GT == XS_GRID_UNIONIZED ? 2 : 3;
+  switch (v) {
     case 1: return launch_gather_t<GT, 1, 3, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
     case 3: return launch_gather_t<GT, 2, 1, 3, CHECK>(g, P, st);
-    case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
