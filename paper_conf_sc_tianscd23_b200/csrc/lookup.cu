@@ -104,6 +104,7 @@ struct Params {
   LookupRec* tmp;   // [count] records in batch order
   uint8_t* mat8;    // [count] material (n_mats = invalid)
   uint32_t* partials;  // A2 scan: per-chunk sums -> offsets
+  uint32_t* perm;      // A2: batch positions in (material, energy) order (else null)
   // outputs
   double* out_M;
   double* out_E;
@@ -407,7 +408,12 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
 #pragma unroll
     for (int it = 0; it < kPrepItems; ++it) {
       const uint64_t i = c0 + static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
-      if (i < P.count) P.recs[BINNED ? rank[it] : s_base[mm[it]] + rank[it]] = rec[it];
+      if (i < P.count) {
+        if (BINNED)
+          P.perm[rank[it]] = static_cast<uint32_t>(i);  // 4-B writes into an L2-resident array
+        else
+          P.recs[s_base[mm[it]] + rank[it]] = rec[it];
+      }
     }
     if (!BINNED) __syncthreads();
   }
@@ -428,6 +434,18 @@ __device__ __forceinline__ int32_t bracket_of(const Params& P, int32_t gidx, int
 constexpr int kGatherThreads = 256;
 constexpr int kG = 3;                 // lanes per lookup
 constexpr int kLPT = 32 / kG;         // lookups per warp task (10)
+
+// Record at bucket position pos: A2 batches go through the permutation
+// (tmp holds the bin rank in idx; the batch index is the permutation value).
+__device__ __forceinline__ LookupRec load_rec(const Params& P, uint32_t pos) {
+  if (P.perm) {
+    const uint32_t i = __ldg(P.perm + pos);
+    LookupRec r = P.tmp[i];
+    r.idx = i;
+    return r;
+  }
+  return P.recs[pos];
+}
 
 struct alignas(16) MatEntry {
   double conc;
@@ -543,7 +561,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
     const bool valid = (g < kLPT) && (slot < S.cnt[m]);
     LookupRec rec{0.5, 0u, 0};
     if (valid) {
-      rec = P.recs[S.off[m] + slot];
+      rec = load_rec(P, S.off[m] + slot);
     }
     const double p = rec.p;
     const int nn = valid ? S.num[m] : 0;   // invalid lanes load nothing
@@ -748,7 +766,10 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
     for (int r = 0; r < R; ++r) {
       valid[r] = slot0 + r < S.cnt[m];
       LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = P.recs[S.off[m] + slot0 + r];
+      if (valid[r]) {
+        const uint32_t pos = S.off[m] + slot0 + r;
+        rec = load_rec(P, pos);
+      }
       p[r] = rec.p;
       gidx[r] = rec.gidx;
       idx[r] = rec.idx;
@@ -1151,6 +1172,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     e = cudaMemsetAsync(ws.bins, 0, static_cast<size_t>(g.n_mats + 1) * kEnergyBins * 4, st);
     if (e != cudaSuccess) return e;
     P.partials = ws.partials;
+    P.perm = ws.perm;
     const uint32_t nchunks = static_cast<uint32_t>(g.n_mats + 1) * (kEnergyBins / kScanChunk);
     k_sample<GT, true><<<nb, kPrepThreads, 0, st>>>(P);
     mark(1);

@@ -77,8 +77,9 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
   const size_t o_recs = take(count * sizeof(LookupRec));
   const size_t o_tmp = take(count * sizeof(LookupRec));
   const size_t o_mat8 = take(count);
-  size_t o_bins = 0, o_part = 0;
+  size_t o_bins = 0, o_part = 0, o_perm = 0;
   if (flags & XS_FLAG_SORT) {
+    o_perm = take(count * 4);
     o_bins = take(static_cast<size_t>(kMaxMats + 1) * kEnergyBins * 4);
     o_part = take(static_cast<size_t>(kMaxMats + 1) * (kEnergyBins / 4096) * 4);
   }
@@ -89,6 +90,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
     ws->recs = reinterpret_cast<LookupRec*>(b + o_recs);
     ws->bins = reinterpret_cast<uint32_t*>(b + o_bins);
     ws->partials = reinterpret_cast<uint32_t*>(b + o_part);
+    ws->perm = reinterpret_cast<uint32_t*>(b + o_perm);
     ws->tmp = reinterpret_cast<LookupRec*>(b + o_tmp);
     ws->mat8 = reinterpret_cast<uint8_t*>(b + o_mat8);
     ws->total = off;
@@ -232,9 +234,9 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   G.index_len = d->grid_type == XS_GRID_UNIONIZED ? G.NU * I
                 : d->grid_type == XS_GRID_HASH    ? static_cast<int64_t>(G.B) * I
                                                   : 0;
-  if (G.NU) {  // ~64 unionized energies per search-table bin
+  if (G.NU) {  // ~8 unionized energies per search-table bin
     G.UBn = 1024;
-    while (G.UBn < (1 << 22) && static_cast<int64_t>(G.UBn) * 64 < G.NU) G.UBn <<= 1;
+    while (G.UBn < (1 << 23) && static_cast<int64_t>(G.UBn) * 8 < G.NU) G.UBn <<= 1;
   }
   auto cleanup = [&]() {
     cudaFree(G.grid);

@@ -69,6 +69,7 @@ struct Workspace {
   LookupRec* tmp;     // [count] records in batch order
   uint8_t* mat8;      // [count]
   uint32_t* partials; // A2 scan: [(kMaxMats + 1) * kEnergyBins / 4096]
+  uint32_t* perm;     // A2: [count]
   size_t total;
 };
 size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws);
