@@ -793,25 +793,36 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
 #pragma unroll
       for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
 
-    int32_t knext[U][R];
+    // A4.  Unionized grid: every lookup reads its own index-grid entry
+    // (IGT[n][u]: the lane's R lookups hit neighbouring entries), prefetched
+    // one round ahead.  Hash / nuclide grids (whose A4 is a chain of
+    // dependent loads): the lane's first lookup runs the full search; each
+    // later lookup starts from the bracket before it and, when the pair's
+    // energies show it is not its own (E[k] <= p < E[k+1], clamped ends),
+    // walks to the neighbouring interval — an exact local search, so every
+    // lookup still gets k_n(p).
+    constexpr bool kAllIdx = GT == XS_GRID_UNIONIZED;
+    constexpr int RK = kAllIdx ? R : 1;
+    const int32_t kmax = static_cast<int32_t>(P.N - 2);
+    int32_t knext[U][RK];
 #pragma unroll
     for (int t = 0; t < U; ++t)
 #pragma unroll
-      for (int r = 0; r < R; ++r) knext[t][r] = t < nn ? bracket(row[t], r) : 0;
+      for (int r = 0; r < RK; ++r) knext[t][r] = t < nn ? bracket(row[t], r) : 0;
 
     for (int j0 = 0; j0 < nn; j0 += U) {
-      int32_t kcur[U][R];
+      int32_t kcur[U][RK];
 #pragma unroll
       for (int t = 0; t < U; ++t)
 #pragma unroll
-        for (int r = 0; r < R; ++r) kcur[t][r] = knext[t][r];
+        for (int r = 0; r < RK; ++r) kcur[t][r] = knext[t][r];
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const int j = j0 + U + t;
 #pragma unroll
-        for (int r = 0; r < R; ++r) knext[t][r] = j < nn ? bracket(row[j], r) : 0;
+        for (int r = 0; r < RK; ++r) knext[t][r] = j < nn ? bracket(row[j], r) : 0;
       }
-      // A5: the pair of each nuclide's first lookup
+      // A5: the record pair of each nuclide's first bracket
       double2 c[U][6];
       double cc[U];
       uint32_t noff[U];
@@ -831,6 +842,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
           // per pair: lo = (E, t | s, a | f, nf) = c[0..2], hi = c[3..5];
           // bd, its reciprocal and the channel differences are shared by
           // every lookup of the lane that falls in this pair
+          int32_t k = kcur[t][0];
           double bd, rc, d0, d1, d2, d3, d4;
           auto pair_terms = [&]() {
             bd = dsub(c[t][3].x, c[t][0].x);
@@ -844,11 +856,25 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
           pair_terms();
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (r > 0 && kcur[t][r] != kcur[t][r - 1]) {  // rare: a different pair
-              const double2* pr = grid2 + static_cast<uint64_t>(noff[t] + kcur[t][r]) * 3;
+            if (r > 0) {
+              int32_t kr;
+              if (kAllIdx) {
+                kr = kcur[t][kAllIdx ? r : 0];
+              } else {
+                kr = k;
+                if (valid[r]) {
+                  const double* rec = P.grid + static_cast<uint64_t>(noff[t]) * 6;
+                  while (kr > 0 && p[r] < rec_energy(rec, kr)) --kr;
+                  while (kr < kmax && p[r] >= rec_energy(rec, kr + 1)) ++kr;
+                }
+              }
+              if (kr != k) {  // rare: this lookup lies in another interval
+                k = kr;
+                const double2* pr = grid2 + static_cast<uint64_t>(noff[t] + k) * 3;
 #pragma unroll
-              for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
-              pair_terms();
+                for (int q = 0; q < 6; ++q) c[t][q] = __ldg(pr + q);
+                pair_terms();
+              }
             }
             // A6: f = (hi.E - p) / (hi.E - lo.E), correctly rounded
             const double an = dsub(c[t][3].x, p[r]);
@@ -1102,14 +1128,15 @@ static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStr
 
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  // (lookups per lane R, nuclides per round U, min blocks); default measured
-  // best on B200: unionized (4, 1, 2), hash / nuclide (2, 1, 3)
+  // (lookups per lane R, nuclides per round U, min blocks); measured best:
+  // unionized (4, 1, 2); hash / nuclide (2, 1, 3)
   int v = g.unroll;
   if (v == 0) v = GT == XS_GRID_UNIONIZED ? 2 : 3;
   switch (v) {
-    case 1: return launch_gather_t<GT, 1, 3, 2, CHECK>(g, P, st);
+    case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
     case 3: return launch_gather_t<GT, 2, 1, 3, CHECK>(g, P, st);
+    case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
