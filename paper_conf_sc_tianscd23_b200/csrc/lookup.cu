@@ -300,21 +300,22 @@ __global__ void __launch_bounds__(1024) k_scan_partial(Params P) {
 
 __global__ void __launch_bounds__(1024) k_scan_top(Params P, uint32_t nchunks) {
   constexpr uint32_t kPer = kEnergyBins / kScanChunk;
-  // nchunks <= 1024 * 4 is guaranteed by the workspace layout
-  uint32_t v[4];
+  constexpr int kMaxPer = 8;  // nchunks <= 8192 (65 materials x 64 chunks)
+  const uint32_t per = (nchunks + 1023) / 1024;
+  uint32_t v[kMaxPer];
   uint32_t sum = 0;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const uint32_t i = threadIdx.x * 4 + q;
-    v[q] = i < nchunks ? P.partials[i] : 0u;
+  for (int q = 0; q < kMaxPer; ++q) {
+    const uint32_t i = threadIdx.x * per + q;
+    v[q] = (q < static_cast<int>(per) && i < nchunks) ? P.partials[i] : 0u;
     sum += v[q];
   }
   uint32_t ex;
   block_excl_scan(sum, &ex);
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const uint32_t i = threadIdx.x * 4 + q;
-    if (i < nchunks) {
+  for (int q = 0; q < kMaxPer; ++q) {
+    const uint32_t i = threadIdx.x * per + q;
+    if (q < static_cast<int>(per) && i < nchunks) {
       P.partials[i] = ex;
       if (v[q]) atomicAdd(&P.counts[i / kPer], v[q]);
       ex += v[q];
@@ -940,6 +941,213 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
   }
 }
 
+// ------------------------------------------ pipelined sorted gather -------
+// k_gather_p: k_gather_t with a two-stage software pipeline over the
+// nuclide list: while nuclide j is interpolated, the record pair of j+1 is
+// already in flight and the index entries of j+2 are being read, so the
+// pair-load latency (the dominant stall of k_gather_t in ncu's source view)
+// overlaps a full nuclide of arithmetic.
+template <int GT, int R, int MINB, bool CHECK>
+__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_p(Params P) {
+  constexpr int kTask = 32 * R;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t warps_per_block = blockDim.x >> 5;
+  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
+  const uint32_t nw = gridDim.x * warps_per_block;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+  const int32_t kmax = static_cast<int32_t>(P.N - 2);
+  constexpr bool kAllIdx = GT == XS_GRID_UNIONIZED;
+  constexpr int RK = kAllIdx ? R : 1;
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nw) {
+    while (task >= S.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < S.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, S.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+    const int nn = S.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+
+    auto bracket = [&](const MatEntry& me, int r) -> int32_t {
+      if (GT == XS_GRID_UNIONIZED) {
+        if (!P.index) return __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + gidx[r]);
+        return __ldg(P.index + static_cast<int64_t>(gidx[r]) * P.I + me.n);
+      }
+      const RowView<GT> rv(P, gidx[r]);
+      return rv.bracket(P, me.n, me.noff, p[r]);
+    };
+    auto load_pair = [&](double2 (&c)[6], uint32_t off) {
+      const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
+#pragma unroll
+      for (int q = 0; q < 6; ++q) c[q] = __ldg(pr + q);
+    };
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    // pipeline state: kA = brackets of nuclide j+1, kB = of j+2, cN = pair of j+1
+    int32_t kA[RK], kB[RK];
+    double2 cN[6];
+#pragma unroll
+    for (int r = 0; r < RK; ++r) {
+      kA[r] = bracket(row[0], r);
+      kB[r] = nn > 1 ? bracket(row[1], r) : 0;
+    }
+    load_pair(cN, row[0].noff + static_cast<uint32_t>(kA[0]));
+
+    for (int j = 0; j < nn; ++j) {
+      double2 c[6];
+#pragma unroll
+      for (int q = 0; q < 6; ++q) c[q] = cN[q];
+      int32_t kc[RK];
+#pragma unroll
+      for (int r = 0; r < RK; ++r) {
+        kc[r] = kA[r];
+        kA[r] = kB[r];
+      }
+      const MatEntry me = row[j];
+      if (j + 1 < nn) load_pair(cN, row[j + 1].noff + static_cast<uint32_t>(kA[0]));
+      if (j + 2 < nn) {
+#pragma unroll
+        for (int r = 0; r < RK; ++r) kB[r] = bracket(row[j + 2], r);
+      }
+      // A6 + A7 for nuclide j (see k_gather_t)
+      int32_t k = kc[0];
+      double bd, rc, d0, d1, d2, d3, d4;
+      auto pair_terms = [&]() {
+        bd = dsub(c[3].x, c[0].x);
+        rc = recip_nr(bd);
+        d0 = dsub(c[3].y, c[0].y);
+        d1 = dsub(c[4].x, c[1].x);
+        d2 = dsub(c[4].y, c[1].y);
+        d3 = dsub(c[5].x, c[2].x);
+        d4 = dsub(c[5].y, c[2].y);
+      };
+      pair_terms();
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (r > 0) {
+          int32_t kr;
+          if (kAllIdx) {
+            kr = kc[kAllIdx ? r : 0];
+          } else {
+            kr = k;
+            if (valid[r]) {
+              const double* rec = P.grid + static_cast<uint64_t>(me.noff) * 6;
+              while (kr > 0 && p[r] < rec_energy(rec, kr)) --kr;
+              while (kr < kmax && p[r] >= rec_energy(rec, kr + 1)) ++kr;
+            }
+          }
+          if (kr != k) {  // rare: this lookup lies in another interval
+            k = kr;
+            load_pair(c, me.noff + static_cast<uint32_t>(k));
+            pair_terms();
+          }
+        }
+        const double an = dsub(c[3].x, p[r]);
+        double f = div_by_recip(an, bd, rc);
+        if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+        const double x0 = dsub(c[3].y, dmul(f, d0));
+        const double x1 = dsub(c[4].x, dmul(f, d1));
+        const double x2 = dsub(c[4].y, dmul(f, d2));
+        const double x3 = dsub(c[5].x, dmul(f, d3));
+        const double x4 = dsub(c[5].y, dmul(f, d4));
+        M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
+        M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
+        M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
+        M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
+        M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
+  if (lane == 0) {
+    s_red[0][threadIdx.x >> 5] = acc_v;
+    s_red[1][threadIdx.x >> 5] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (uint32_t w = 0; w < warps_per_block; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -1126,6 +1334,23 @@ static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
+template <int GT, int R, int MINB, bool CHECK>
+static cudaError_t launch_gather_p(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
+  auto kern = k_gather_p<GT, R, MINB, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // (lookups per lane R, nuclides per round U, min blocks); measured best:
@@ -1137,6 +1362,10 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
     case 3: return launch_gather_t<GT, 2, 1, 3, CHECK>(g, P, st);
     case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
+    case 5: return launch_gather_p<GT, 4, 1, CHECK>(g, P, st);
+    case 6: return launch_gather_p<GT, 4, 2, CHECK>(g, P, st);
+    case 7: return launch_gather_p<GT, 2, 2, CHECK>(g, P, st);
+    case 8: return launch_gather_p<GT, 2, 3, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }

@@ -66,7 +66,8 @@ struct DeviceGuard {
 
 static size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
 
-size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws) {
+size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* base,
+                        Workspace* ws) {
   size_t off = 0;
   auto take = [&](size_t bytes) {
     size_t o = off;
@@ -80,8 +81,8 @@ size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* w
   size_t o_bins = 0, o_part = 0, o_perm = 0;
   if (flags & XS_FLAG_SORT) {
     o_perm = take(count * 4);
-    o_bins = take(static_cast<size_t>(kMaxMats + 1) * kEnergyBins * 4);
-    o_part = take(static_cast<size_t>(kMaxMats + 1) * (kEnergyBins / 4096) * 4);
+    o_bins = take(static_cast<size_t>(n_mats + 1) * kEnergyBins * 4);
+    o_part = take(static_cast<size_t>(n_mats + 1) * (kEnergyBins / 4096) * 4);
   }
   if (ws) {
     char* b = static_cast<char*>(base);
@@ -134,8 +135,8 @@ static size_t staging_layout(uint64_t count, void* base, Staging* s) {
   return off;
 }
 
-static size_t total_workspace(uint64_t count, uint32_t flags) {
-  size_t w = workspace_layout(count, flags, nullptr, nullptr);
+static size_t total_workspace(uint64_t count, uint32_t flags, int32_t n_mats) {
+  size_t w = workspace_layout(count, flags, n_mats, nullptr, nullptr);
   if (flags & XS_FLAG_HOST_IO) w += staging_layout(count, nullptr, nullptr);
   return w;
 }
@@ -369,7 +370,7 @@ xs_status xs_grid_get_info(const xs_grid* g, xs_grid_info* info) {
 xs_status xs_workspace_size(const xs_grid* g, uint64_t count, uint32_t flags, size_t* bytes) {
   if (!g || !bytes) return fail(XS_ERR_INVALID_ARG, "NULL grid/bytes");
   if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
-  *bytes = total_workspace(count, flags);
+  *bytes = total_workspace(count, flags, g->d.n_mats);
   return XS_OK;
 }
 
@@ -383,7 +384,7 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE))
     return fail(XS_ERR_INVALID_ARG, "unknown flag bits");
   if (count == 0) return XS_OK;
-  const size_t need = total_workspace(count, flags);
+  const size_t need = total_workspace(count, flags, g->d.n_mats);
   if (!workspace || ws_bytes < need)
     return fail(XS_ERR_INVALID_ARG, "workspace too small: need " + std::to_string(need) + " bytes");
   if (reinterpret_cast<uintptr_t>(workspace) & 255)
@@ -392,7 +393,7 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   if (!guard.ok) return fail(XS_ERR_CUDA, "cudaSetDevice failed");
   cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
   Workspace ws;
-  const size_t wbytes = workspace_layout(count, flags, workspace, &ws);
+  const size_t wbytes = workspace_layout(count, flags, g->d.n_mats, workspace, &ws);
   LookupArgs a;
   a.first_id = first_id;
   a.count = static_cast<uint32_t>(count);
@@ -518,7 +519,7 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
-    if (value < 0 || value > 4) return fail(XS_ERR_INVALID_ARG, "variant in [0,4]");
+    if (value < 0 || value > 8) return fail(XS_ERR_INVALID_ARG, "variant in [0,8]");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "blocks_per_sm")) {
     if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");

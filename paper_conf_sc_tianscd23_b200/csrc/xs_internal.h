@@ -17,7 +17,7 @@ struct alignas(16) LookupRec {
 };
 
 constexpr int kMaxMats = 64;  // materials supported by the bucketed kernels
-constexpr uint32_t kEnergyBins = 65536;  // A2: energy bins per material
+constexpr uint32_t kEnergyBins = 1u << 18;  // A2: energy bins per material
 
 struct DeviceGrid {
   int device = 0;
@@ -65,14 +65,15 @@ struct Workspace {
   uint32_t* counts;   // [kMaxMats + 1]
   uint32_t* cursor;   // [kMaxMats + 1]
   LookupRec* recs;    // [count]
-  uint32_t* bins;     // A2: [(kMaxMats + 1) * kEnergyBins]
+  uint32_t* bins;     // A2: [(n_mats + 1) * kEnergyBins]
   LookupRec* tmp;     // [count] records in batch order
   uint8_t* mat8;      // [count]
-  uint32_t* partials; // A2 scan: [(kMaxMats + 1) * kEnergyBins / 4096]
+  uint32_t* partials; // A2 scan: [(n_mats + 1) * kEnergyBins / 4096]
   uint32_t* perm;     // A2: [count]
   size_t total;
 };
-size_t workspace_layout(uint64_t count, uint32_t flags, void* base, Workspace* ws);
+size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* base,
+                        Workspace* ws);
 
 // grid_build.cu
 cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st);

@@ -69,7 +69,8 @@ def _compare(out, ref, mode_index=True):
 
 # ------------------------------------------------------------------- tiny --
 @pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
-                                     "sort-v1", "sort-v3", "sort-v4"])
+                                     "sort-v1", "sort-v3", "sort-v4", "sort-v5", "sort-v6", "sort-v7",
+                                     "sort-v8"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
