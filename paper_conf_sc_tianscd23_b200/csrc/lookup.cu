@@ -941,6 +941,239 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
   }
 }
 
+// ------------------------------------------- windowed sorted gather -------
+// k_gather_w: k_gather_t (U = 1) where each lane first orders its R lookups
+// by energy and loads a three-record window (k, k+1, k+2) of the lowest
+// lookup's bracket k: the lane's other lookups almost always lie in pair
+// (k, k+1) or (k+1, k+2), so a straddled grid point costs arithmetic, not a
+// dependent reload (which k_gather_t's source-level profile shows as the
+// main stall).  The grid allocation carries one padding record so that
+// k+2 is always addressable.
+template <int GT, int R, int MINB, bool CHECK>
+__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_w(Params P) {
+  constexpr int kTask = 32 * R;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t warps_per_block = blockDim.x >> 5;
+  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
+  const uint32_t nw = gridDim.x * warps_per_block;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+  const int32_t kmax = static_cast<int32_t>(P.N - 2);
+  constexpr bool kAllIdx = GT == XS_GRID_UNIONIZED;
+  constexpr int RK = kAllIdx ? R : 1;
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nw) {
+    while (task >= S.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < S.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, S.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+    // order the lane's lookups by energy (valid ones first): an odd-even
+    // transposition network over R registers
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    const int nn = S.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+
+    auto bracket = [&](const MatEntry& me, int r) -> int32_t {
+      if (GT == XS_GRID_UNIONIZED) {
+        if (!P.index) return __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + gidx[r]);
+        return __ldg(P.index + static_cast<int64_t>(gidx[r]) * P.I + me.n);
+      }
+      const RowView<GT> rv(P, gidx[r]);
+      return rv.bracket(P, me.n, me.noff, p[r]);
+    };
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    int32_t knext[RK];
+#pragma unroll
+    for (int r = 0; r < RK; ++r) knext[r] = bracket(row[0], r);
+
+    for (int j = 0; j < nn; ++j) {
+      int32_t kc[RK];
+#pragma unroll
+      for (int r = 0; r < RK; ++r) {
+        kc[r] = knext[r];
+        knext[r] = j + 1 < nn ? bracket(row[j + 1], r) : 0;
+      }
+      const MatEntry me = row[j];
+      const int32_t kb = kc[0];  // bracket of the lane's lowest energy
+      // A5: window of records kb, kb+1, kb+2 (9 x 16 B)
+      double2 c[9];
+      {
+        const double2* pr = grid2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(kb)) * 3;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) c[q] = __ldg(pr + q);
+      }
+      // pair (kb, kb+1): shared terms
+      const double bdA = dsub(c[3].x, c[0].x);
+      const double rcA = recip_nr(bdA);
+      const double dA0 = dsub(c[3].y, c[0].y);
+      const double dA1 = dsub(c[4].x, c[1].x);
+      const double dA2 = dsub(c[4].y, c[1].y);
+      const double dA3 = dsub(c[5].x, c[2].x);
+      const double dA4 = dsub(c[5].y, c[2].y);
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        int32_t kr = kb;
+        if (r > 0) {
+          if (kAllIdx) {
+            kr = kc[kAllIdx ? r : 0];
+          } else if (valid[r] && kb < kmax && p[r] >= c[3].x) {
+            kr = (kb + 1 == kmax || p[r] < c[6].x) ? kb + 1 : kb + 2;  // kb+2: walk on below
+          }
+        }
+        double x0, x1, x2, x3, x4;
+        if (kr == kb) {
+          const double an = dsub(c[3].x, p[r]);
+          double f = div_by_recip(an, bdA, rcA);
+          if (CHECK && !div_in_range(an, bdA)) f = ddiv(an, bdA);
+          x0 = dsub(c[3].y, dmul(f, dA0));
+          x1 = dsub(c[4].x, dmul(f, dA1));
+          x2 = dsub(c[4].y, dmul(f, dA2));
+          x3 = dsub(c[5].x, dmul(f, dA3));
+          x4 = dsub(c[5].y, dmul(f, dA4));
+        } else {
+          // pair (kb+1, kb+2) from the window, or (rare) a reload further on
+          double2 lo[3], hi[3];
+          if (kr == kb + 1) {
+#pragma unroll
+            for (int q = 0; q < 3; ++q) {
+              lo[q] = c[3 + q];
+              hi[q] = c[6 + q];
+            }
+          } else {
+            if (!kAllIdx) {  // exact local walk from kb+1
+              const double* rec = P.grid + static_cast<uint64_t>(me.noff) * 6;
+              kr = kb + 1;
+              while (kr < kmax && p[r] >= rec_energy(rec, kr + 1)) ++kr;
+            }
+            const double2* pr = grid2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(kr)) * 3;
+#pragma unroll
+            for (int q = 0; q < 3; ++q) {
+              lo[q] = __ldg(pr + q);
+              hi[q] = __ldg(pr + 3 + q);
+            }
+          }
+          const double bd = dsub(hi[0].x, lo[0].x);
+          const double an = dsub(hi[0].x, p[r]);
+          double f = div_nr(an, bd);
+          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+          x0 = dsub(hi[0].y, dmul(f, dsub(hi[0].y, lo[0].y)));
+          x1 = dsub(hi[1].x, dmul(f, dsub(hi[1].x, lo[1].x)));
+          x2 = dsub(hi[1].y, dmul(f, dsub(hi[1].y, lo[1].y)));
+          x3 = dsub(hi[2].x, dmul(f, dsub(hi[2].x, lo[2].x)));
+          x4 = dsub(hi[2].y, dmul(f, dsub(hi[2].y, lo[2].y)));
+        }
+        M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
+        M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
+        M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
+        M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
+        M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
+  if (lane == 0) {
+    s_red[0][threadIdx.x >> 5] = acc_v;
+    s_red[1][threadIdx.x >> 5] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (uint32_t w = 0; w < warps_per_block; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // ------------------------------------------ pipelined sorted gather -------
 // k_gather_p: k_gather_t with a two-stage software pipeline over the
 // nuclide list: while nuclide j is interpolated, the record pair of j+1 is
@@ -1351,12 +1584,30 @@ static cudaError_t launch_gather_p(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
+template <int GT, int R, int MINB, bool CHECK>
+static cudaError_t launch_gather_w(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
+  auto kern = k_gather_w<GT, R, MINB, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  // (lookups per lane R, nuclides per round U, min blocks); measured best:
-  // unionized (4, 1, 2); hash / nuclide (2, 1, 3)
+  // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
+  // blocks); 5-6 pipelined; 7-8 windowed.  Measured best on B200 (large):
+  // unionized k_gather_t (4, 1, 2); hash / nuclide k_gather_w (R = 4).
   int v = g.unroll;
-  if (v == 0) v = GT == XS_GRID_UNIONIZED ? 2 : 3;
+  if (v == 0) v = GT == XS_GRID_UNIONIZED ? 2 : 7;
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
@@ -1364,8 +1615,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
     case 5: return launch_gather_p<GT, 4, 1, CHECK>(g, P, st);
     case 6: return launch_gather_p<GT, 4, 2, CHECK>(g, P, st);
-    case 7: return launch_gather_p<GT, 2, 2, CHECK>(g, P, st);
-    case 8: return launch_gather_p<GT, 2, 3, CHECK>(g, P, st);
+    case 7: return launch_gather_w<GT, 4, 2, CHECK>(g, P, st);
+    case 8: return launch_gather_w<GT, 2, 3, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }

@@ -250,7 +250,11 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cudaFree(G.concs);
   };
   const size_t grid_bytes = static_cast<size_t>(I) * N * 6 * sizeof(double);
-  cudaError_t e = cudaMalloc(&G.grid, grid_bytes);
+  // one padding record after the last nuclide: the windowed gather reads
+  // records k..k+2 with k <= N-2 (the padding is never interpolated)
+  cudaError_t e = cudaMalloc(&G.grid, grid_bytes + 6 * sizeof(double));
+  if (e == cudaSuccess) e = cudaMemsetAsync(reinterpret_cast<char*>(G.grid) + grid_bytes, 0,
+                                            6 * sizeof(double), st);
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.UB, (static_cast<size_t>(G.UBn) + 1) * 4);
   if (e == cudaSuccess && G.index_len && (G.index_layout & XS_INDEX_ROW))
