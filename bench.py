@@ -48,6 +48,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend (gloo: host-side A9, for single-GPU testing "
+                         "of the multi-rank path; ranks then share GPUs round-robin)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0,
                     help="target CPU seconds of the oracle sample")
     return ap.parse_args()
@@ -225,10 +228,14 @@ def run_ours(a, pre, cfg):
     rank, world, local = D.env_rank()
     if world != a.gpus:
         raise SystemExit(f"--gpus {a.gpus} but WORLD_SIZE={world}")
+    local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if a.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     sort = not a.no_sort
     L_cfg = a.lookups or pre["lookups"]
     first, L = D.shard_range(rank, world, L_cfg, a.scaling)
@@ -262,7 +269,10 @@ def run_ours(a, pre, cfg):
         vsum.zero_()
         g.lookup(first, L, sort=sort, vsum=vsum)
         if world > 1:
-            D.combine_vsum(vsum)          # A9
+            if a.backend == "nccl":
+                D.combine_vsum(vsum)      # A9 over NCCL (NVLink / NVSwitch)
+            else:
+                vsum.copy_(D.combine_vsum(vsum.cpu()))
 
     for _ in range(a.warmup):
         step()
@@ -286,7 +296,7 @@ def run_ours(a, pre, cfg):
     ms_local = ev0.elapsed_time(ev1)
     tm = g.timing_read()
     g.timing(False)
-    ms = D.max_over_ranks(ms_local, device=dev)
+    ms = D.max_over_ranks(ms_local, device=dev if a.backend == "nccl" else None)
     total_lookups = L * world * a.steps if a.scaling == "weak" else L_cfg * a.steps
     value = total_lookups / (ms / 1e3)
     vglob = [int(x) for x in vsum.cpu()]
@@ -317,7 +327,8 @@ def run_ours(a, pre, cfg):
                                   for k in ("ms_count", "ms_bucket", "ms_gather")},
             "gpu_launches": int(tm["kernel_launches"]),
             "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
-            "hash_matches_oracle": hash_check, "init_s": round(init_s, 2)}
+            "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
+            "grid_device_bytes": int(g.info.device_bytes)}
     # ------------------------------------------------------------- e2e leg
     if not a.no_e2e:
         e_host = res0["energy"].cpu().pin_memory()
@@ -331,7 +342,7 @@ def run_ours(a, pre, cfg):
             vs_h.zero_()
             g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)  # H2D, lookup, D2H
         dt = time.perf_counter() - t0
-        dt = D.max_over_ranks(dt, device=dev)
+        dt = D.max_over_ranks(dt, device=dev if a.backend == "nccl" else None)
         e2e_total = L * world * a.e2e_steps if a.scaling == "weak" else L_cfg * a.e2e_steps
         line["e2e"] = {"value": e2e_total / dt, "unit": "lookups/s",
                        "h2d_bytes_per_step": int(L * 12), "d2h_bytes_per_step": 16,
@@ -365,9 +376,10 @@ def main():
            "n_gridpoints": pre["n_gridpoints"], "grid": pre["grid_type"],
            "hash_bins": pre.get("hash_bins"), "lookups_per_gpu": per_gpu if a.scaling == "weak"
            else None, "lookups_total": per_gpu if a.scaling == "strong" else per_gpu * a.gpus,
-           "sort": ("A2 material+energy binning (65536 energy bins per material)"
+           "sort": ("A2 material+energy binning (2^18 energy bins per material)"
                     if not a.no_sort else "none"),
-           "l2": "not flushed: tables (5.9 GB for large) far exceed the 126 MB L2",
+           "l2": "not flushed: the resident tables (GBs, see grid_device_bytes) far exceed "
+                 "the 126 MB L2",
            "parallelism": f"dp{a.gpus} (lookup shards, grid replicated)"}
     if a.impl == "reference":
         return run_reference(a, pre, cfg)

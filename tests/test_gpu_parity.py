@@ -359,3 +359,30 @@ def test_shard_invariance_small(X):
         torch.cuda.synchronize()
         sums.append(vsum.cpu().tolist())
     assert all(s == [GOLDEN["small"]["sum_v"], L] for s in sums)
+
+
+def test_bench_multirank_path_on_one_gpu(X):
+    """bench.py's N > 1 path (shards, barrier, max-over-ranks, A9 all-reduce)
+    with two ranks sharing the box's GPU over gloo."""
+    import subprocess
+    import sys
+    root = os.path.dirname(HERE)
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+                        "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
+                        "29541", "bench.py", "--gpus", "2", "--backend", "gloo", "--config", "small",
+                        "--steps", "3", "--warmup", "3", "--no-cpu-baseline", "--no-e2e"],
+                       cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["lookups_per_step"] == 2 * 17_000_000
+    # ids [0, 34M): rank 0's shard is the golden small batch; the global sum
+    # must equal the oracle's over both shards
+    assert d["hash"] == (GOLDEN["small"]["sum_v"] + _small_second_shard_sum()) % 999983
+
+
+def _small_second_shard_sum():
+    o = oracle.Oracle.from_spec(68, 11303, conc_seed=CONC_SEED, material_rule=0, hash_bins=8192,
+                                nthreads=NT)
+    return o.run(17_000_000, 17_000_000, mode=oracle.HASH, nthreads=NT)
