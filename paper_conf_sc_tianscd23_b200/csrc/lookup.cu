@@ -1381,6 +1381,276 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_p(Params P) {
   }
 }
 
+// ------------------------------------------- TMA-staged sorted gather ------
+// k_gather_s: for energy-sorted batches.  A warp owns a task of 32*R
+// consecutive lookups of one material (lane l: lookups R*l..R*l+R-1, ordered
+// by energy).  Because the task is energy-sorted, for every nuclide n its
+// lookups' brackets lie in [k_lo, k_hi] with k_lo / k_hi the brackets of the
+// task's lowest / highest energy (A4 via the index grid for those two
+// lookups: IGT is monotone in u).  So per nuclide the warp needs one
+// contiguous window of records [k_lo, k_hi + 1].  One lane streams these
+// windows into shared memory with TMA bulk copies (cp.async.bulk +
+// mbarrier), D nuclides ahead; every lane then walks its lookups through the
+// window (an exact search: E[k] <= p < E[k+1], clamped) and interpolates
+// from shared memory.  Record pairs never wait in registers for global
+// memory and each warp reads each window from L2/HBM once.  Windows larger
+// than W records (sparse tasks) are read in place from global memory.
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
+  constexpr int kTask = 32 * R;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  // per warp: D windows of W records, D mbarriers, k_lo/k_hi per nuclide
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
+  const size_t win_bytes = static_cast<size_t>(D) * W * 48;
+  const size_t kw_bytes = ((static_cast<size_t>(P.max_nucs) * 2 * 4 + 15) / 16) * 16;
+  const size_t per_warp = win_bytes + kw_bytes + D * 8;
+  unsigned char* mine = wbase + per_warp * warp;
+  double2* s_win = reinterpret_cast<double2*>(mine);                  // [D][W*3]
+  int32_t* s_klo = reinterpret_cast<int32_t*>(mine + win_bytes);      // [max_nucs]
+  int32_t* s_khi = s_klo + P.max_nucs;
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(mine + win_bytes + kw_bytes);
+
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  if (lane == 0) {
+    for (int d = 0; d < D; ++d) mbar_init(&s_bar[d], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+  const int32_t kmax = static_cast<int32_t>(P.N - 2);
+  uint32_t phase = 0;  // parity bit per slot
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+    while (task >= S.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < S.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, S.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+    // order the lane's lookups by energy, valid ones first
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    // task extremes: lowest / highest energy (and unionized index) of the
+    // task's valid lookups (u is monotone in p)
+    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
+    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid[r]) {
+        phi = p[r];
+        uhi = gidx[r];
+      }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
+      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
+      plo = a < plo ? a : plo;
+      phi = b > phi ? b : phi;
+    }
+    ulo = __reduce_min_sync(0xffffffffu, ulo);
+    uhi = __reduce_max_sync(0xffffffffu, uhi);
+    const int nn = S.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    // A4 for the two extremes of every nuclide of the material
+    for (int j = lane; j < nn; j += 32) {
+      const MatEntry me = row[j];
+      int32_t klo, khi;
+      if (GT == XS_GRID_UNIONIZED) {
+        if (P.index_t) {
+          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
+          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
+        } else {
+          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
+          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
+        }
+      } else {
+        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
+        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
+        klo = rlo.bracket(P, me.n, me.noff, plo);
+        khi = rhi.bracket(P, me.n, me.noff, phi);
+      }
+      s_klo[j] = klo;
+      s_khi[j] = khi;
+    }
+    __syncwarp();
+    // A5 producer: window of nuclide j into slot j % D
+    auto issue = [&](int j) {
+      const int d = j % D;
+      const int32_t klo = s_klo[j], khi = s_khi[j];
+      const int32_t w = khi - klo + 2;  // records klo .. khi+1
+      if (w <= W) {
+        const double2* src = grid2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(klo)) * 3;
+        mbar_arrive_expect_tx(&s_bar[d], static_cast<uint32_t>(w) * 48u);
+        bulk_copy_g2s(s_win + d * W * 3, src, static_cast<uint32_t>(w) * 48u, &s_bar[d]);
+      } else {
+        mbar_arrive_expect_tx(&s_bar[d], 0u);  // read in place from global memory
+      }
+    };
+    if (lane == 0)
+      for (int j = 0; j < D && j < nn; ++j) issue(j);
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    for (int j = 0; j < nn; ++j) {
+      const int d = j % D;
+      mbar_wait(&s_bar[d], (phase >> d) & 1u);
+      phase ^= 1u << d;
+      const MatEntry me = row[j];
+      const int32_t klo = s_klo[j], khi = s_khi[j];
+      const double2* win = (khi - klo + 2 <= W)
+                               ? s_win + d * W * 3
+                               : grid2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(klo)) * 3;
+      int32_t k = klo;
+      double2 c[6];
+      auto load_pair = [&]() {
+        const double2* pr = win + (k - klo) * 3;
+#pragma unroll
+        for (int q = 0; q < 6; ++q) c[q] = pr[q];
+      };
+      load_pair();
+      double bd, rc, d0, d1, d2, d3, d4;
+      auto pair_terms = [&]() {
+        bd = dsub(c[3].x, c[0].x);
+        rc = recip_nr(bd);
+        d0 = dsub(c[3].y, c[0].y);
+        d1 = dsub(c[4].x, c[1].x);
+        d2 = dsub(c[4].y, c[1].y);
+        d3 = dsub(c[5].x, c[2].x);
+        d4 = dsub(c[5].y, c[2].y);
+      };
+      pair_terms();
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (valid[r]) {
+          // A4 (exact local search): advance to k_n(p) within [klo, khi]
+          if (k < khi && p[r] >= c[3].x) {
+            do {
+              ++k;
+            } while (k < khi && p[r] >= win[(k - klo + 1) * 3].x);
+            load_pair();
+            pair_terms();
+          }
+          const double an = dsub(c[3].x, p[r]);
+          double f = div_by_recip(an, bd, rc);
+          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+          const double x0 = dsub(c[3].y, dmul(f, d0));
+          const double x1 = dsub(c[4].x, dmul(f, d1));
+          const double x2 = dsub(c[4].y, dmul(f, d2));
+          const double x3 = dsub(c[5].x, dmul(f, d3));
+          const double x4 = dsub(c[5].y, dmul(f, d4));
+          M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
+          M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
+          M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
+          M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
+          M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
+        }
+      }
+      __syncwarp();  // every lane is done with slot d
+      if (lane == 0 && j + D < nn) issue(j + D);
+    }
+    (void)kmax;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -1601,13 +1871,35 @@ static cudaError_t launch_gather_w(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t win_bytes = static_cast<size_t>(D) * W * 48;
+  const size_t kw_bytes = ((static_cast<size_t>(g.max_nucs) * 2 * 4 + 15) / 16) * 16;
+  const size_t smem = sizeof(GatherSmem) +
+                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
+                      NW * (win_bytes + kw_bytes + D * 8);
+  auto kern = k_gather_s<GT, R, D, W, NW, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
-  // blocks); 5-6 pipelined; 7-8 windowed.  Measured best on B200 (large):
-  // unionized k_gather_t (4, 1, 2); hash / nuclide k_gather_w (R = 4).
+  // blocks); 5-6 pipelined; 7-8 windowed; 9-12 TMA-staged (R, stages D,
+  // window W records, warps per block).  Measured best on B200 (large and
+  // large-hash): k_gather_s (4, 4, 16, 16).
   int v = g.unroll;
-  if (v == 0) v = GT == XS_GRID_UNIONIZED ? 2 : 7;
+  if (v == 0) v = 9;
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
@@ -1617,6 +1909,10 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 6: return launch_gather_p<GT, 4, 2, CHECK>(g, P, st);
     case 7: return launch_gather_w<GT, 4, 2, CHECK>(g, P, st);
     case 8: return launch_gather_w<GT, 2, 3, CHECK>(g, P, st);
+    case 9: return launch_gather_s<GT, 4, 4, 16, 16, CHECK>(g, P, st);
+    case 10: return launch_gather_s<GT, 4, 6, 16, 12, CHECK>(g, P, st);
+    case 11: return launch_gather_s<GT, 2, 4, 16, 16, CHECK>(g, P, st);
+    case 12: return launch_gather_s<GT, 8, 4, 16, 8, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }

@@ -523,7 +523,7 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
-    if (value < 0 || value > 8) return fail(XS_ERR_INVALID_ARG, "variant in [0,8]");
+    if (value < 0 || value > 12) return fail(XS_ERR_INVALID_ARG, "variant in [0,12]");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "blocks_per_sm")) {
     if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");

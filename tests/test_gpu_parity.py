@@ -70,7 +70,7 @@ def _compare(out, ref, mode_index=True):
 # ------------------------------------------------------------------- tiny --
 @pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
                                      "sort-v1", "sort-v3", "sort-v4", "sort-v5", "sort-v6", "sort-v7",
-                                     "sort-v8"])
+                                     "sort-v8", "sort-v9", "sort-v10", "sort-v11", "sort-v12"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -78,8 +78,8 @@ def test_tiny_full_parity(X, variant):
         kw["sort"] = True
     if variant == "baseline":
         kw["baseline"] = True
-    if variant.startswith("v"):
-        g.set_param("variant", int(variant[-1]))
+    if variant.startswith("v") or variant.startswith("sort-v"):
+        g.set_param("variant", int(variant.split("v")[-1]))
     S, ref = oracle_for("tiny").run(0, 100_000, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
     vs, out = _full_outputs(g, 0, 100_000, **kw)
     _compare(out, ref)

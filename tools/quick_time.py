@@ -35,7 +35,7 @@ def main():
         if var.startswith("sort"):
             kw["sort"] = True
             if var != "sort":
-                g.set_param("variant", int(var[-1]))
+                g.set_param("variant", int(var.split("-v")[-1]))
         if var == "baseline":
             kw["baseline"] = True
         for bps in [0]:
