@@ -1408,7 +1408,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
   unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
   const size_t win_bytes = static_cast<size_t>(D) * W * 48;
   const size_t kw_bytes = ((static_cast<size_t>(P.max_nucs) * 2 * 4 + 15) / 16) * 16;
-  const size_t per_warp = win_bytes + kw_bytes + D * 8;
+  const size_t per_warp = win_bytes + kw_bytes + ((D * 8 + 15) / 16) * 16;
   unsigned char* mine = wbase + per_warp * warp;
   double2* s_win = reinterpret_cast<double2*>(mine);                  // [D][W*3]
   int32_t* s_klo = reinterpret_cast<int32_t*>(mine + win_bytes);      // [max_nucs]
@@ -1502,6 +1502,11 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
     }
     ulo = __reduce_min_sync(0xffffffffu, ulo);
     uhi = __reduce_max_sync(0xffffffffu, uhi);
+    // slots without a lookup take the lane's last valid energy (or the task
+    // minimum) so that the hot loop needs no validity test
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
     const int nn = S.num[m];
     const MatEntry* row = s_tab + m * P.max_nucs;
     // A4 for the two extremes of every nuclide of the material
@@ -1578,29 +1583,27 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
       pair_terms();
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        if (valid[r]) {
-          // A4 (exact local search): advance to k_n(p) within [klo, khi]
-          if (k < khi && p[r] >= c[3].x) {
-            do {
-              ++k;
-            } while (k < khi && p[r] >= win[(k - klo + 1) * 3].x);
-            load_pair();
-            pair_terms();
-          }
-          const double an = dsub(c[3].x, p[r]);
-          double f = div_by_recip(an, bd, rc);
-          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
-          const double x0 = dsub(c[3].y, dmul(f, d0));
-          const double x1 = dsub(c[4].x, dmul(f, d1));
-          const double x2 = dsub(c[4].y, dmul(f, d2));
-          const double x3 = dsub(c[5].x, dmul(f, d3));
-          const double x4 = dsub(c[5].y, dmul(f, d4));
-          M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
-          M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
-          M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
-          M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
-          M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
+        // A4 (exact local search): advance to k_n(p) within [klo, khi]
+        if (k < khi && p[r] >= c[3].x) {
+          do {
+            ++k;
+          } while (k < khi && p[r] >= win[(k - klo + 1) * 3].x);
+          load_pair();
+          pair_terms();
         }
+        const double an = dsub(c[3].x, p[r]);
+        double f = div_by_recip(an, bd, rc);
+        if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
+        const double x0 = dsub(c[3].y, dmul(f, d0));
+        const double x1 = dsub(c[4].x, dmul(f, d1));
+        const double x2 = dsub(c[4].y, dmul(f, d2));
+        const double x3 = dsub(c[5].x, dmul(f, d3));
+        const double x4 = dsub(c[5].y, dmul(f, d4));
+        M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
+        M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
+        M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
+        M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
+        M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
       }
       __syncwarp();  // every lane is done with slot d
       if (lane == 0 && j + D < nn) issue(j + D);
@@ -1877,7 +1880,7 @@ static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStr
   const size_t kw_bytes = ((static_cast<size_t>(g.max_nucs) * 2 * 4 + 15) / 16) * 16;
   const size_t smem = sizeof(GatherSmem) +
                       static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
-                      NW * (win_bytes + kw_bytes + D * 8);
+                      NW * (win_bytes + kw_bytes + ((D * 8 + 15) / 16) * 16);
   auto kern = k_gather_s<GT, R, D, W, NW, CHECK>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
@@ -1910,9 +1913,9 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 7: return launch_gather_w<GT, 4, 2, CHECK>(g, P, st);
     case 8: return launch_gather_w<GT, 2, 3, CHECK>(g, P, st);
     case 9: return launch_gather_s<GT, 4, 4, 16, 16, CHECK>(g, P, st);
-    case 10: return launch_gather_s<GT, 4, 6, 16, 12, CHECK>(g, P, st);
-    case 11: return launch_gather_s<GT, 2, 4, 16, 16, CHECK>(g, P, st);
-    case 12: return launch_gather_s<GT, 8, 4, 16, 8, CHECK>(g, P, st);
+    case 10: return launch_gather_s<GT, 4, 3, 16, 16, CHECK>(g, P, st);
+    case 11: return launch_gather_s<GT, 4, 6, 12, 16, CHECK>(g, P, st);
+    case 12: return launch_gather_s<GT, 4, 4, 12, 8, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
