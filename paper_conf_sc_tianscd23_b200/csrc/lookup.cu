@@ -105,6 +105,8 @@ struct Params {
   uint8_t* mat8;    // [count] material (n_mats = invalid)
   uint32_t* partials;  // A2 scan: per-chunk sums -> offsets
   uint32_t* perm;      // A2: batch positions in (material, energy) order (else null)
+  int need_gidx;       // k_sample must search u per lookup (else the staged gather
+                       // searches only each task's extreme energies)
   // outputs
   double* out_M;
   double* out_E;
@@ -144,6 +146,31 @@ __device__ __forceinline__ void write_invalid(const Params& P, uint32_t i) {
     for (int c = 0; c < 5; ++c)
       P.out_M[static_cast<uint64_t>(i) * 5 + c] = __longlong_as_double(0x7ff8000000000000LL);
   if (P.out_v) P.out_v[i] = 0;
+}
+
+// u = clamp(ub(U, p) - 1, 0, NU-2): the XSBench bisection loop started from
+// the equal-width table's range [UB[b] - 1, UB[b+1]] (the loop invariant
+// U[lo] <= p < U[hi] holds there, so the result is the full search's).
+__device__ __forceinline__ int32_t union_index_tab(const Params& P, double p) {
+  const double q = p * static_cast<double>(P.UBn);
+  const int32_t b = q > 0.0 ? (q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q) : P.UBn - 1) : 0;
+  const int64_t l = q > 0.0 ? static_cast<int64_t>(__ldg(P.UB + b)) - 1 : 0;  // p <= 0: from 0
+  int64_t lo = l < 0 ? 0 : (l > P.NU - 2 ? P.NU - 2 : l);
+  int64_t hi = P.NU - 1;
+  if (q < static_cast<double>(P.UBn)) {
+    const int64_t h = __ldg(P.UB + b + 1);
+    hi = h < P.NU - 1 ? h : P.NU - 1;
+  }
+  int64_t len = hi - lo;
+  while (len > 1) {
+    const int64_t mid = lo + (len >> 1);
+    if (__ldg(P.U + mid) > p)
+      hi = mid;
+    else
+      lo = mid;
+    len = hi - lo;
+  }
+  return static_cast<int32_t>(lo);
 }
 
 // k_sample: A1 + A3 in batch order.  Thread t of a block handles lookups
@@ -187,7 +214,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
         const int32_t b = q > 0.0 ? (q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q)
                                                                     : P.UBn - 1)
                                   : 0;
-        const int64_t l = static_cast<int64_t>(__ldg(P.UB + b)) - 1;
+        const int64_t l = q > 0.0 ? static_cast<int64_t>(__ldg(P.UB + b)) - 1 : 0;
         lo[it] = l < 0 ? 0 : (l > P.NU - 2 ? P.NU - 2 : l);
         if (q < static_cast<double>(P.UBn)) {  // p < 1: U[UB[b+1]] > p
           const int64_t h = __ldg(P.UB + b + 1);
@@ -196,7 +223,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
       }
     }
     if (!P.in_energy) __syncthreads();  // s_state is rewritten next chunk
-    if (GT == XS_GRID_UNIONIZED) {
+    if (GT == XS_GRID_UNIONIZED && P.need_gidx) {
       // XSBench grid_search loop on [lo, hi] (invariant U[lo] <= p < U[hi]),
       // the kPrepItems searches interleaved
       bool busy = true;
@@ -1500,8 +1527,14 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
       plo = a < plo ? a : plo;
       phi = b > phi ? b : phi;
     }
-    ulo = __reduce_min_sync(0xffffffffu, ulo);
-    uhi = __reduce_max_sync(0xffffffffu, uhi);
+    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
+      // A3 for the task's extreme energies (u is monotone in p)
+      ulo = union_index_tab(P, plo);
+      uhi = union_index_tab(P, phi);
+    } else {
+      ulo = __reduce_min_sync(0xffffffffu, ulo);
+      uhi = __reduce_max_sync(0xffffffffu, uhi);
+    }
     // slots without a lookup take the lane's last valid energy (or the task
     // minimum) so that the hot loop needs no validity test
 #pragma unroll
@@ -1971,6 +2004,10 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   if (e != cudaSuccess) return e;
   const bool binned = a.flags & XS_FLAG_SORT;
   const unsigned nb = grid_cap(a.count, kPrepThreads * kPrepItems, g.sm_count, 16);
+  // the staged gather (default for sorted batches) only needs u at each task's
+  // extreme energies; per-lookup u is searched when reported or otherwise used
+  const int variant = g.unroll;
+  P.need_gidx = (!binned || a.out.grid_index || (variant != 0 && variant < 9)) ? 1 : 0;
   P.tmp = ws.tmp;
   P.mat8 = ws.mat8;
   if (binned) {
