@@ -209,9 +209,11 @@ xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t
 xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
                        void* host_dst);
 
-/* Tuning knobs: "variant" (gather kernel shape: 0 = default, 1-4 = (nuclides
- * per round, min resident blocks) in {(3,3), (3,4), (6,2), (6,3)}) and
- * "blocks_per_sm" (0 = occupancy calculator).  INVALID_ARG for an
+/* Tuning knobs: "variant" (gather kernel: 0 = default, 1-12 = the kernel
+ * shapes listed in DESIGN.md §4), "blocks_per_sm" (0 = occupancy calculator)
+ * and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in
+ * chunks of this many lookups, overlapped with the lookups of the previous
+ * chunk; default 10^7, split evenly).  INVALID_ARG for an
  * unknown name or value.  Never changes results. */
 xs_status xs_set_param(xs_grid* g, const char* name, int64_t value);
 

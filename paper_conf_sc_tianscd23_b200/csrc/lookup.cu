@@ -1616,11 +1616,18 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
       pair_terms();
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        // A4 (exact local search): advance to k_n(p) within [klo, khi]
+        // A4 (exact local search): advance to k_n(p) within [klo, khi] by
+        // bisection on the window energies (E[k] <= p is known; k_n(p) <= khi)
         if (k < khi && p[r] >= c[3].x) {
-          do {
-            ++k;
-          } while (k < khi && p[r] >= win[(k - klo + 1) * 3].x);
+          int32_t lo = k + 1, hi = khi + 1;
+          while (hi - lo > 1) {
+            const int32_t mid = (lo + hi) >> 1;
+            if (win[(mid - klo) * 3].x <= p[r])
+              lo = mid;
+            else
+              hi = mid;
+          }
+          k = lo;
           load_pair();
           pair_terms();
         }

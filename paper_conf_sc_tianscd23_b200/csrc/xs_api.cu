@@ -3,6 +3,7 @@
 // grid_build.cu / lookup.cu; there is no host compute path and no fallback.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <array>
 #include <cstdio>
 #include <cstring>
@@ -19,6 +20,10 @@
 
 struct xs_grid {
   xs::DeviceGrid d;
+  // chunked host-input pipeline (XS_FLAG_HOST_IO)
+  uint64_t host_chunk = 10000000;  // host-input chunk (lookups), measured on B200 (large)
+  cudaStream_t copy_stream = nullptr;
+  std::vector<cudaEvent_t> chunk_ev;
   // per-phase event timing (xs_timing_enable / xs_timing_read)
   bool timing = false;
   std::vector<std::array<cudaEvent_t, 4>> ev;
@@ -417,11 +422,20 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   ++g->calls;
   Staging sg{};
   const bool host_io = flags & XS_FLAG_HOST_IO;
+  // host inputs larger than one chunk are uploaded chunk by chunk on a copy
+  // stream while the previous chunk is being looked up (each chunk is a
+  // batch of its own: same results, lookups never interact)
+  // equal chunks of at most host_chunk lookups
+  const uint64_t nch = (count + g->host_chunk - 1) / g->host_chunk;
+  const uint64_t chunk = (count + nch - 1) / nch;
+  const bool chunked = host_io && energy && nch > 1;
   if (host_io) {
     staging_layout(count, static_cast<char*>(workspace) + wbytes, &sg);
-    if (energy) {
+    if (energy && !chunked) {
       XS_TRY(cudaMemcpyAsync(sg.energy, energy, count * 8, cudaMemcpyHostToDevice, st), "H2D energy");
       XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * 4, cudaMemcpyHostToDevice, st), "H2D mat");
+    }
+    if (energy) {
       a.in_energy = sg.energy;
       a.in_mat = sg.mat;
     }
@@ -433,7 +447,45 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
     a.out.grid_index = out->grid_index ? sg.gidx : nullptr;
     a.out.verification = out->verification ? sg.v : nullptr;
   }
-  cudaError_t e = run_lookup(g->d, a, ws, st);
+  cudaError_t e = cudaSuccess;
+  if (!chunked) {
+    e = run_lookup(g->d, a, ws, st);
+  } else {
+    if (!g->copy_stream)
+      XS_TRY(cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking), "copy stream");
+    const uint64_t nchunks = (count + chunk - 1) / chunk;
+    while (g->chunk_ev.size() < nchunks + 1) {
+      cudaEvent_t ev;
+      XS_TRY(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming), "cudaEventCreate");
+      g->chunk_ev.push_back(ev);
+    }
+    // the copies may only start once earlier work on the caller's stream is done
+    XS_TRY(cudaEventRecord(g->chunk_ev[nchunks], st), "event");
+    XS_TRY(cudaStreamWaitEvent(g->copy_stream, g->chunk_ev[nchunks], 0), "wait");
+    for (uint64_t k = 0; k < nchunks; ++k) {
+      const uint64_t b = k * chunk, n = std::min(chunk, count - b);
+      XS_TRY(cudaMemcpyAsync(sg.energy + b, energy + b, n * 8, cudaMemcpyHostToDevice,
+                             g->copy_stream), "H2D energy");
+      XS_TRY(cudaMemcpyAsync(sg.mat + b, mat + b, n * 4, cudaMemcpyHostToDevice, g->copy_stream),
+             "H2D mat");
+      XS_TRY(cudaEventRecord(g->chunk_ev[k], g->copy_stream), "event");
+    }
+    LookupArgs c = a;
+    c.ev = nullptr;  // phase timing covers whole, unchunked batches only
+    for (uint64_t k = 0; k < nchunks && e == cudaSuccess; ++k) {
+      const uint64_t b = k * chunk, n = std::min(chunk, count - b);
+      XS_TRY(cudaStreamWaitEvent(st, g->chunk_ev[k], 0), "wait");
+      c.count = static_cast<uint32_t>(n);
+      c.in_energy = sg.energy + b;
+      c.in_mat = sg.mat + b;
+      c.out.macro_xs = a.out.macro_xs ? a.out.macro_xs + b * 5 : nullptr;
+      c.out.energy = a.out.energy ? a.out.energy + b : nullptr;
+      c.out.mat = a.out.mat ? a.out.mat + b : nullptr;
+      c.out.grid_index = a.out.grid_index ? a.out.grid_index + b : nullptr;
+      c.out.verification = a.out.verification ? a.out.verification + b : nullptr;
+      e = run_lookup(g->d, c, ws, st);
+    }
+  }
   if (e != cudaSuccess) return fail(XS_ERR_CUDA, "lookup launch", e);
   if (host_io) {
     struct {
@@ -525,6 +577,9 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!std::strcmp(name, "variant")) {
     if (value < 0 || value > 12) return fail(XS_ERR_INVALID_ARG, "variant in [0,12]");
     G.unroll = static_cast<int>(value);
+  } else if (!std::strcmp(name, "host_chunk")) {
+    if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
+    g->host_chunk = static_cast<uint64_t>(value);
   } else if (!std::strcmp(name, "blocks_per_sm")) {
     if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");
     G.blocks_per_sm = static_cast<int>(value);
@@ -572,6 +627,8 @@ void xs_free_grid(xs_grid* g) {
   DeviceGuard guard(g->d.device);
   for (auto& e : g->ev)
     for (auto x : e) cudaEventDestroy(x);
+  for (auto x : g->chunk_ev) cudaEventDestroy(x);
+  if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   cudaFree(g->d.grid);
   cudaFree(g->d.U);
   cudaFree(g->d.UB);

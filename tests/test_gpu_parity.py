@@ -386,3 +386,22 @@ def _small_second_shard_sum():
     o = oracle.Oracle.from_spec(68, 11303, conc_seed=CONC_SEED, material_rule=0, hash_bins=8192,
                                 nthreads=NT)
     return o.run(17_000_000, 17_000_000, mode=oracle.HASH, nthreads=NT)
+
+
+@pytest.mark.parametrize("sort", [False, True])
+def test_explicit_host_io_chunked(X, sort):
+    # XS_FLAG_HOST_IO inputs larger than host_chunk are uploaded and looked up
+    # chunk by chunk (overlapped); results must not depend on the chunking
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    rng = np.random.default_rng(21)
+    p = rng.random(50_003)
+    m = rng.integers(0, 12, p.size).astype(np.int32)
+    S, M, v = o.run_explicit(p, m, mode=oracle.UNIONIZED, nthreads=NT)
+    for chunk in (1 << 22, 7_001, 1_024):
+        g.set_param("host_chunk", chunk)
+        vs, res = g.lookup_explicit(torch.tensor(p), torch.tensor(m), sort=sort,
+                                    want=("macro_xs", "verification"))
+        assert vs.tolist() == [S, p.size]
+        assert np.array_equal(res["macro_xs"].numpy(), M)
+        assert np.array_equal(res["verification"].numpy(), v)
