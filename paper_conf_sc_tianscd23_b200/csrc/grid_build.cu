@@ -4,6 +4,7 @@
 //   K0a  U  = sorted multiset of all I*N energies      (in-house LSD radix sort)
 //   K0b  IG[e][n] = clamp(ub(E_n, U[e]) - 1, 0, N-2)   (chunked search + sweep)
 //   K0c  HG[b][n] = clamp(ub(E_n, b du) - 1, 0, N-2)   (one search per entry)
+//   K0d  IV[n][k]  = interval terms of record pair (k, k+1) (see below)
 // Definitions: DESIGN.md R6, R7 (north_star: "the unionized (or
 // hash-accelerated) energy grid").
 #include "common.cuh"
@@ -184,6 +185,41 @@ __global__ void k_union_table(const double* __restrict__ U, int64_t NU, int32_t 
 cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st) {
   k_union_table<<<grid_for(static_cast<uint64_t>(g.UBn) + 1, 256, g.sm_count), 256, 0, st>>>(
       g.U, g.NU, g.UBn, g.UB);
+  return cudaGetLastError();
+}
+
+// K0d: interval table.  For the record pair (k, k+1) of nuclide n, the 14
+// doubles {E[k+1], E[k+1] - E[k], recip(E[k+1] - E[k]), 0, then hi.c,
+// hi.c - lo.c for c = 0..4}: the pair-only terms of A6 (DESIGN.md
+// R10), computed with the same IEEE operations the lookup kernels use
+// (dsub, recip_nr), so interpolating from them is bit-identical to
+// interpolating from the two records.  Entry k = N-1 (no pair) is zero.
+__global__ void k_build_intervals(const double* __restrict__ grid, uint64_t total, int64_t N,
+                                  double* __restrict__ IV) {
+  for (uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; t < total;
+       t += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    double* o = IV + t * kIvDoubles;
+    if (static_cast<int64_t>(t % static_cast<uint64_t>(N)) == N - 1) {
+      for (int q = 0; q < kIvDoubles; ++q) o[q] = 0.0;
+      continue;
+    }
+    const double* lo = grid + t * 6;
+    const double* hi = lo + 6;
+    const double bd = dsub(hi[0], lo[0]);
+    o[0] = hi[0];
+    o[1] = bd;
+    o[2] = recip_nr(bd);
+    o[3] = 0.0;
+    for (int c = 0; c < 5; ++c) {
+      o[4 + 2 * c] = hi[1 + c];
+      o[5 + 2 * c] = dsub(hi[1 + c], lo[1 + c]);
+    }
+  }
+}
+
+cudaError_t build_intervals(const DeviceGrid& g, cudaStream_t st) {
+  const uint64_t total = static_cast<uint64_t>(g.I) * g.N;
+  k_build_intervals<<<grid_for(total, 256, g.sm_count), 256, 0, st>>>(g.grid, total, g.N, g.iv);
   return cudaGetLastError();
 }
 

@@ -77,6 +77,7 @@ __device__ __forceinline__ Sample sample_lookup(uint64_t seed, uint64_t id) {
 struct Params {
   // grid
   const double* grid;
+  const double* iv;         // interval table [I][N][kIvDoubles] (K0d)
   int32_t I;
   int64_t N;
   const double* U;
@@ -1694,6 +1695,629 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
   }
 }
 
+// -------------------------------------- TMA-staged sorted gather, v2 ------
+// k_gather_s2: the k_gather_s decomposition (warp = task of 32*R energy-sorted
+// lookups of one material, lane = R consecutive lookups, per-nuclide record
+// window [k_lo, k_hi + 1] staged in shared memory by TMA bulk copies) with
+// the per-nuclide instruction overhead cut:
+//  * the window is read with shared-memory loads (LDS) on its own code path;
+//    windows longer than W records take a separate global-memory path (never
+//    a generic pointer that merges the two);
+//  * each lane finds the brackets of its first and last lookup with a
+//    warp-uniform binary lifting over the window's interior energies; when
+//    every lane's lookups share one record pair (the common case: a task spans
+//    ~0.6 intervals of a fuel nuclide), the R interpolations run as one
+//    straight-line block with no per-lookup test, so the compiler interleaves
+//    R independent FP64 chains; otherwise lanes walk their lookups through
+//    the window as in k_gather_s;
+//  * the bulk copies are issued D at a time by D lanes in parallel into a
+//    ring of 2D slots (D to 2D nuclides ahead), not one per nuclide by lane 0.
+// Arithmetic and order are those of k_gather_s (bit-identical results).
+template <int R>
+struct PairTerms {
+  double hiE, bd, rc, h[5], d[5];
+};
+
+template <int R, bool CHECK>
+__device__ __forceinline__ void pair_terms_of(const double2 (&c)[6], PairTerms<R>& t) {
+  t.hiE = c[3].x;
+  t.bd = dsub(c[3].x, c[0].x);
+  t.rc = recip_nr(t.bd);
+  t.h[0] = c[3].y;
+  t.h[1] = c[4].x;
+  t.h[2] = c[4].y;
+  t.h[3] = c[5].x;
+  t.h[4] = c[5].y;
+  t.d[0] = dsub(c[3].y, c[0].y);
+  t.d[1] = dsub(c[4].x, c[1].x);
+  t.d[2] = dsub(c[4].y, c[1].y);
+  t.d[3] = dsub(c[5].x, c[2].x);
+  t.d[4] = dsub(c[5].y, c[2].y);
+}
+
+// A6 + A7 for one lookup at energy p with the pair terms t (R10/R11)
+template <int R, bool CHECK>
+__device__ __forceinline__ void interp_acc(const PairTerms<R>& t, double p, double conc,
+                                           double (&M)[5]) {
+  const double an = dsub(t.hiE, p);
+  double f = div_by_recip(an, t.bd, t.rc);
+  if (CHECK && !div_in_range(an, t.bd)) f = ddiv(an, t.bd);
+#pragma unroll
+  for (int c = 0; c < 5; ++c) M[c] = dadd(M[c], dmul(dsub(t.h[c], dmul(f, t.d[c])), conc));
+}
+
+// One nuclide of a task: win = records k_lo .. k_lo + n_int + 1 (shared or
+// global memory), lookups p[0..R-1] ascending.
+template <int R, bool CHECK, bool SHARED>
+__device__ __forceinline__ void stage_nuclide(const double2* win, int n_int, double conc,
+                                              const double (&p)[R], double (&M)[R][5]) {
+  auto E = [&](int t) -> double { return SHARED ? win[t * 3].x : __ldg(&win[t * 3].x); };
+  auto load = [&](int k, double2 (&c)[6]) {
+    const double2* pr = win + k * 3;
+#pragma unroll
+    for (int q = 0; q < 6; ++q) c[q] = SHARED ? pr[q] : __ldg(pr + q);
+  };
+  // bracket offsets (within the window) of the lane's first and last lookup:
+  // i = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p}
+  int i0 = 0, iL = 0;
+  if (n_int > 0) {
+    for (int step = 1 << (31 - __clz(n_int)); step > 0; step >>= 1) {
+      if (i0 + step <= n_int && E(i0 + step) <= p[0]) i0 += step;
+      if (iL + step <= n_int && E(iL + step) <= p[R - 1]) iL += step;
+    }
+  }
+  double2 c[6];
+  PairTerms<R> t;
+  if (__all_sync(0xffffffffu, i0 == iL)) {
+    load(i0, c);
+    pair_terms_of<R, CHECK>(c, t);
+#pragma unroll
+    for (int r = 0; r < R; ++r) interp_acc<R, CHECK>(t, p[r], conc, M[r]);
+    return;
+  }
+  int k = i0;
+  load(k, c);
+  pair_terms_of<R, CHECK>(c, t);
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (r > 0 && k < iL && p[r] >= t.hiE) {
+      if (SHARED) {
+        ++k;
+        while (k < iL && E(k + 1) <= p[r]) ++k;
+      } else {
+        int lo = k + 1, hi = iL + 1;  // E[lo] <= p < E[hi] (hi = iL + 1: p[r] <= p[R-1])
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (E(mid) <= p[r])
+            lo = mid;
+          else
+            hi = mid;
+        }
+        k = lo;
+      }
+      load(k, c);
+      pair_terms_of<R, CHECK>(c, t);
+    }
+    interp_acc<R, CHECK>(t, p[r], conc, M[r]);
+  }
+}
+
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s2(Params P) {
+  constexpr int kTask = 32 * R;
+  constexpr int S = 2 * D;  // window slots per warp
+  static_assert(D <= 32 && S <= 32, "slots");
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
+  constexpr size_t win_bytes = static_cast<size_t>(S) * W * 48;
+  const size_t k_bytes = ((static_cast<size_t>(P.max_nucs) * 8 + 15) / 16) * 16;
+  constexpr size_t bar_bytes = ((S * 8 + 15) / 16) * 16;
+  const size_t per_warp = win_bytes + k_bytes + bar_bytes;
+  unsigned char* mine = wbase + per_warp * warp;
+  double2* s_win = reinterpret_cast<double2*>(mine);               // [S][W*3]
+  int2* s_k = reinterpret_cast<int2*>(mine + win_bytes);           // [max_nucs] {k_lo, k_hi}
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(mine + win_bytes + k_bytes);
+
+  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
+    const int32_t n = P.mats[i];
+    MatEntry me;
+    me.conc = P.concs[i];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[i] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      G.num[m] = P.num_nucs[m];
+      G.off[m] = run;
+      G.cnt[m] = c;
+      G.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    G.off[P.n_mats] = run;
+    G.toff[P.n_mats] = trun;
+  }
+  if (lane == 0) {
+    for (int d = 0; d < S; ++d) mbar_init(&s_bar[d], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = G.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
+  uint32_t phase = 0;  // parity bit per slot
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+    while (task >= G.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < G.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
+    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid[r]) {
+        phi = p[r];
+        uhi = gidx[r];
+      }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
+      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
+      plo = a < plo ? a : plo;
+      phi = b > phi ? b : phi;
+    }
+    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
+      ulo = union_index_tab(P, plo);
+      uhi = union_index_tab(P, phi);
+    } else {
+      ulo = __reduce_min_sync(0xffffffffu, ulo);
+      uhi = __reduce_max_sync(0xffffffffu, uhi);
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
+    const int nn = G.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    // A4 for the two extremes of every nuclide of the material
+    for (int j = lane; j < nn; j += 32) {
+      const MatEntry me = row[j];
+      int32_t klo, khi;
+      if (GT == XS_GRID_UNIONIZED) {
+        if (P.index_t) {
+          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
+          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
+        } else {
+          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
+          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
+        }
+      } else {
+        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
+        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
+        klo = rlo.bracket(P, me.n, me.noff, plo);
+        khi = rhi.bracket(P, me.n, me.noff, phi);
+      }
+      s_k[j] = make_int2(klo, khi);
+    }
+    __syncwarp();
+    // A5 producer: lanes 0..D-1 stage the windows of nuclides g*D .. g*D+D-1
+    auto issue_group = [&](int g) {
+      const int j = g * D + lane;
+      if (lane < D && j < nn) {
+        const int slot = j % S;
+        const int2 kk = s_k[j];
+        const int32_t w = kk.y - kk.x + 2;  // records k_lo .. k_hi + 1
+        if (w <= W) {
+          const double2* src = grid2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * 3;
+          mbar_arrive_expect_tx(&s_bar[slot], static_cast<uint32_t>(w) * 48u);
+          bulk_copy_g2s(s_win + slot * W * 3, src, static_cast<uint32_t>(w) * 48u, &s_bar[slot]);
+        } else {
+          mbar_arrive_expect_tx(&s_bar[slot], 0u);  // read in place from global memory
+        }
+      }
+    };
+    issue_group(0);
+    issue_group(1);
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    for (int j = 0; j < nn; ++j) {
+      const int slot = j % S;
+      if (j >= D && j % D == 0) {
+        __syncwarp();  // every lane is done with the slots of group j/D - 1
+        issue_group(j / D + 1);
+      }
+      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
+      phase ^= 1u << slot;
+      const double conc = row[j].conc;
+      const int2 kk = s_k[j];
+      const int n_int = kk.y - kk.x;
+      if (n_int + 2 <= W) {
+        stage_nuclide<R, CHECK, true>(s_win + slot * W * 3, n_int, conc, p, M);
+      } else {
+        const double2* gw2 = grid2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * 3;
+        stage_nuclide<R, CHECK, false>(gw2, n_int, conc, p, M);
+      }
+    }
+    __syncwarp();  // all slots consumed before the next task reuses them
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
+// ------------------------------- TMA-staged sorted gather, interval table --
+// k_gather_s3: as k_gather_s2, but the window holds entries of the interval
+// table (grid_build.cu K0d: per record pair {E[k+1], gap, recip(gap), hi.c,
+// hi.c - lo.c}) instead of raw records, so no pair-only arithmetic (5 DFMA
+// reciprocal chain + 6 subtractions) runs in the timed loop: a lookup is
+// 4 FP64 ops for f and 4 per channel.  Each lane locates every lookup's
+// interval in the window by warp-uniform binary lifting; when all lanes'
+// lookups share one interval the R interpolations run as one straight-line
+// block, otherwise a lane reloads the 7 x 16 B entry (shared memory) only
+// when the interval changes.  Bit-identical to k_gather_s.
+// Entry layout (7 x 16 B): {E[k+1], gap} {recip(gap), 0} {hi.c, hi.c - lo.c} x 5.
+// A6 + A7 for lookups r in [r0, r1) that all lie in entry q (channel terms are
+// read from the window per channel to keep register pressure low).
+template <int R, bool CHECK, bool SHARED>
+__device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R], double conc,
+                                          double (&M)[R][5], int r0, int r1) {
+  auto ld = [&](int u) -> double2 { return SHARED ? q[u] : __ldg(q + u); };
+  const double2 a0 = ld(0), a1 = ld(1);
+  double f[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (r < r0 || r >= r1) continue;
+    const double an = dsub(a0.x, p[r]);
+    f[r] = div_by_recip(an, a0.y, a1.x);
+    if (CHECK && !div_in_range(an, a0.y)) f[r] = ddiv(an, a0.y);
+  }
+#pragma unroll
+  for (int c = 0; c < 5; ++c) {
+    const double2 hd = ld(2 + c);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (r < r0 || r >= r1) continue;
+      M[r][c] = dadd(M[r][c], dmul(dsub(hd.x, dmul(f[r], hd.y)), conc));
+    }
+  }
+}
+
+// One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
+template <int R, bool CHECK, bool SHARED>
+__device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
+                                                 const double (&p)[R], double (&M)[R][5]) {
+  constexpr int kE = kIvDoubles / 2;
+  // E[k_lo + t] = first double of entry t - 1
+  auto E = [&](int t) -> double {
+    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
+    return SHARED ? q[0] : __ldg(q);
+  };
+  int i[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) i[r] = 0;
+  if (n_int > 0) {
+    for (int step = 1 << (31 - __clz(n_int)); step > 0; step >>= 1) {
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (i[r] + step <= n_int && E(i[r] + step) <= p[r]) i[r] += step;
+    }
+  }
+  if (__all_sync(0xffffffffu, i[0] == i[R - 1])) {
+    iv_interp<R, CHECK, SHARED>(win + i[0] * kE, p, conc, M, 0, R);
+    return;
+  }
+#pragma unroll
+  for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
+}
+
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
+  constexpr int kTask = 32 * R;
+  constexpr int S = 2 * D;               // window slots per warp
+  constexpr int kEntry = kIvDoubles * 8;  // bytes per interval entry
+  static_assert(S <= 32, "slots");
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
+  constexpr size_t win_bytes = static_cast<size_t>(S) * W * kEntry;
+  const size_t k_bytes = ((static_cast<size_t>(P.max_nucs) * 8 + 15) / 16) * 16;
+  constexpr size_t bar_bytes = ((S * 8 + 15) / 16) * 16;
+  const size_t per_warp = win_bytes + k_bytes + bar_bytes;
+  unsigned char* mine = wbase + per_warp * warp;
+  double2* s_win = reinterpret_cast<double2*>(mine);               // [S][W * 7]
+  int2* s_k = reinterpret_cast<int2*>(mine + win_bytes);           // [max_nucs] {k_lo, k_hi}
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(mine + win_bytes + k_bytes);
+
+  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
+    const int32_t n = P.mats[i];
+    MatEntry me;
+    me.conc = P.concs[i];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[i] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      G.num[m] = P.num_nucs[m];
+      G.off[m] = run;
+      G.cnt[m] = c;
+      G.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    G.off[P.n_mats] = run;
+    G.toff[P.n_mats] = trun;
+  }
+  if (lane == 0) {
+    for (int d = 0; d < S; ++d) mbar_init(&s_bar[d], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = G.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(P.iv);
+  uint32_t phase = 0;  // parity bit per slot
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+    while (task >= G.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < G.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
+    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid[r]) {
+        phi = p[r];
+        uhi = gidx[r];
+      }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
+      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
+      plo = a < plo ? a : plo;
+      phi = b > phi ? b : phi;
+    }
+    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
+      ulo = union_index_tab(P, plo);
+      uhi = union_index_tab(P, phi);
+    } else {
+      ulo = __reduce_min_sync(0xffffffffu, ulo);
+      uhi = __reduce_max_sync(0xffffffffu, uhi);
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
+    const int nn = G.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    // A4 for the two extremes of every nuclide of the material
+    for (int j = lane; j < nn; j += 32) {
+      const MatEntry me = row[j];
+      int32_t klo, khi;
+      if (GT == XS_GRID_UNIONIZED) {
+        if (P.index_t) {
+          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
+          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
+        } else {
+          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
+          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
+        }
+      } else {
+        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
+        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
+        klo = rlo.bracket(P, me.n, me.noff, plo);
+        khi = rhi.bracket(P, me.n, me.noff, phi);
+      }
+      s_k[j] = make_int2(klo, khi);
+    }
+    __syncwarp();
+    // A5 producer: lanes 0..D-1 stage the entries k_lo .. k_hi of nuclides
+    // g*D .. g*D+D-1
+    auto issue_group = [&](int g) {
+      const int j = g * D + lane;
+      if (lane < D && j < nn) {
+        const int slot = j % S;
+        const int2 kk = s_k[j];
+        const int32_t w = kk.y - kk.x + 1;
+        if (w <= W) {
+          const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
+          mbar_arrive_expect_tx(&s_bar[slot], static_cast<uint32_t>(w) * kEntry);
+          bulk_copy_g2s(s_win + slot * W * (kIvDoubles / 2), src, static_cast<uint32_t>(w) * kEntry,
+                        &s_bar[slot]);
+        } else {
+          mbar_arrive_expect_tx(&s_bar[slot], 0u);  // read in place from global memory
+        }
+      }
+    };
+    issue_group(0);
+    issue_group(1);
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    for (int j = 0; j < nn; ++j) {
+      const int slot = j % S;
+      if (j >= D && j % D == 0) {
+        __syncwarp();  // every lane is done with the slots of group j/D - 1
+        issue_group(j / D + 1);
+      }
+      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
+      phase ^= 1u << slot;
+      const double conc = row[j].conc;
+      const int2 kk = s_k[j];
+      const int n_int = kk.y - kk.x;
+      if (n_int < W) {
+        stage_nuclide_iv<R, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
+      } else {
+        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
+        stage_nuclide_iv<R, CHECK, false>(g2, n_int, conc, p, M);
+      }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -1805,6 +2429,7 @@ __global__ void k_nuclide_index(Params P, const double* __restrict__ energy,
 static Params make_params(const DeviceGrid& g) {
   Params P{};
   P.grid = g.grid;
+  P.iv = g.iv;
   P.I = g.I;
   P.N = g.N;
   P.U = g.U;
@@ -1935,14 +2560,57 @@ static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+static cudaError_t launch_gather_s2(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * 48;
+  const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
+  const size_t smem = sizeof(GatherSmem) +
+                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
+                      NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
+  auto kern = k_gather_s2<GT, R, D, W, NW, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
+template <int GT, int R, int D, int W, int NW, bool CHECK>
+static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * kIvDoubles * 8;
+  const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
+  const size_t smem = sizeof(GatherSmem) +
+                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
+                      NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
+  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
   // blocks); 5-6 pipelined; 7-8 windowed; 9-12 TMA-staged (R, stages D,
-  // window W records, warps per block).  Measured best on B200 (large and
-  // large-hash): k_gather_s (4, 4, 16, 16).
+  // window W records, warps per block); 13-16 TMA-staged v2; 17-20
+  // TMA-staged from the interval table.  Measured best on B200 (large,
+  // large-hash, small): k_gather_s3 (4, 2, 8, 16) = variant 19.
   int v = g.unroll;
-  if (v == 0) v = 9;
+  if (v == 0) v = 19;
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
@@ -1956,6 +2624,14 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 10: return launch_gather_s<GT, 4, 3, 16, 16, CHECK>(g, P, st);
     case 11: return launch_gather_s<GT, 4, 6, 12, 16, CHECK>(g, P, st);
     case 12: return launch_gather_s<GT, 4, 4, 12, 8, CHECK>(g, P, st);
+    case 13: return launch_gather_s2<GT, 4, 4, 16, 16, CHECK>(g, P, st);
+    case 14: return launch_gather_s2<GT, 4, 4, 16, 12, CHECK>(g, P, st);
+    case 15: return launch_gather_s2<GT, 4, 4, 16, 8, CHECK>(g, P, st);
+    case 16: return launch_gather_s2<GT, 2, 2, 12, 24, CHECK>(g, P, st);
+    case 17: return launch_gather_s3<GT, 4, 4, 8, 12, CHECK>(g, P, st);
+    case 18: return launch_gather_s3<GT, 4, 4, 8, 16, CHECK>(g, P, st);
+    case 19: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK>(g, P, st);
+    case 20: return launch_gather_s3<GT, 2, 2, 8, 24, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }

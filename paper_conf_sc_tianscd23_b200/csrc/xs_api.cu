@@ -246,6 +246,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   }
   auto cleanup = [&]() {
     cudaFree(G.grid);
+    cudaFree(G.iv);
     cudaFree(G.U);
     cudaFree(G.UB);
     cudaFree(G.index);
@@ -260,6 +261,8 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   cudaError_t e = cudaMalloc(&G.grid, grid_bytes + 6 * sizeof(double));
   if (e == cudaSuccess) e = cudaMemsetAsync(reinterpret_cast<char*>(G.grid) + grid_bytes, 0,
                                             6 * sizeof(double), st);
+  const size_t iv_bytes = static_cast<size_t>(I) * N * kIvDoubles * sizeof(double);
+  if (e == cudaSuccess) e = cudaMalloc(&G.iv, iv_bytes);
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.UB, (static_cast<size_t>(G.UBn) + 1) * 4);
   if (e == cudaSuccess && G.index_len && (G.index_layout & XS_INDEX_ROW))
@@ -273,12 +276,13 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cleanup();
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
-  G.device_bytes = grid_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
+  G.device_bytes = grid_bytes + iv_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
   e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.mats, d->mats, tab * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.concs, d->concs, tab * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = build_intervals(G, st);
   if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
     e = build_union_grid(G, G.U, st);
     if (e == cudaSuccess) e = build_union_table(G, st);
@@ -575,7 +579,7 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
-    if (value < 0 || value > 12) return fail(XS_ERR_INVALID_ARG, "variant in [0,12]");
+    if (value < 0 || value > 20) return fail(XS_ERR_INVALID_ARG, "variant in [0,20]");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
@@ -630,6 +634,7 @@ void xs_free_grid(xs_grid* g) {
   for (auto x : g->chunk_ev) cudaEventDestroy(x);
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   cudaFree(g->d.grid);
+  cudaFree(g->d.iv);
   cudaFree(g->d.U);
   cudaFree(g->d.UB);
   cudaFree(g->d.index);

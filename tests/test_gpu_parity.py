@@ -70,7 +70,9 @@ def _compare(out, ref, mode_index=True):
 # ------------------------------------------------------------------- tiny --
 @pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
                                      "sort-v1", "sort-v3", "sort-v4", "sort-v5", "sort-v6", "sort-v7",
-                                     "sort-v8", "sort-v9", "sort-v10", "sort-v11", "sort-v12"])
+                                     "sort-v8", "sort-v9", "sort-v10", "sort-v11", "sort-v12",
+                                     "sort-v13", "sort-v14", "sort-v15", "sort-v16",
+                                     "sort-v17", "sort-v18", "sort-v19", "sort-v20"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -97,6 +99,20 @@ def test_tiny_other_grids(X, grid_type, bins, sort):
     vs, out = _full_outputs(g, 0, 100_000, sort=sort)
     _compare(out, ref)
     assert vs == [S, 100_000]
+
+
+@pytest.mark.parametrize("grid_type,bins", [("hash", 97), ("hash", 8192), ("nuclide", 0)])
+@pytest.mark.parametrize("variant", [9, 13, 16, 17, 20])
+def test_tiny_other_grids_staged(X, grid_type, bins, variant):
+    """The TMA-staged sorted gathers on the hash and nuclide grids."""
+    g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
+    g.set_param("variant", variant)
+    mode = oracle.HASH if grid_type == "hash" else oracle.NUCLIDE
+    S, ref = oracle_for("tiny", hash_bins=bins).run(3, 70_001, mode=mode, nthreads=NT,
+                                                    outputs=True)
+    vs, out = _full_outputs(g, 3, 70_001, sort=True)
+    _compare(out, ref)
+    assert vs == [S, 70_001]
 
 
 @pytest.mark.parametrize("layout", ["row", "col", "both"])

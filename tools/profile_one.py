@@ -18,12 +18,12 @@ ap.add_argument("--config", default="large")
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--sort", action="store_true")
 ap.add_argument("--baseline", action="store_true")
-ap.add_argument("--unroll", type=int, default=0)
+ap.add_argument("--variant", type=int, default=0)
 ap.add_argument("--lookups", type=int, default=0)
 a = ap.parse_args()
 g = X.Grid.from_preset(a.config)
-if a.unroll:
-    g.set_param("unroll", a.unroll)
+if a.variant:
+    g.set_param("variant", a.variant)
 L = a.lookups or min(X.PRESETS[a.config]["lookups"], 17_000_000)
 sort = a.sort or X.PRESETS[a.config].get("sort", False)
 vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
