@@ -174,6 +174,26 @@ __device__ __forceinline__ int32_t union_index_tab(const Params& P, double p) {
   return static_cast<int32_t>(lo);
 }
 
+// Conservative A3 bounds from the equal-width table alone (no bisection):
+// ulo <= u(p) for p >= plo and uhi >= u(p) for p <= phi.  UB[b] = ub(U, b/UBn)
+// and b/UBn <= p < (b+1)/UBn give ub(U, p) in [UB[b], UB[b+1]].  IGT is
+// monotone in u, so the brackets read at ulo / uhi bound every bracket of the
+// energies in [plo, phi]; the exact bracket is then found inside the window.
+__device__ __forceinline__ int32_t union_lower_tab(const Params& P, double p) {
+  const double q = p * static_cast<double>(P.UBn);
+  if (!(q > 0.0)) return 0;
+  const int32_t b = q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q) : P.UBn;
+  const int32_t l = __ldg(P.UB + b) - 1;
+  return l < 0 ? 0 : (l > P.NU - 2 ? static_cast<int32_t>(P.NU - 2) : l);
+}
+__device__ __forceinline__ int32_t union_upper_tab(const Params& P, double p) {
+  const double q = p * static_cast<double>(P.UBn);
+  const int32_t b = q > 0.0 ? (q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q) : P.UBn) : 0;
+  if (b >= P.UBn) return static_cast<int32_t>(P.NU - 2);
+  const int32_t h = __ldg(P.UB + b + 1) - 1;
+  return h < 0 ? 0 : (h > P.NU - 2 ? static_cast<int32_t>(P.NU - 2) : h);
+}
+
 // k_sample: A1 + A3 in batch order.  Thread t of a block handles lookups
 // c0 + it*256 + t, it < kPrepItems; their unionized searches run in
 // lockstep (kPrepItems independent probes in flight per thread).  Writes
@@ -2064,6 +2084,8 @@ __device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R]
 }
 
 // One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
+// i(p) = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p} by binary lifting
+// (warp-uniform trip count; loads clamped so the loop has no branches).
 template <int R, bool CHECK, bool SHARED>
 __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
                                                  const double (&p)[R], double (&M)[R][5]) {
@@ -2073,25 +2095,94 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
     return SHARED ? q[0] : __ldg(q);
   };
-  int i[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) i[r] = 0;
-  if (n_int > 0) {
-    for (int step = 1 << (31 - __clz(n_int)); step > 0; step >>= 1) {
-#pragma unroll
-      for (int r = 0; r < R; ++r)
-        if (i[r] + step <= n_int && E(i[r] + step) <= p[r]) i[r] += step;
-    }
+  int i0 = 0, iL = 0;
+  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
+  for (int step = top; step > 0; step >>= 1) {
+    const int t0 = i0 + step, tL = iL + step;
+    const double e0 = E(t0 <= n_int ? t0 : n_int), eL = E(tL <= n_int ? tL : n_int);
+    if (t0 <= n_int && e0 <= p[0]) i0 = t0;
+    if (tL <= n_int && eL <= p[R - 1]) iL = tL;
   }
-  if (__all_sync(0xffffffffu, i[0] == i[R - 1])) {
-    iv_interp<R, CHECK, SHARED>(win + i[0] * kE, p, conc, M, 0, R);
+  if (__all_sync(0xffffffffu, i0 == iL)) {
+    iv_interp<R, CHECK, SHARED>(win + i0 * kE, p, conc, M, 0, R);
     return;
+  }
+  int i[R];
+  i[0] = i0;
+  i[R - 1] = iL;
+#pragma unroll
+  for (int r = 1; r < R - 1; ++r) i[r] = i0;
+  if (R > 2) {
+    for (int step = top; step > 0; step >>= 1) {
+#pragma unroll
+      for (int r = 1; r < R - 1; ++r) {
+        const int t = i[r] + step;
+        const double e = E(t <= n_int ? t : n_int);
+        if (t <= n_int && e <= p[r]) i[r] = t;
+      }
+    }
   }
 #pragma unroll
   for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK>
+// Branch-free variant: every lookup's entry index by binary lifting, the
+// entry terms reloaded (predicated) only where the index changes between a
+// lane's consecutive lookups; one straight-line block per nuclide.
+template <int R, bool CHECK, bool SHARED>
+__device__ __forceinline__ void stage_nuclide_iv_pred(const double2* win, int n_int, double conc,
+                                                      const double (&p)[R], double (&M)[R][5]) {
+  constexpr int kE = kIvDoubles / 2;
+  auto ld = [&](int u) -> double2 { return SHARED ? win[u] : __ldg(win + u); };
+  auto E = [&](int t) -> double {
+    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
+    return SHARED ? q[0] : __ldg(q);
+  };
+  int i[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) i[r] = 0;
+  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
+  for (int step = top; step > 0; step >>= 1) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int t = i[r] + step;
+      const double e = E(t <= n_int ? t : n_int);
+      if (t <= n_int && e <= p[r]) i[r] = t;
+    }
+  }
+  double f[R];
+  double2 a0 = ld(i[0] * kE), a1 = ld(i[0] * kE + 1);
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (r > 0 && i[r] != i[r - 1]) {
+      a0 = ld(i[r] * kE);
+      a1 = ld(i[r] * kE + 1);
+    }
+    const double an = dsub(a0.x, p[r]);
+    f[r] = div_by_recip(an, a0.y, a1.x);
+    if (CHECK && !div_in_range(an, a0.y)) f[r] = ddiv(an, a0.y);
+  }
+#pragma unroll
+  for (int c = 0; c < 5; ++c) {
+    double2 hd = ld(i[0] * kE + 2 + c);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (r > 0 && i[r] != i[r - 1]) hd = ld(i[r] * kE + 2 + c);
+      M[r][c] = dadd(M[r][c], dmul(dsub(hd.x, dmul(f[r], hd.y)), conc));
+    }
+  }
+}
+
+template <int R, int MODE, bool CHECK, bool SHARED>
+__device__ __forceinline__ void stage_nuclide_sel(const double2* win, int n_int, double conc,
+                                                  const double (&p)[R], double (&M)[R][5]) {
+  if (MODE == 1)
+    stage_nuclide_iv_pred<R, CHECK, SHARED>(win, n_int, conc, p, M);
+  else
+    stage_nuclide_iv<R, CHECK, SHARED>(win, n_int, conc, p, M);
+}
+
+template <int GT, int R, int D, int W, int NW, bool CHECK, int MODE = 0>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   constexpr int kTask = 32 * R;
   constexpr int S = 2 * D;               // window slots per warp
@@ -2195,8 +2286,8 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       phi = b > phi ? b : phi;
     }
     if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
-      ulo = union_index_tab(P, plo);
-      uhi = union_index_tab(P, phi);
+      ulo = union_lower_tab(P, plo);
+      uhi = union_upper_tab(P, phi);
     } else {
       ulo = __reduce_min_sync(0xffffffffu, ulo);
       uhi = __reduce_max_sync(0xffffffffu, uhi);
@@ -2266,10 +2357,10 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
       if (n_int < W) {
-        stage_nuclide_iv<R, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
+        stage_nuclide_sel<R, MODE, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
       } else {
         const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
-        stage_nuclide_iv<R, CHECK, false>(g2, n_int, conc, p, M);
+        stage_nuclide_sel<R, MODE, CHECK, false>(g2, n_int, conc, p, M);
       }
     }
     __syncwarp();
@@ -2581,14 +2672,14 @@ static cudaError_t launch_gather_s2(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK>
+template <int GT, int R, int D, int W, int NW, bool CHECK, int MODE = 0>
 static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * kIvDoubles * 8;
   const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
   const size_t smem = sizeof(GatherSmem) +
                       static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
                       NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
-  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK>;
+  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK, MODE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -2632,6 +2723,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 18: return launch_gather_s3<GT, 4, 4, 8, 16, CHECK>(g, P, st);
     case 19: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK>(g, P, st);
     case 20: return launch_gather_s3<GT, 2, 2, 8, 24, CHECK>(g, P, st);
+    case 21: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 1>(g, P, st);
+    case 22: return launch_gather_s3<GT, 4, 2, 8, 12, CHECK, 1>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
