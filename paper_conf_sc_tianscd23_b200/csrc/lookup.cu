@@ -2083,10 +2083,42 @@ __device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R]
   }
 }
 
+// A6 + A7 for lookups in (possibly) different entries i[r] of the window:
+// the entry terms are reloaded (predicated) only where the entry changes
+// between a lane's consecutive lookups.
+template <int R, bool CHECK, bool SHARED>
+__device__ __forceinline__ void iv_interp_var(const double2* win, const int (&i)[R],
+                                              const double (&p)[R], double conc,
+                                              double (&M)[R][5]) {
+  constexpr int kE = kIvDoubles / 2;
+  auto ld = [&](int u) -> double2 { return SHARED ? win[u] : __ldg(win + u); };
+  double f[R];
+  double2 a0 = ld(i[0] * kE), a1 = ld(i[0] * kE + 1);
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (r > 0 && i[r] != i[r - 1]) {
+      a0 = ld(i[r] * kE);
+      a1 = ld(i[r] * kE + 1);
+    }
+    const double an = dsub(a0.x, p[r]);
+    f[r] = div_by_recip(an, a0.y, a1.x);
+    if (CHECK && !div_in_range(an, a0.y)) f[r] = ddiv(an, a0.y);
+  }
+#pragma unroll
+  for (int c = 0; c < 5; ++c) {
+    double2 hd = ld(i[0] * kE + 2 + c);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (r > 0 && i[r] != i[r - 1]) hd = ld(i[r] * kE + 2 + c);
+      M[r][c] = dadd(M[r][c], dmul(dsub(hd.x, dmul(f[r], hd.y)), conc));
+    }
+  }
+}
+
 // One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
 // i(p) = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p} by binary lifting
 // (warp-uniform trip count; loads clamped so the loop has no branches).
-template <int R, bool CHECK, bool SHARED>
+template <int R, bool CHECK, bool SHARED, bool PRED = false>
 __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
                                                  const double (&p)[R], double (&M)[R][5]) {
   constexpr int kE = kIvDoubles / 2;
@@ -2122,6 +2154,49 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
       }
     }
   }
+  if (PRED) {
+    iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
+    return;
+  }
+#pragma unroll
+  for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
+}
+
+// Second half of stage_nuclide_iv for a caller that already lifted the first
+// and last lookup (i0, iL): the software-pipelined loop of k_gather_s3 MODE 2.
+template <int R, bool CHECK, bool SHARED, bool PRED = false>
+__device__ __forceinline__ void stage_apply_iv(const double2* win, int n_int, double conc,
+                                               const double (&p)[R], double (&M)[R][5], int i0,
+                                               int iL) {
+  constexpr int kE = kIvDoubles / 2;
+  auto E = [&](int t) -> double {
+    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
+    return SHARED ? q[0] : __ldg(q);
+  };
+  if (__all_sync(0xffffffffu, i0 == iL)) {
+    iv_interp<R, CHECK, SHARED>(win + i0 * kE, p, conc, M, 0, R);
+    return;
+  }
+  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
+  int i[R];
+  i[0] = i0;
+  i[R - 1] = iL;
+#pragma unroll
+  for (int r = 1; r < R - 1; ++r) i[r] = i0;
+  if (R > 2) {
+    for (int step = top; step > 0; step >>= 1) {
+#pragma unroll
+      for (int r = 1; r < R - 1; ++r) {
+        const int t = i[r] + step;
+        const double e = E(t <= n_int ? t : n_int);
+        if (t <= n_int && e <= p[r]) i[r] = t;
+      }
+    }
+  }
+  if (PRED) {
+    iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
+    return;
+  }
 #pragma unroll
   for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
 }
@@ -2150,27 +2225,7 @@ __device__ __forceinline__ void stage_nuclide_iv_pred(const double2* win, int n_
       if (t <= n_int && e <= p[r]) i[r] = t;
     }
   }
-  double f[R];
-  double2 a0 = ld(i[0] * kE), a1 = ld(i[0] * kE + 1);
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    if (r > 0 && i[r] != i[r - 1]) {
-      a0 = ld(i[r] * kE);
-      a1 = ld(i[r] * kE + 1);
-    }
-    const double an = dsub(a0.x, p[r]);
-    f[r] = div_by_recip(an, a0.y, a1.x);
-    if (CHECK && !div_in_range(an, a0.y)) f[r] = ddiv(an, a0.y);
-  }
-#pragma unroll
-  for (int c = 0; c < 5; ++c) {
-    double2 hd = ld(i[0] * kE + 2 + c);
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (r > 0 && i[r] != i[r - 1]) hd = ld(i[r] * kE + 2 + c);
-      M[r][c] = dadd(M[r][c], dmul(dsub(hd.x, dmul(f[r], hd.y)), conc));
-    }
-  }
+  iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
 }
 
 template <int R, int MODE, bool CHECK, bool SHARED>
@@ -2178,6 +2233,8 @@ __device__ __forceinline__ void stage_nuclide_sel(const double2* win, int n_int,
                                                   const double (&p)[R], double (&M)[R][5]) {
   if (MODE == 1)
     stage_nuclide_iv_pred<R, CHECK, SHARED>(win, n_int, conc, p, M);
+  else if (MODE == 3)
+    stage_nuclide_iv<R, CHECK, SHARED, true>(win, n_int, conc, p, M);
   else
     stage_nuclide_iv<R, CHECK, SHARED>(win, n_int, conc, p, M);
 }
@@ -2345,24 +2402,325 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 #pragma unroll
       for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
 
-    for (int j = 0; j < nn; ++j) {
-      const int slot = j % S;
-      if (j >= D && j % D == 0) {
-        __syncwarp();  // every lane is done with the slots of group j/D - 1
-        issue_group(j / D + 1);
+    if constexpr (MODE == 2) {
+      // software-pipelined: the barrier wait, table reads and first lifting
+      // step of nuclide j+1 are issued before the interpolation of nuclide j,
+      // so their latency hides behind it
+      constexpr int kE = kIvDoubles / 2;
+      struct Head {
+        double conc, etop;
+        int n_int, top, woff, j;
+      };
+      auto head_load = [&](int j, Head& h) {
+        const int slot = j % S;
+        mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
+        phase ^= 1u << slot;
+        h.j = j;
+        h.conc = row[j].conc;
+        const int2 kk = s_k[j];
+        h.n_int = kk.y - kk.x;
+        h.top = h.n_int > 0 ? 1 << (31 - __clz(h.n_int)) : 0;
+        h.woff = slot * W * kE;
+        h.etop = 0.0;
+        if (h.n_int > 0 && h.n_int < W)  // E[k_lo + top] (every lane's first probe)
+          h.etop = reinterpret_cast<const double*>(s_win + h.woff + (h.top - 1) * kE)[0];
+      };
+      auto head_lift = [&](const Head& h, int& i0, int& iL) {
+        i0 = iL = 0;
+        if (h.n_int <= 0 || h.n_int >= W) return;
+        if (h.etop <= p[0]) i0 = h.top;
+        if (h.etop <= p[R - 1]) iL = h.top;
+        const double2* win = s_win + h.woff;
+        for (int step = h.top >> 1; step > 0; step >>= 1) {
+          const int t0 = i0 + step, tL = iL + step;
+          const double e0 = reinterpret_cast<const double*>(win + ((t0 <= h.n_int ? t0 : h.n_int) - 1) * kE)[0];
+          const double eL = reinterpret_cast<const double*>(win + ((tL <= h.n_int ? tL : h.n_int) - 1) * kE)[0];
+          if (t0 <= h.n_int && e0 <= p[0]) i0 = t0;
+          if (tL <= h.n_int && eL <= p[R - 1]) iL = tL;
+        }
+      };
+      Head cur, nxt;
+      int i0 = 0, iL = 0;
+      if (nn > 0) {
+        head_load(0, cur);
+        head_lift(cur, i0, iL);
       }
-      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
-      phase ^= 1u << slot;
+      for (int j = 0; j < nn; ++j) {
+        if (j >= D && j % D == 0) {
+          __syncwarp();  // every lane is done with the slots of group j/D - 1
+          issue_group(j / D + 1);
+        }
+        const bool more = j + 1 < nn;
+        if (more) head_load(j + 1, nxt);
+        if (cur.n_int < W) {
+          stage_apply_iv<R, CHECK, true>(s_win + cur.woff, cur.n_int, cur.conc, p, M, i0, iL);
+        } else {
+          const int2 kk = s_k[j];
+          const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
+          stage_nuclide_iv<R, CHECK, false>(g2, cur.n_int, cur.conc, p, M);
+        }
+        if (more) {
+          cur = nxt;
+          head_lift(cur, i0, iL);
+        }
+      }
+    } else {
+      for (int j = 0; j < nn; ++j) {
+        const int slot = j % S;
+        if (j >= D && j % D == 0) {
+          __syncwarp();  // every lane is done with the slots of group j/D - 1
+          issue_group(j / D + 1);
+        }
+        mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
+        phase ^= 1u << slot;
+        const double conc = row[j].conc;
+        const int2 kk = s_k[j];
+        const int n_int = kk.y - kk.x;
+        if (n_int < W) {
+          stage_nuclide_sel<R, MODE, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
+        } else {
+          const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
+          stage_nuclide_sel<R, MODE, CHECK, false>(g2, n_int, conc, p, M);
+        }
+      }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[r][c] > mx) {
+          mx = M[r][c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
+template <int GT, int R, int D, int CAP, int NW, bool CHECK>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
+  constexpr int kTask = 32 * R;
+  constexpr int kE = kIvDoubles / 2;       // 16-B chunks per interval entry
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
+  constexpr size_t buf_bytes = static_cast<size_t>(2) * CAP * kIvDoubles * 8;
+  const size_t k_bytes = ((static_cast<size_t>(P.max_nucs) * 8 + 15) / 16) * 16;
+  unsigned char* mine = wbase + (buf_bytes + k_bytes) * warp;
+  double2* s_buf = reinterpret_cast<double2*>(mine);               // [2][CAP * 7]
+  int2* s_k = reinterpret_cast<int2*>(mine + buf_bytes);           // [max_nucs] {k_lo, k_hi}
+
+  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
+    const int32_t n = P.mats[i];
+    MatEntry me;
+    me.conc = P.concs[i];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[i] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      G.num[m] = P.num_nucs[m];
+      G.off[m] = run;
+      G.cnt[m] = c;
+      G.toff[m] = trun;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+    }
+    G.off[P.n_mats] = run;
+    G.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = G.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(P.iv);
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+    while (task >= G.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < G.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
+    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid[r]) {
+        phi = p[r];
+        uhi = gidx[r];
+      }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
+      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
+      plo = a < plo ? a : plo;
+      phi = b > phi ? b : phi;
+    }
+    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
+      ulo = union_lower_tab(P, plo);
+      uhi = union_upper_tab(P, phi);
+    } else {
+      ulo = __reduce_min_sync(0xffffffffu, ulo);
+      uhi = __reduce_max_sync(0xffffffffu, uhi);
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
+    const int nn = G.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    // A4 for the two extremes of every nuclide of the material
+    for (int j = lane; j < nn; j += 32) {
+      const MatEntry me = row[j];
+      int32_t klo, khi;
+      if (GT == XS_GRID_UNIONIZED) {
+        if (P.index_t) {
+          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
+          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
+        } else {
+          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
+          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
+        }
+      } else {
+        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
+        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
+        klo = rlo.bracket(P, me.n, me.noff, plo);
+        khi = rhi.bracket(P, me.n, me.noff, phi);
+      }
+      s_k[j] = make_int2(klo, khi);
+    }
+    __syncwarp();
+    // A5: the windows (entries k_lo .. k_hi) of the D nuclides of group g
+    // are packed in order into buffer g & 1 (CAP entries; a window that does
+    // not fit is read in place from global memory) by per-lane 16-B async
+    // copies, one commit group per nuclide group.
+    auto issue_group = [&](int g) {
+      const int j0 = g * D;
+      int off[D], w[D];
+      uint32_t src[D];
+      int tot = 0;
+#pragma unroll
+      for (int t = 0; t < D; ++t) {
+        w[t] = 0;
+        off[t] = tot;
+        src[t] = 0;
+        if (j0 + t < nn) {
+          const int2 kk = s_k[j0 + t];
+          const int wt = kk.y - kk.x + 1;
+          if (tot + wt <= CAP) {
+            w[t] = wt;
+            src[t] = row[j0 + t].noff + static_cast<uint32_t>(kk.x);
+            tot += wt;
+          }
+        }
+      }
+      double2* dst = s_buf + (g & 1) * CAP * kE;
+      for (int c = lane; c < tot * kE; c += 32) {
+        const int e = c / kE, part = c - e * kE;
+        uint32_t rec = 0;
+#pragma unroll
+        for (int t = 0; t < D; ++t)
+          if (e >= off[t] && e < off[t] + w[t]) rec = src[t] + static_cast<uint32_t>(e - off[t]);
+        cp_async16(dst + c, iv2 + static_cast<uint64_t>(rec) * kE + part);
+      }
+      cp_async_commit();
+    };
+    issue_group(0);
+
+    double M[R][5];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+
+    int coff = 0;
+    for (int j = 0; j < nn; ++j) {
+      if (j % D == 0) {
+        __syncwarp();  // every lane is done with buffer (j/D + 1) & 1
+        issue_group(j / D + 1);
+        cp_async_wait<1>();  // this lane's copies of group j/D have landed
+        __syncwarp();        // ... and every other lane's
+        coff = 0;
+      }
       const double conc = row[j].conc;
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
-      if (n_int < W) {
-        stage_nuclide_sel<R, MODE, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
+      if (coff + n_int + 1 <= CAP) {
+        stage_nuclide_iv<R, CHECK, true>(s_buf + ((j / D) & 1) * CAP * kE + coff * kE, n_int, conc,
+                                         p, M);
+        coff += n_int + 1;
       } else {
-        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
-        stage_nuclide_sel<R, MODE, CHECK, false>(g2, n_int, conc, p, M);
+        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
+        stage_nuclide_iv<R, CHECK, false>(g2, n_int, conc, p, M);
       }
     }
+    cp_async_wait<0>();
     __syncwarp();
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -2693,6 +3051,27 @@ static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
+template <int GT, int R, int D, int CAP, int NW, bool CHECK>
+static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  constexpr size_t buf_bytes = static_cast<size_t>(2) * CAP * kIvDoubles * 8;
+  const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
+  const size_t smem = sizeof(GatherSmem) +
+                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
+                      NW * (buf_bytes + k_bytes);
+  auto kern = k_gather_s4<GT, R, D, CAP, NW, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
@@ -2725,6 +3104,14 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 20: return launch_gather_s3<GT, 2, 2, 8, 24, CHECK>(g, P, st);
     case 21: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 1>(g, P, st);
     case 22: return launch_gather_s3<GT, 4, 2, 8, 12, CHECK, 1>(g, P, st);
+    case 23: return launch_gather_s4<GT, 4, 4, 12, 16, CHECK>(g, P, st);
+    case 24: return launch_gather_s4<GT, 4, 2, 8, 16, CHECK>(g, P, st);
+    case 25: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK>(g, P, st);
+    case 26: return launch_gather_s3<GT, 4, 2, 4, 16, CHECK>(g, P, st);
+    case 27: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 2>(g, P, st);
+    case 28: return launch_gather_s3<GT, 4, 3, 8, 16, CHECK, 2>(g, P, st);
+    case 29: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 3>(g, P, st);
+    case 30: return launch_gather_s3<GT, 4, 2, 8, 12, CHECK, 3>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
