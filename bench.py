@@ -122,6 +122,27 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
+GATHER_KERNEL = {True: "k_gather_s3 (A4-A8, TMA-staged interval-table windows)",
+                 False: "k_gather (A4-A8, 3 lanes per lookup)"}
+FP64_OPS_PER_LOOKUP_NUCLIDE = 24
+FP64_LANES_PER_SM = 64   # B200: 37 TFLOP/s FP64 (FMA = 2) = 148 SMs x 64 lanes x 2 x 1.965 GHz
+
+
+def fp64_pipe_peak():
+    """FP64 pipe peak in T ops/s: 148 SMs x 64 FP64 lanes x max SM clock
+    (tools/fp64_peak.cu measures 63.8 DADD/DMUL per SM per clock)."""
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    mhz, src = 1965.0, "derived: 148 SMs x 64 FP64 lanes x 1965 MHz (B200 max SM clock)"
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        if d.get("sm_max_mhz"):
+            mhz = float(d["sm_max_mhz"])
+            src = (f"derived: 148 SMs x 64 FP64 lanes x {mhz:.0f} MHz (MEASURED_PEAKS.json "
+                   "sm_max_mhz); measured 18.55 T DADD/s (profiles/fp64_peak.json)")
+    return 148 * FP64_LANES_PER_SM * mhz * 1e6 / 1e12, src
+
+
 def golden():
     with open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")) as f:
         return json.load(f)
@@ -305,15 +326,34 @@ def run_ours(a, pre, cfg):
     gather_ms = tm["ms_gather"] / max(1, tm["calls"])
     achieved = gather_bytes / (gather_ms / 1e3) / 1e9
     traffic_per_lookup, traffic_src = ncu_traffic(a.config, sort)
-    roofline = {"bound": "hbm", "kernel": "k_gather (A4-A8)", "achieved": achieved,
-                "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic_per_lookup * L if traffic_per_lookup else None,
-                "peak_source": peak_src,
-                "algorithmic_bytes_per_launch": gather_bytes,
-                "gather_ms_per_launch": gather_ms,
-                "traffic_source": traffic_src,
-                "note": "algorithmic bytes = sum over lookups of n_nuclides(mat) x "
-                        f"({idx_bytes} B index + 96 B record pair); L2 hits let frac exceed 1"}
+    roofline_hbm = {"bound": "hbm", "kernel": GATHER_KERNEL[sort], "achieved": achieved,
+                    "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                    "traffic": traffic_per_lookup * L if traffic_per_lookup else None,
+                    "peak_source": peak_src,
+                    "algorithmic_bytes_per_launch": gather_bytes,
+                    "gather_ms_per_launch": gather_ms,
+                    "traffic_source": traffic_src,
+                    "note": "algorithmic bytes = sum over lookups of n_nuclides(mat) x "
+                            f"({idx_bytes} B index + 96 B record pair); L2/L1/shared-memory "
+                            "reuse lets frac exceed 1"}
+    if sort:
+        # energy-sorted batches re-read each record pair from shared memory for
+        # ~40 lookups: the staged gather is bound by the FP64 pipe
+        fp64_peak, fp64_src = fp64_pipe_peak()
+        ops = nuc_lookups * FP64_OPS_PER_LOOKUP_NUCLIDE
+        fp64_achieved = ops / (gather_ms / 1e3) / 1e12
+        roofline = {"bound": "alu", "kernel": GATHER_KERNEL[sort], "achieved": fp64_achieved,
+                    "peak": fp64_peak, "unit": "TFLOP/s", "frac": fp64_achieved / fp64_peak,
+                    "traffic": roofline_hbm["traffic"], "peak_source": fp64_src,
+                    "algorithmic_fp64_ops_per_launch": ops,
+                    "gather_ms_per_launch": gather_ms, "traffic_source": traffic_src,
+                    "note": "FP64 pipe operations (DADD/DMUL/DFMA count one each): "
+                            f"{FP64_OPS_PER_LOOKUP_NUCLIDE} per (lookup, nuclide) = f (1 sub "
+                            "+ 3 for the correctly rounded division by a precomputed "
+                            "reciprocal) + 5 channels x (mul, sub, mul, add); traffic = DRAM "
+                            "bytes per launch from ncu"}
+    else:
+        roofline = roofline_hbm
     step_frac = balg_per_lookup * (value / world) / 8e12
 
     line = {"metric": "XS lookups/sec", "value": value, "unit": "lookups/s", "n_gpus": world,
@@ -321,6 +361,7 @@ def run_ours(a, pre, cfg):
             "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None,
             "dtype": "f64", "data": "synthetic", "config": cfg,
             "roofline": roofline,
+            "roofline_hbm": roofline_hbm,
             "hbm_gather_roofline_frac_8TBs": step_frac,
             "balg_bytes_per_lookup": balg_per_lookup,
             "phase_ms_per_step": {k: tm[k] / max(1, tm["calls"])

@@ -3,25 +3,18 @@
 // A8 verify (BASELINE.json north_star).
 //
 // Pipeline of one xs_lookup_batch call (all on the caller's stream):
-//   k_count     A1: per-material histogram of the batch (materials only)
-//   k_bucket    A1+A3: sample (p, m) again, search p on U (or hash bin),
-//               write a 16-B LookupRec into the material bucket.  With
-//               XS_FLAG_SORT (A2) the bucket key is (material, energy bin)
-//               with 4096 energy bins per material: one in-house radix
-//               pass (k_count histogram, k_scan_bins scan, k_bucket
-//               scatter) that leaves each material's lookups ordered by
-//               energy to 2^-12, so the lookups sharing a warp touch the
-//               same record pairs.
-//   k_gather    A4-A8: warp-per-task over material buckets; each group of
-//               G=3 lanes owns one lookup and walks the material's nuclides
-//               in list order; per nuclide the 3 lanes gather the 96-B
-//               record pair as 2x3 128-bit loads (lane r takes 16-B chunk r
-//               of the low and of the high record), lane 0 computes the
-//               interpolation weight f and broadcasts it, each lane
-//               interpolates its two channels and accumulates them in list
-//               order (exact binary64, no FMA), so every M_c is bit-identical
-//               to the serial definition.
-//   verification: v = 1 + argmax; per-block reduction, one atomic per block.
+//   k_sample    A1 + A3: sample (p, m) from the counter-based stream (or read
+//               the caller's energies), search u (unionized) / bin b (hash)
+//               when needed, write a 16-B LookupRec in batch order, and count
+//               lookups per material (A2 off) or per (material, energy bin)
+//               with the lookup's rank inside its bin (A2 on).
+//   k_scan_*    A2: exclusive scan of the (material, energy bin) histogram.
+//   k_scatter   A2 on: permutation into (material, energy) order; A2 off:
+//               records into their material buckets.
+//   k_gather*   A4-A8 over material buckets (variants below; the default for
+//               energy-sorted batches is k_gather_s3, for unsorted batches
+//               k_gather), verification v = 1 + argmax fused, one atomic pair
+//               per block into vsum.
 #include <cfloat>
 #include <type_traits>
 
@@ -989,446 +982,6 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
   }
 }
 
-// ------------------------------------------- windowed sorted gather -------
-// k_gather_w: k_gather_t (U = 1) where each lane first orders its R lookups
-// by energy and loads a three-record window (k, k+1, k+2) of the lowest
-// lookup's bracket k: the lane's other lookups almost always lie in pair
-// (k, k+1) or (k+1, k+2), so a straddled grid point costs arithmetic, not a
-// dependent reload (which k_gather_t's source-level profile shows as the
-// main stall).  The grid allocation carries one padding record so that
-// k+2 is always addressable.
-template <int GT, int R, int MINB, bool CHECK>
-__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_w(Params P) {
-  constexpr int kTask = 32 * R;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
-  const int tab = P.n_mats * P.max_nucs;
-  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
-  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
-    const int32_t n = P.mats[t];
-    MatEntry me;
-    me.conc = P.concs[t];
-    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
-    me.n = n;
-    s_tab[t] = me;
-  }
-  if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      S.num[m] = P.num_nucs[m];
-      S.off[m] = run;
-      S.cnt[m] = c;
-      S.toff[m] = trun;
-      run += c;
-      trun += (c + kTask - 1) / kTask;
-    }
-    S.off[P.n_mats] = run;
-    S.toff[P.n_mats] = trun;
-  }
-  __syncthreads();
-
-  const int lane = threadIdx.x & 31;
-  const uint32_t total_tasks = S.toff[P.n_mats];
-  const uint32_t warps_per_block = blockDim.x >> 5;
-  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
-  const uint32_t nw = gridDim.x * warps_per_block;
-  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
-  const int32_t kmax = static_cast<int32_t>(P.N - 2);
-  constexpr bool kAllIdx = GT == XS_GRID_UNIONIZED;
-  constexpr int RK = kAllIdx ? R : 1;
-
-  unsigned long long acc_v = 0, acc_n = 0;
-  int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nw) {
-    while (task >= S.toff[m + 1]) ++m;
-    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
-    double p[R];
-    int32_t gidx[R];
-    uint32_t idx[R];
-    bool valid[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      valid[r] = slot0 + r < S.cnt[m];
-      LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = load_rec(P, S.off[m] + slot0 + r);
-      p[r] = rec.p;
-      gidx[r] = rec.gidx;
-      idx[r] = rec.idx;
-    }
-    // order the lane's lookups by energy (valid ones first): an odd-even
-    // transposition network over R registers
-#pragma unroll
-    for (int pass = 0; pass < R; ++pass) {
-#pragma unroll
-      for (int r = pass & 1; r + 1 < R; r += 2) {
-        const bool swap = (valid[r + 1] && !valid[r]) ||
-                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
-        if (swap) {
-          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
-          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
-          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
-          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
-        }
-      }
-    }
-    const int nn = S.num[m];
-    const MatEntry* row = s_tab + m * P.max_nucs;
-
-    auto bracket = [&](const MatEntry& me, int r) -> int32_t {
-      if (GT == XS_GRID_UNIONIZED) {
-        if (!P.index) return __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + gidx[r]);
-        return __ldg(P.index + static_cast<int64_t>(gidx[r]) * P.I + me.n);
-      }
-      const RowView<GT> rv(P, gidx[r]);
-      return rv.bracket(P, me.n, me.noff, p[r]);
-    };
-
-    double M[R][5];
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
-
-    int32_t knext[RK];
-#pragma unroll
-    for (int r = 0; r < RK; ++r) knext[r] = bracket(row[0], r);
-
-    for (int j = 0; j < nn; ++j) {
-      int32_t kc[RK];
-#pragma unroll
-      for (int r = 0; r < RK; ++r) {
-        kc[r] = knext[r];
-        knext[r] = j + 1 < nn ? bracket(row[j + 1], r) : 0;
-      }
-      const MatEntry me = row[j];
-      const int32_t kb = kc[0];  // bracket of the lane's lowest energy
-      // A5: window of records kb, kb+1, kb+2 (9 x 16 B)
-      double2 c[9];
-      {
-        const double2* pr = grid2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(kb)) * 3;
-#pragma unroll
-        for (int q = 0; q < 9; ++q) c[q] = __ldg(pr + q);
-      }
-      // pair (kb, kb+1): shared terms
-      const double bdA = dsub(c[3].x, c[0].x);
-      const double rcA = recip_nr(bdA);
-      const double dA0 = dsub(c[3].y, c[0].y);
-      const double dA1 = dsub(c[4].x, c[1].x);
-      const double dA2 = dsub(c[4].y, c[1].y);
-      const double dA3 = dsub(c[5].x, c[2].x);
-      const double dA4 = dsub(c[5].y, c[2].y);
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        int32_t kr = kb;
-        if (r > 0) {
-          if (kAllIdx) {
-            kr = kc[kAllIdx ? r : 0];
-          } else if (valid[r] && kb < kmax && p[r] >= c[3].x) {
-            kr = (kb + 1 == kmax || p[r] < c[6].x) ? kb + 1 : kb + 2;  // kb+2: walk on below
-          }
-        }
-        double x0, x1, x2, x3, x4;
-        if (kr == kb) {
-          const double an = dsub(c[3].x, p[r]);
-          double f = div_by_recip(an, bdA, rcA);
-          if (CHECK && !div_in_range(an, bdA)) f = ddiv(an, bdA);
-          x0 = dsub(c[3].y, dmul(f, dA0));
-          x1 = dsub(c[4].x, dmul(f, dA1));
-          x2 = dsub(c[4].y, dmul(f, dA2));
-          x3 = dsub(c[5].x, dmul(f, dA3));
-          x4 = dsub(c[5].y, dmul(f, dA4));
-        } else {
-          // pair (kb+1, kb+2) from the window, or (rare) a reload further on
-          double2 lo[3], hi[3];
-          if (kr == kb + 1) {
-#pragma unroll
-            for (int q = 0; q < 3; ++q) {
-              lo[q] = c[3 + q];
-              hi[q] = c[6 + q];
-            }
-          } else {
-            if (!kAllIdx) {  // exact local walk from kb+1
-              const double* rec = P.grid + static_cast<uint64_t>(me.noff) * 6;
-              kr = kb + 1;
-              while (kr < kmax && p[r] >= rec_energy(rec, kr + 1)) ++kr;
-            }
-            const double2* pr = grid2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(kr)) * 3;
-#pragma unroll
-            for (int q = 0; q < 3; ++q) {
-              lo[q] = __ldg(pr + q);
-              hi[q] = __ldg(pr + 3 + q);
-            }
-          }
-          const double bd = dsub(hi[0].x, lo[0].x);
-          const double an = dsub(hi[0].x, p[r]);
-          double f = div_nr(an, bd);
-          if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
-          x0 = dsub(hi[0].y, dmul(f, dsub(hi[0].y, lo[0].y)));
-          x1 = dsub(hi[1].x, dmul(f, dsub(hi[1].x, lo[1].x)));
-          x2 = dsub(hi[1].y, dmul(f, dsub(hi[1].y, lo[1].y)));
-          x3 = dsub(hi[2].x, dmul(f, dsub(hi[2].x, lo[2].x)));
-          x4 = dsub(hi[2].y, dmul(f, dsub(hi[2].y, lo[2].y)));
-        }
-        M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
-        M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
-        M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
-        M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
-        M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
-      }
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!valid[r]) continue;
-      double mx = -1.0;
-      int vi = 0;
-#pragma unroll
-      for (int c = 0; c < 5; ++c)
-        if (M[r][c] > mx) {
-          mx = M[r][c];
-          vi = c;
-        }
-      acc_v += static_cast<unsigned long long>(vi + 1);
-      acc_n += 1;
-      if (P.out_v) P.out_v[idx[r]] = vi + 1;
-      if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
-#pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
-    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
-  }
-  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
-  if (lane == 0) {
-    s_red[0][threadIdx.x >> 5] = acc_v;
-    s_red[1][threadIdx.x >> 5] = acc_n;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, n = 0;
-    for (uint32_t w = 0; w < warps_per_block; ++w) {
-      v += s_red[0][w];
-      n += s_red[1][w];
-    }
-    if (n) {
-      atomicAdd(P.vsum, v);
-      atomicAdd(P.vsum + 1, n);
-    }
-  }
-}
-
-// ------------------------------------------ pipelined sorted gather -------
-// k_gather_p: k_gather_t with a two-stage software pipeline over the
-// nuclide list: while nuclide j is interpolated, the record pair of j+1 is
-// already in flight and the index entries of j+2 are being read, so the
-// pair-load latency (the dominant stall of k_gather_t in ncu's source view)
-// overlaps a full nuclide of arithmetic.
-template <int GT, int R, int MINB, bool CHECK>
-__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_p(Params P) {
-  constexpr int kTask = 32 * R;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
-  const int tab = P.n_mats * P.max_nucs;
-  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
-  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
-    const int32_t n = P.mats[t];
-    MatEntry me;
-    me.conc = P.concs[t];
-    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
-    me.n = n;
-    s_tab[t] = me;
-  }
-  if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      S.num[m] = P.num_nucs[m];
-      S.off[m] = run;
-      S.cnt[m] = c;
-      S.toff[m] = trun;
-      run += c;
-      trun += (c + kTask - 1) / kTask;
-    }
-    S.off[P.n_mats] = run;
-    S.toff[P.n_mats] = trun;
-  }
-  __syncthreads();
-
-  const int lane = threadIdx.x & 31;
-  const uint32_t total_tasks = S.toff[P.n_mats];
-  const uint32_t warps_per_block = blockDim.x >> 5;
-  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
-  const uint32_t nw = gridDim.x * warps_per_block;
-  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
-  const int32_t kmax = static_cast<int32_t>(P.N - 2);
-  constexpr bool kAllIdx = GT == XS_GRID_UNIONIZED;
-  constexpr int RK = kAllIdx ? R : 1;
-
-  unsigned long long acc_v = 0, acc_n = 0;
-  int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nw) {
-    while (task >= S.toff[m + 1]) ++m;
-    const uint32_t slot0 = (task - S.toff[m]) * kTask + lane * R;
-    double p[R];
-    int32_t gidx[R];
-    uint32_t idx[R];
-    bool valid[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      valid[r] = slot0 + r < S.cnt[m];
-      LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = load_rec(P, S.off[m] + slot0 + r);
-      p[r] = rec.p;
-      gidx[r] = rec.gidx;
-      idx[r] = rec.idx;
-    }
-    const int nn = S.num[m];
-    const MatEntry* row = s_tab + m * P.max_nucs;
-
-    auto bracket = [&](const MatEntry& me, int r) -> int32_t {
-      if (GT == XS_GRID_UNIONIZED) {
-        if (!P.index) return __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + gidx[r]);
-        return __ldg(P.index + static_cast<int64_t>(gidx[r]) * P.I + me.n);
-      }
-      const RowView<GT> rv(P, gidx[r]);
-      return rv.bracket(P, me.n, me.noff, p[r]);
-    };
-    auto load_pair = [&](double2 (&c)[6], uint32_t off) {
-      const double2* pr = grid2 + static_cast<uint64_t>(off) * 3;
-#pragma unroll
-      for (int q = 0; q < 6; ++q) c[q] = __ldg(pr + q);
-    };
-
-    double M[R][5];
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
-
-    // pipeline state: kA = brackets of nuclide j+1, kB = of j+2, cN = pair of j+1
-    int32_t kA[RK], kB[RK];
-    double2 cN[6];
-#pragma unroll
-    for (int r = 0; r < RK; ++r) {
-      kA[r] = bracket(row[0], r);
-      kB[r] = nn > 1 ? bracket(row[1], r) : 0;
-    }
-    load_pair(cN, row[0].noff + static_cast<uint32_t>(kA[0]));
-
-    for (int j = 0; j < nn; ++j) {
-      double2 c[6];
-#pragma unroll
-      for (int q = 0; q < 6; ++q) c[q] = cN[q];
-      int32_t kc[RK];
-#pragma unroll
-      for (int r = 0; r < RK; ++r) {
-        kc[r] = kA[r];
-        kA[r] = kB[r];
-      }
-      const MatEntry me = row[j];
-      if (j + 1 < nn) load_pair(cN, row[j + 1].noff + static_cast<uint32_t>(kA[0]));
-      if (j + 2 < nn) {
-#pragma unroll
-        for (int r = 0; r < RK; ++r) kB[r] = bracket(row[j + 2], r);
-      }
-      // A6 + A7 for nuclide j (see k_gather_t)
-      int32_t k = kc[0];
-      double bd, rc, d0, d1, d2, d3, d4;
-      auto pair_terms = [&]() {
-        bd = dsub(c[3].x, c[0].x);
-        rc = recip_nr(bd);
-        d0 = dsub(c[3].y, c[0].y);
-        d1 = dsub(c[4].x, c[1].x);
-        d2 = dsub(c[4].y, c[1].y);
-        d3 = dsub(c[5].x, c[2].x);
-        d4 = dsub(c[5].y, c[2].y);
-      };
-      pair_terms();
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        if (r > 0) {
-          int32_t kr;
-          if (kAllIdx) {
-            kr = kc[kAllIdx ? r : 0];
-          } else {
-            kr = k;
-            if (valid[r]) {
-              const double* rec = P.grid + static_cast<uint64_t>(me.noff) * 6;
-              while (kr > 0 && p[r] < rec_energy(rec, kr)) --kr;
-              while (kr < kmax && p[r] >= rec_energy(rec, kr + 1)) ++kr;
-            }
-          }
-          if (kr != k) {  // rare: this lookup lies in another interval
-            k = kr;
-            load_pair(c, me.noff + static_cast<uint32_t>(k));
-            pair_terms();
-          }
-        }
-        const double an = dsub(c[3].x, p[r]);
-        double f = div_by_recip(an, bd, rc);
-        if (CHECK && !div_in_range(an, bd)) f = ddiv(an, bd);
-        const double x0 = dsub(c[3].y, dmul(f, d0));
-        const double x1 = dsub(c[4].x, dmul(f, d1));
-        const double x2 = dsub(c[4].y, dmul(f, d2));
-        const double x3 = dsub(c[5].x, dmul(f, d3));
-        const double x4 = dsub(c[5].y, dmul(f, d4));
-        M[r][0] = dadd(M[r][0], dmul(x0, me.conc));
-        M[r][1] = dadd(M[r][1], dmul(x1, me.conc));
-        M[r][2] = dadd(M[r][2], dmul(x2, me.conc));
-        M[r][3] = dadd(M[r][3], dmul(x3, me.conc));
-        M[r][4] = dadd(M[r][4], dmul(x4, me.conc));
-      }
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!valid[r]) continue;
-      double mx = -1.0;
-      int vi = 0;
-#pragma unroll
-      for (int c = 0; c < 5; ++c)
-        if (M[r][c] > mx) {
-          mx = M[r][c];
-          vi = c;
-        }
-      acc_v += static_cast<unsigned long long>(vi + 1);
-      acc_n += 1;
-      if (P.out_v) P.out_v[idx[r]] = vi + 1;
-      if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
-#pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
-    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
-  }
-  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
-  if (lane == 0) {
-    s_red[0][threadIdx.x >> 5] = acc_v;
-    s_red[1][threadIdx.x >> 5] = acc_n;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, n = 0;
-    for (uint32_t w = 0; w < warps_per_block; ++w) {
-      v += s_red[0][w];
-      n += s_red[1][w];
-    }
-    if (n) {
-      atomicAdd(P.vsum, v);
-      atomicAdd(P.vsum + 1, n);
-    }
-  }
-}
-
 // ------------------------------------------- TMA-staged sorted gather ------
 // k_gather_s: for energy-sorted batches.  A warp owns a task of 32*R
 // consecutive lookups of one material (lane l: lookups R*l..R*l+R-1, ordered
@@ -1715,347 +1268,26 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
   }
 }
 
-// -------------------------------------- TMA-staged sorted gather, v2 ------
-// k_gather_s2: the k_gather_s decomposition (warp = task of 32*R energy-sorted
-// lookups of one material, lane = R consecutive lookups, per-nuclide record
-// window [k_lo, k_hi + 1] staged in shared memory by TMA bulk copies) with
-// the per-nuclide instruction overhead cut:
-//  * the window is read with shared-memory loads (LDS) on its own code path;
-//    windows longer than W records take a separate global-memory path (never
-//    a generic pointer that merges the two);
-//  * each lane finds the brackets of its first and last lookup with a
-//    warp-uniform binary lifting over the window's interior energies; when
-//    every lane's lookups share one record pair (the common case: a task spans
-//    ~0.6 intervals of a fuel nuclide), the R interpolations run as one
-//    straight-line block with no per-lookup test, so the compiler interleaves
-//    R independent FP64 chains; otherwise lanes walk their lookups through
-//    the window as in k_gather_s;
-//  * the bulk copies are issued D at a time by D lanes in parallel into a
-//    ring of 2D slots (D to 2D nuclides ahead), not one per nuclide by lane 0.
-// Arithmetic and order are those of k_gather_s (bit-identical results).
-template <int R>
-struct PairTerms {
-  double hiE, bd, rc, h[5], d[5];
-};
-
-template <int R, bool CHECK>
-__device__ __forceinline__ void pair_terms_of(const double2 (&c)[6], PairTerms<R>& t) {
-  t.hiE = c[3].x;
-  t.bd = dsub(c[3].x, c[0].x);
-  t.rc = recip_nr(t.bd);
-  t.h[0] = c[3].y;
-  t.h[1] = c[4].x;
-  t.h[2] = c[4].y;
-  t.h[3] = c[5].x;
-  t.h[4] = c[5].y;
-  t.d[0] = dsub(c[3].y, c[0].y);
-  t.d[1] = dsub(c[4].x, c[1].x);
-  t.d[2] = dsub(c[4].y, c[1].y);
-  t.d[3] = dsub(c[5].x, c[2].x);
-  t.d[4] = dsub(c[5].y, c[2].y);
-}
-
-// A6 + A7 for one lookup at energy p with the pair terms t (R10/R11)
-template <int R, bool CHECK>
-__device__ __forceinline__ void interp_acc(const PairTerms<R>& t, double p, double conc,
-                                           double (&M)[5]) {
-  const double an = dsub(t.hiE, p);
-  double f = div_by_recip(an, t.bd, t.rc);
-  if (CHECK && !div_in_range(an, t.bd)) f = ddiv(an, t.bd);
-#pragma unroll
-  for (int c = 0; c < 5; ++c) M[c] = dadd(M[c], dmul(dsub(t.h[c], dmul(f, t.d[c])), conc));
-}
-
-// One nuclide of a task: win = records k_lo .. k_lo + n_int + 1 (shared or
-// global memory), lookups p[0..R-1] ascending.
-template <int R, bool CHECK, bool SHARED>
-__device__ __forceinline__ void stage_nuclide(const double2* win, int n_int, double conc,
-                                              const double (&p)[R], double (&M)[R][5]) {
-  auto E = [&](int t) -> double { return SHARED ? win[t * 3].x : __ldg(&win[t * 3].x); };
-  auto load = [&](int k, double2 (&c)[6]) {
-    const double2* pr = win + k * 3;
-#pragma unroll
-    for (int q = 0; q < 6; ++q) c[q] = SHARED ? pr[q] : __ldg(pr + q);
-  };
-  // bracket offsets (within the window) of the lane's first and last lookup:
-  // i = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p}
-  int i0 = 0, iL = 0;
-  if (n_int > 0) {
-    for (int step = 1 << (31 - __clz(n_int)); step > 0; step >>= 1) {
-      if (i0 + step <= n_int && E(i0 + step) <= p[0]) i0 += step;
-      if (iL + step <= n_int && E(iL + step) <= p[R - 1]) iL += step;
-    }
-  }
-  double2 c[6];
-  PairTerms<R> t;
-  if (__all_sync(0xffffffffu, i0 == iL)) {
-    load(i0, c);
-    pair_terms_of<R, CHECK>(c, t);
-#pragma unroll
-    for (int r = 0; r < R; ++r) interp_acc<R, CHECK>(t, p[r], conc, M[r]);
-    return;
-  }
-  int k = i0;
-  load(k, c);
-  pair_terms_of<R, CHECK>(c, t);
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    if (r > 0 && k < iL && p[r] >= t.hiE) {
-      if (SHARED) {
-        ++k;
-        while (k < iL && E(k + 1) <= p[r]) ++k;
-      } else {
-        int lo = k + 1, hi = iL + 1;  // E[lo] <= p < E[hi] (hi = iL + 1: p[r] <= p[R-1])
-        while (hi - lo > 1) {
-          const int mid = (lo + hi) >> 1;
-          if (E(mid) <= p[r])
-            lo = mid;
-          else
-            hi = mid;
-        }
-        k = lo;
-      }
-      load(k, c);
-      pair_terms_of<R, CHECK>(c, t);
-    }
-    interp_acc<R, CHECK>(t, p[r], conc, M[r]);
-  }
-}
-
-template <int GT, int R, int D, int W, int NW, bool CHECK>
-__global__ void __launch_bounds__(32 * NW, 1) k_gather_s2(Params P) {
-  constexpr int kTask = 32 * R;
-  constexpr int S = 2 * D;  // window slots per warp
-  static_assert(D <= 32 && S <= 32, "slots");
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
-  const int tab = P.n_mats * P.max_nucs;
-  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
-  constexpr size_t win_bytes = static_cast<size_t>(S) * W * 48;
-  const size_t k_bytes = ((static_cast<size_t>(P.max_nucs) * 8 + 15) / 16) * 16;
-  constexpr size_t bar_bytes = ((S * 8 + 15) / 16) * 16;
-  const size_t per_warp = win_bytes + k_bytes + bar_bytes;
-  unsigned char* mine = wbase + per_warp * warp;
-  double2* s_win = reinterpret_cast<double2*>(mine);               // [S][W*3]
-  int2* s_k = reinterpret_cast<int2*>(mine + win_bytes);           // [max_nucs] {k_lo, k_hi}
-  uint64_t* s_bar = reinterpret_cast<uint64_t*>(mine + win_bytes + k_bytes);
-
-  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
-    const int32_t n = P.mats[i];
-    MatEntry me;
-    me.conc = P.concs[i];
-    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
-    me.n = n;
-    s_tab[i] = me;
-  }
-  if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      G.num[m] = P.num_nucs[m];
-      G.off[m] = run;
-      G.cnt[m] = c;
-      G.toff[m] = trun;
-      run += c;
-      trun += (c + kTask - 1) / kTask;
-    }
-    G.off[P.n_mats] = run;
-    G.toff[P.n_mats] = trun;
-  }
-  if (lane == 0) {
-    for (int d = 0; d < S; ++d) mbar_init(&s_bar[d], 1);
-    mbar_fence_init();
-  }
-  __syncthreads();
-
-  const uint32_t total_tasks = G.toff[P.n_mats];
-  const uint32_t gw = blockIdx.x * NW + warp;
-  const uint32_t nwarps = gridDim.x * NW;
-  const double2* __restrict__ grid2 = reinterpret_cast<const double2*>(P.grid);
-  uint32_t phase = 0;  // parity bit per slot
-
-  unsigned long long acc_v = 0, acc_n = 0;
-  int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
-    while (task >= G.toff[m + 1]) ++m;
-    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
-    double p[R];
-    int32_t gidx[R];
-    uint32_t idx[R];
-    bool valid[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      valid[r] = slot0 + r < G.cnt[m];
-      LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
-      p[r] = rec.p;
-      gidx[r] = rec.gidx;
-      idx[r] = rec.idx;
-    }
-#pragma unroll
-    for (int pass = 0; pass < R; ++pass) {
-#pragma unroll
-      for (int r = pass & 1; r + 1 < R; r += 2) {
-        const bool swap = (valid[r + 1] && !valid[r]) ||
-                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
-        if (swap) {
-          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
-          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
-          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
-          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
-        }
-      }
-    }
-    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
-    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (valid[r]) {
-        phi = p[r];
-        uhi = gidx[r];
-      }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
-      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
-      plo = a < plo ? a : plo;
-      phi = b > phi ? b : phi;
-    }
-    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
-      ulo = union_index_tab(P, plo);
-      uhi = union_index_tab(P, phi);
-    } else {
-      ulo = __reduce_min_sync(0xffffffffu, ulo);
-      uhi = __reduce_max_sync(0xffffffffu, uhi);
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
-    const int nn = G.num[m];
-    const MatEntry* row = s_tab + m * P.max_nucs;
-    // A4 for the two extremes of every nuclide of the material
-    for (int j = lane; j < nn; j += 32) {
-      const MatEntry me = row[j];
-      int32_t klo, khi;
-      if (GT == XS_GRID_UNIONIZED) {
-        if (P.index_t) {
-          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
-          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
-        } else {
-          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
-          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
-        }
-      } else {
-        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
-        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
-        klo = rlo.bracket(P, me.n, me.noff, plo);
-        khi = rhi.bracket(P, me.n, me.noff, phi);
-      }
-      s_k[j] = make_int2(klo, khi);
-    }
-    __syncwarp();
-    // A5 producer: lanes 0..D-1 stage the windows of nuclides g*D .. g*D+D-1
-    auto issue_group = [&](int g) {
-      const int j = g * D + lane;
-      if (lane < D && j < nn) {
-        const int slot = j % S;
-        const int2 kk = s_k[j];
-        const int32_t w = kk.y - kk.x + 2;  // records k_lo .. k_hi + 1
-        if (w <= W) {
-          const double2* src = grid2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * 3;
-          mbar_arrive_expect_tx(&s_bar[slot], static_cast<uint32_t>(w) * 48u);
-          bulk_copy_g2s(s_win + slot * W * 3, src, static_cast<uint32_t>(w) * 48u, &s_bar[slot]);
-        } else {
-          mbar_arrive_expect_tx(&s_bar[slot], 0u);  // read in place from global memory
-        }
-      }
-    };
-    issue_group(0);
-    issue_group(1);
-
-    double M[R][5];
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
-
-    for (int j = 0; j < nn; ++j) {
-      const int slot = j % S;
-      if (j >= D && j % D == 0) {
-        __syncwarp();  // every lane is done with the slots of group j/D - 1
-        issue_group(j / D + 1);
-      }
-      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
-      phase ^= 1u << slot;
-      const double conc = row[j].conc;
-      const int2 kk = s_k[j];
-      const int n_int = kk.y - kk.x;
-      if (n_int + 2 <= W) {
-        stage_nuclide<R, CHECK, true>(s_win + slot * W * 3, n_int, conc, p, M);
-      } else {
-        const double2* gw2 = grid2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * 3;
-        stage_nuclide<R, CHECK, false>(gw2, n_int, conc, p, M);
-      }
-    }
-    __syncwarp();  // all slots consumed before the next task reuses them
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!valid[r]) continue;
-      double mx = -1.0;
-      int vi = 0;
-#pragma unroll
-      for (int c = 0; c < 5; ++c)
-        if (M[r][c] > mx) {
-          mx = M[r][c];
-          vi = c;
-        }
-      acc_v += static_cast<unsigned long long>(vi + 1);
-      acc_n += 1;
-      if (P.out_v) P.out_v[idx[r]] = vi + 1;
-      if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
-#pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
-    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
-  }
-  __shared__ unsigned long long s_red[2][NW];
-  if (lane == 0) {
-    s_red[0][warp] = acc_v;
-    s_red[1][warp] = acc_n;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, n = 0;
-    for (int w = 0; w < NW; ++w) {
-      v += s_red[0][w];
-      n += s_red[1][w];
-    }
-    if (n) {
-      atomicAdd(P.vsum, v);
-      atomicAdd(P.vsum + 1, n);
-    }
-  }
-}
-
 // ------------------------------- TMA-staged sorted gather, interval table --
-// k_gather_s3: as k_gather_s2, but the window holds entries of the interval
-// table (grid_build.cu K0d: per record pair {E[k+1], gap, recip(gap), hi.c,
-// hi.c - lo.c}) instead of raw records, so no pair-only arithmetic (5 DFMA
-// reciprocal chain + 6 subtractions) runs in the timed loop: a lookup is
-// 4 FP64 ops for f and 4 per channel.  Each lane locates every lookup's
-// interval in the window by warp-uniform binary lifting; when all lanes'
-// lookups share one interval the R interpolations run as one straight-line
-// block, otherwise a lane reloads the 7 x 16 B entry (shared memory) only
-// when the interval changes.  Bit-identical to k_gather_s.
+// k_gather_s3 (default for energy-sorted batches): the k_gather_s
+// decomposition (warp = task of 32*R energy-sorted lookups of one material,
+// lane = R consecutive lookups, per-nuclide window [k_lo, k_hi] staged in
+// shared memory by TMA bulk copies), with the window holding entries of the
+// interval table (grid_build.cu K0d: per record pair {E[k+1], gap,
+// recip(gap), hi.c, hi.c - lo.c}) instead of raw records, so no pair-only
+// arithmetic (5-DFMA reciprocal chain, 6 subtractions) runs in the timed
+// loop: a lookup costs 4 FP64 ops for f and 4 per channel.
+//  * Each lane finds the window entries of its first and last lookup by
+//    warp-uniform binary lifting over the entries' upper energies (loads
+//    clamped, no branches).  When every lane's lookups share one entry (the
+//    common case: a fuel task spans ~0.6 intervals of a nuclide) the R
+//    interpolations run as one straight-line block (R independent FP64
+//    chains); otherwise every lookup reads its own entry.
+//  * Windows are read with shared-memory loads on their own code path;
+//    windows longer than W entries (sparse tasks) take a global-memory path.
+//  * Bulk copies are issued D at a time by D lanes into a ring of 2D slots
+//    (D to 2D nuclides ahead), completing on per-slot mbarriers.
+// Same operations in the same order as the oracle (bit-identical M).
 // Entry layout (7 x 16 B): {E[k+1], gap} {recip(gap), 0} {hi.c, hi.c - lo.c} x 5.
 // A6 + A7 for lookups r in [r0, r1) that all lie in entry q (channel terms are
 // read from the window per channel to keep register pressure low).
@@ -2083,42 +1315,10 @@ __device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R]
   }
 }
 
-// A6 + A7 for lookups in (possibly) different entries i[r] of the window:
-// the entry terms are reloaded (predicated) only where the entry changes
-// between a lane's consecutive lookups.
-template <int R, bool CHECK, bool SHARED>
-__device__ __forceinline__ void iv_interp_var(const double2* win, const int (&i)[R],
-                                              const double (&p)[R], double conc,
-                                              double (&M)[R][5]) {
-  constexpr int kE = kIvDoubles / 2;
-  auto ld = [&](int u) -> double2 { return SHARED ? win[u] : __ldg(win + u); };
-  double f[R];
-  double2 a0 = ld(i[0] * kE), a1 = ld(i[0] * kE + 1);
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    if (r > 0 && i[r] != i[r - 1]) {
-      a0 = ld(i[r] * kE);
-      a1 = ld(i[r] * kE + 1);
-    }
-    const double an = dsub(a0.x, p[r]);
-    f[r] = div_by_recip(an, a0.y, a1.x);
-    if (CHECK && !div_in_range(an, a0.y)) f[r] = ddiv(an, a0.y);
-  }
-#pragma unroll
-  for (int c = 0; c < 5; ++c) {
-    double2 hd = ld(i[0] * kE + 2 + c);
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (r > 0 && i[r] != i[r - 1]) hd = ld(i[r] * kE + 2 + c);
-      M[r][c] = dadd(M[r][c], dmul(dsub(hd.x, dmul(f[r], hd.y)), conc));
-    }
-  }
-}
-
 // One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
 // i(p) = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p} by binary lifting
 // (warp-uniform trip count; loads clamped so the loop has no branches).
-template <int R, bool CHECK, bool SHARED, bool PRED = false>
+template <int R, bool CHECK, bool SHARED>
 __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
                                                  const double (&p)[R], double (&M)[R][5]) {
   constexpr int kE = kIvDoubles / 2;
@@ -2154,92 +1354,11 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
       }
     }
   }
-  if (PRED) {
-    iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
-    return;
-  }
 #pragma unroll
   for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
 }
 
-// Second half of stage_nuclide_iv for a caller that already lifted the first
-// and last lookup (i0, iL): the software-pipelined loop of k_gather_s3 MODE 2.
-template <int R, bool CHECK, bool SHARED, bool PRED = false>
-__device__ __forceinline__ void stage_apply_iv(const double2* win, int n_int, double conc,
-                                               const double (&p)[R], double (&M)[R][5], int i0,
-                                               int iL) {
-  constexpr int kE = kIvDoubles / 2;
-  auto E = [&](int t) -> double {
-    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
-    return SHARED ? q[0] : __ldg(q);
-  };
-  if (__all_sync(0xffffffffu, i0 == iL)) {
-    iv_interp<R, CHECK, SHARED>(win + i0 * kE, p, conc, M, 0, R);
-    return;
-  }
-  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
-  int i[R];
-  i[0] = i0;
-  i[R - 1] = iL;
-#pragma unroll
-  for (int r = 1; r < R - 1; ++r) i[r] = i0;
-  if (R > 2) {
-    for (int step = top; step > 0; step >>= 1) {
-#pragma unroll
-      for (int r = 1; r < R - 1; ++r) {
-        const int t = i[r] + step;
-        const double e = E(t <= n_int ? t : n_int);
-        if (t <= n_int && e <= p[r]) i[r] = t;
-      }
-    }
-  }
-  if (PRED) {
-    iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
-    return;
-  }
-#pragma unroll
-  for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
-}
-
-// Branch-free variant: every lookup's entry index by binary lifting, the
-// entry terms reloaded (predicated) only where the index changes between a
-// lane's consecutive lookups; one straight-line block per nuclide.
-template <int R, bool CHECK, bool SHARED>
-__device__ __forceinline__ void stage_nuclide_iv_pred(const double2* win, int n_int, double conc,
-                                                      const double (&p)[R], double (&M)[R][5]) {
-  constexpr int kE = kIvDoubles / 2;
-  auto ld = [&](int u) -> double2 { return SHARED ? win[u] : __ldg(win + u); };
-  auto E = [&](int t) -> double {
-    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
-    return SHARED ? q[0] : __ldg(q);
-  };
-  int i[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) i[r] = 0;
-  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
-  for (int step = top; step > 0; step >>= 1) {
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      const int t = i[r] + step;
-      const double e = E(t <= n_int ? t : n_int);
-      if (t <= n_int && e <= p[r]) i[r] = t;
-    }
-  }
-  iv_interp_var<R, CHECK, SHARED>(win, i, p, conc, M);
-}
-
-template <int R, int MODE, bool CHECK, bool SHARED>
-__device__ __forceinline__ void stage_nuclide_sel(const double2* win, int n_int, double conc,
-                                                  const double (&p)[R], double (&M)[R][5]) {
-  if (MODE == 1)
-    stage_nuclide_iv_pred<R, CHECK, SHARED>(win, n_int, conc, p, M);
-  else if (MODE == 3)
-    stage_nuclide_iv<R, CHECK, SHARED, true>(win, n_int, conc, p, M);
-  else
-    stage_nuclide_iv<R, CHECK, SHARED>(win, n_int, conc, p, M);
-}
-
-template <int GT, int R, int D, int W, int NW, bool CHECK, int MODE = 0>
+template <int GT, int R, int D, int W, int NW, bool CHECK>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   constexpr int kTask = 32 * R;
   constexpr int S = 2 * D;               // window slots per warp
@@ -2402,325 +1521,24 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 #pragma unroll
       for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
 
-    if constexpr (MODE == 2) {
-      // software-pipelined: the barrier wait, table reads and first lifting
-      // step of nuclide j+1 are issued before the interpolation of nuclide j,
-      // so their latency hides behind it
-      constexpr int kE = kIvDoubles / 2;
-      struct Head {
-        double conc, etop;
-        int n_int, top, woff, j;
-      };
-      auto head_load = [&](int j, Head& h) {
-        const int slot = j % S;
-        mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
-        phase ^= 1u << slot;
-        h.j = j;
-        h.conc = row[j].conc;
-        const int2 kk = s_k[j];
-        h.n_int = kk.y - kk.x;
-        h.top = h.n_int > 0 ? 1 << (31 - __clz(h.n_int)) : 0;
-        h.woff = slot * W * kE;
-        h.etop = 0.0;
-        if (h.n_int > 0 && h.n_int < W)  // E[k_lo + top] (every lane's first probe)
-          h.etop = reinterpret_cast<const double*>(s_win + h.woff + (h.top - 1) * kE)[0];
-      };
-      auto head_lift = [&](const Head& h, int& i0, int& iL) {
-        i0 = iL = 0;
-        if (h.n_int <= 0 || h.n_int >= W) return;
-        if (h.etop <= p[0]) i0 = h.top;
-        if (h.etop <= p[R - 1]) iL = h.top;
-        const double2* win = s_win + h.woff;
-        for (int step = h.top >> 1; step > 0; step >>= 1) {
-          const int t0 = i0 + step, tL = iL + step;
-          const double e0 = reinterpret_cast<const double*>(win + ((t0 <= h.n_int ? t0 : h.n_int) - 1) * kE)[0];
-          const double eL = reinterpret_cast<const double*>(win + ((tL <= h.n_int ? tL : h.n_int) - 1) * kE)[0];
-          if (t0 <= h.n_int && e0 <= p[0]) i0 = t0;
-          if (tL <= h.n_int && eL <= p[R - 1]) iL = tL;
-        }
-      };
-      Head cur, nxt;
-      int i0 = 0, iL = 0;
-      if (nn > 0) {
-        head_load(0, cur);
-        head_lift(cur, i0, iL);
-      }
-      for (int j = 0; j < nn; ++j) {
-        if (j >= D && j % D == 0) {
-          __syncwarp();  // every lane is done with the slots of group j/D - 1
-          issue_group(j / D + 1);
-        }
-        const bool more = j + 1 < nn;
-        if (more) head_load(j + 1, nxt);
-        if (cur.n_int < W) {
-          stage_apply_iv<R, CHECK, true>(s_win + cur.woff, cur.n_int, cur.conc, p, M, i0, iL);
-        } else {
-          const int2 kk = s_k[j];
-          const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
-          stage_nuclide_iv<R, CHECK, false>(g2, cur.n_int, cur.conc, p, M);
-        }
-        if (more) {
-          cur = nxt;
-          head_lift(cur, i0, iL);
-        }
-      }
-    } else {
-      for (int j = 0; j < nn; ++j) {
-        const int slot = j % S;
-        if (j >= D && j % D == 0) {
-          __syncwarp();  // every lane is done with the slots of group j/D - 1
-          issue_group(j / D + 1);
-        }
-        mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
-        phase ^= 1u << slot;
-        const double conc = row[j].conc;
-        const int2 kk = s_k[j];
-        const int n_int = kk.y - kk.x;
-        if (n_int < W) {
-          stage_nuclide_sel<R, MODE, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
-        } else {
-          const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
-          stage_nuclide_sel<R, MODE, CHECK, false>(g2, n_int, conc, p, M);
-        }
-      }
-    }
-    __syncwarp();
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!valid[r]) continue;
-      double mx = -1.0;
-      int vi = 0;
-#pragma unroll
-      for (int c = 0; c < 5; ++c)
-        if (M[r][c] > mx) {
-          mx = M[r][c];
-          vi = c;
-        }
-      acc_v += static_cast<unsigned long long>(vi + 1);
-      acc_n += 1;
-      if (P.out_v) P.out_v[idx[r]] = vi + 1;
-      if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
-#pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
-    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
-  }
-  __shared__ unsigned long long s_red[2][NW];
-  if (lane == 0) {
-    s_red[0][warp] = acc_v;
-    s_red[1][warp] = acc_n;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, n = 0;
-    for (int w = 0; w < NW; ++w) {
-      v += s_red[0][w];
-      n += s_red[1][w];
-    }
-    if (n) {
-      atomicAdd(P.vsum, v);
-      atomicAdd(P.vsum + 1, n);
-    }
-  }
-}
-
-template <int GT, int R, int D, int CAP, int NW, bool CHECK>
-__global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
-  constexpr int kTask = 32 * R;
-  constexpr int kE = kIvDoubles / 2;       // 16-B chunks per interval entry
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
-  const int tab = P.n_mats * P.max_nucs;
-  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab + tab);
-  constexpr size_t buf_bytes = static_cast<size_t>(2) * CAP * kIvDoubles * 8;
-  const size_t k_bytes = ((static_cast<size_t>(P.max_nucs) * 8 + 15) / 16) * 16;
-  unsigned char* mine = wbase + (buf_bytes + k_bytes) * warp;
-  double2* s_buf = reinterpret_cast<double2*>(mine);               // [2][CAP * 7]
-  int2* s_k = reinterpret_cast<int2*>(mine + buf_bytes);           // [max_nucs] {k_lo, k_hi}
-
-  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
-    const int32_t n = P.mats[i];
-    MatEntry me;
-    me.conc = P.concs[i];
-    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
-    me.n = n;
-    s_tab[i] = me;
-  }
-  if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      G.num[m] = P.num_nucs[m];
-      G.off[m] = run;
-      G.cnt[m] = c;
-      G.toff[m] = trun;
-      run += c;
-      trun += (c + kTask - 1) / kTask;
-    }
-    G.off[P.n_mats] = run;
-    G.toff[P.n_mats] = trun;
-  }
-  __syncthreads();
-
-  const uint32_t total_tasks = G.toff[P.n_mats];
-  const uint32_t gw = blockIdx.x * NW + warp;
-  const uint32_t nwarps = gridDim.x * NW;
-  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(P.iv);
-
-  unsigned long long acc_v = 0, acc_n = 0;
-  int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
-    while (task >= G.toff[m + 1]) ++m;
-    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
-    double p[R];
-    int32_t gidx[R];
-    uint32_t idx[R];
-    bool valid[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      valid[r] = slot0 + r < G.cnt[m];
-      LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
-      p[r] = rec.p;
-      gidx[r] = rec.gidx;
-      idx[r] = rec.idx;
-    }
-#pragma unroll
-    for (int pass = 0; pass < R; ++pass) {
-#pragma unroll
-      for (int r = pass & 1; r + 1 < R; r += 2) {
-        const bool swap = (valid[r + 1] && !valid[r]) ||
-                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
-        if (swap) {
-          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
-          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
-          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
-          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
-        }
-      }
-    }
-    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
-    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (valid[r]) {
-        phi = p[r];
-        uhi = gidx[r];
-      }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
-      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
-      plo = a < plo ? a : plo;
-      phi = b > phi ? b : phi;
-    }
-    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
-      ulo = union_lower_tab(P, plo);
-      uhi = union_upper_tab(P, phi);
-    } else {
-      ulo = __reduce_min_sync(0xffffffffu, ulo);
-      uhi = __reduce_max_sync(0xffffffffu, uhi);
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
-    const int nn = G.num[m];
-    const MatEntry* row = s_tab + m * P.max_nucs;
-    // A4 for the two extremes of every nuclide of the material
-    for (int j = lane; j < nn; j += 32) {
-      const MatEntry me = row[j];
-      int32_t klo, khi;
-      if (GT == XS_GRID_UNIONIZED) {
-        if (P.index_t) {
-          klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
-          khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
-        } else {
-          klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
-          khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
-        }
-      } else {
-        const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
-        const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
-        klo = rlo.bracket(P, me.n, me.noff, plo);
-        khi = rhi.bracket(P, me.n, me.noff, phi);
-      }
-      s_k[j] = make_int2(klo, khi);
-    }
-    __syncwarp();
-    // A5: the windows (entries k_lo .. k_hi) of the D nuclides of group g
-    // are packed in order into buffer g & 1 (CAP entries; a window that does
-    // not fit is read in place from global memory) by per-lane 16-B async
-    // copies, one commit group per nuclide group.
-    auto issue_group = [&](int g) {
-      const int j0 = g * D;
-      int off[D], w[D];
-      uint32_t src[D];
-      int tot = 0;
-#pragma unroll
-      for (int t = 0; t < D; ++t) {
-        w[t] = 0;
-        off[t] = tot;
-        src[t] = 0;
-        if (j0 + t < nn) {
-          const int2 kk = s_k[j0 + t];
-          const int wt = kk.y - kk.x + 1;
-          if (tot + wt <= CAP) {
-            w[t] = wt;
-            src[t] = row[j0 + t].noff + static_cast<uint32_t>(kk.x);
-            tot += wt;
-          }
-        }
-      }
-      double2* dst = s_buf + (g & 1) * CAP * kE;
-      for (int c = lane; c < tot * kE; c += 32) {
-        const int e = c / kE, part = c - e * kE;
-        uint32_t rec = 0;
-#pragma unroll
-        for (int t = 0; t < D; ++t)
-          if (e >= off[t] && e < off[t] + w[t]) rec = src[t] + static_cast<uint32_t>(e - off[t]);
-        cp_async16(dst + c, iv2 + static_cast<uint64_t>(rec) * kE + part);
-      }
-      cp_async_commit();
-    };
-    issue_group(0);
-
-    double M[R][5];
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
-
-    int coff = 0;
     for (int j = 0; j < nn; ++j) {
-      if (j % D == 0) {
-        __syncwarp();  // every lane is done with buffer (j/D + 1) & 1
+      const int slot = j % S;
+      if (j >= D && j % D == 0) {
+        __syncwarp();  // every lane is done with the slots of group j/D - 1
         issue_group(j / D + 1);
-        cp_async_wait<1>();  // this lane's copies of group j/D have landed
-        __syncwarp();        // ... and every other lane's
-        coff = 0;
       }
+      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
+      phase ^= 1u << slot;
       const double conc = row[j].conc;
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
-      if (coff + n_int + 1 <= CAP) {
-        stage_nuclide_iv<R, CHECK, true>(s_buf + ((j / D) & 1) * CAP * kE + coff * kE, n_int, conc,
-                                         p, M);
-        coff += n_int + 1;
+      if (n_int < W) {
+        stage_nuclide_iv<R, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
       } else {
-        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
+        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
         stage_nuclide_iv<R, CHECK, false>(g2, n_int, conc, p, M);
       }
     }
-    cp_async_wait<0>();
     __syncwarp();
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -2954,40 +1772,6 @@ static cudaError_t launch_gather_t(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
-template <int GT, int R, int MINB, bool CHECK>
-static cudaError_t launch_gather_p(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
-  auto kern = k_gather_p<GT, R, MINB, CHECK>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = g.blocks_per_sm;
-  if (per_sm <= 0) {
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-  }
-  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
-  return cudaGetLastError();
-}
-
-template <int GT, int R, int MINB, bool CHECK>
-static cudaError_t launch_gather_w(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
-  auto kern = k_gather_w<GT, R, MINB, CHECK>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = g.blocks_per_sm;
-  if (per_sm <= 0) {
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-  }
-  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
-  return cudaGetLastError();
-}
-
 template <int GT, int R, int D, int W, int NW, bool CHECK>
 static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   const size_t win_bytes = static_cast<size_t>(D) * W * 48;
@@ -3010,55 +1794,13 @@ static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStr
 }
 
 template <int GT, int R, int D, int W, int NW, bool CHECK>
-static cudaError_t launch_gather_s2(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * 48;
-  const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
-  const size_t smem = sizeof(GatherSmem) +
-                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
-                      NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
-  auto kern = k_gather_s2<GT, R, D, W, NW, CHECK>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = g.blocks_per_sm;
-  if (per_sm <= 0) {
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-  }
-  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
-  return cudaGetLastError();
-}
-
-template <int GT, int R, int D, int W, int NW, bool CHECK, int MODE = 0>
 static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * kIvDoubles * 8;
   const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
   const size_t smem = sizeof(GatherSmem) +
                       static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
                       NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
-  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK, MODE>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = g.blocks_per_sm;
-  if (per_sm <= 0) {
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-  }
-  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
-  return cudaGetLastError();
-}
-
-template <int GT, int R, int D, int CAP, int NW, bool CHECK>
-static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  constexpr size_t buf_bytes = static_cast<size_t>(2) * CAP * kIvDoubles * 8;
-  const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
-  const size_t smem = sizeof(GatherSmem) +
-                      static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
-                      NW * (buf_bytes + k_bytes);
-  auto kern = k_gather_s4<GT, R, D, CAP, NW, CHECK>;
+  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -3075,9 +1817,9 @@ static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaSt
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
-  // blocks); 5-6 pipelined; 7-8 windowed; 9-12 TMA-staged (R, stages D,
-  // window W records, warps per block); 13-16 TMA-staged v2; 17-20
-  // TMA-staged from the interval table.  Measured best on B200 (large,
+  // blocks); 9-12 TMA-staged record windows (R, stages D, window W records,
+  // warps per block); 17-20 TMA-staged interval-table windows (R, group
+  // size D, window W entries, warps per block).  Measured best on B200 (large,
   // large-hash, small): k_gather_s3 (4, 2, 8, 16) = variant 19.
   int v = g.unroll;
   if (v == 0) v = 19;
@@ -3086,32 +1828,14 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
     case 3: return launch_gather_t<GT, 2, 1, 3, CHECK>(g, P, st);
     case 4: return launch_gather_t<GT, 4, 2, 2, CHECK>(g, P, st);
-    case 5: return launch_gather_p<GT, 4, 1, CHECK>(g, P, st);
-    case 6: return launch_gather_p<GT, 4, 2, CHECK>(g, P, st);
-    case 7: return launch_gather_w<GT, 4, 2, CHECK>(g, P, st);
-    case 8: return launch_gather_w<GT, 2, 3, CHECK>(g, P, st);
     case 9: return launch_gather_s<GT, 4, 4, 16, 16, CHECK>(g, P, st);
     case 10: return launch_gather_s<GT, 4, 3, 16, 16, CHECK>(g, P, st);
     case 11: return launch_gather_s<GT, 4, 6, 12, 16, CHECK>(g, P, st);
     case 12: return launch_gather_s<GT, 4, 4, 12, 8, CHECK>(g, P, st);
-    case 13: return launch_gather_s2<GT, 4, 4, 16, 16, CHECK>(g, P, st);
-    case 14: return launch_gather_s2<GT, 4, 4, 16, 12, CHECK>(g, P, st);
-    case 15: return launch_gather_s2<GT, 4, 4, 16, 8, CHECK>(g, P, st);
-    case 16: return launch_gather_s2<GT, 2, 2, 12, 24, CHECK>(g, P, st);
     case 17: return launch_gather_s3<GT, 4, 4, 8, 12, CHECK>(g, P, st);
     case 18: return launch_gather_s3<GT, 4, 4, 8, 16, CHECK>(g, P, st);
     case 19: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK>(g, P, st);
     case 20: return launch_gather_s3<GT, 2, 2, 8, 24, CHECK>(g, P, st);
-    case 21: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 1>(g, P, st);
-    case 22: return launch_gather_s3<GT, 4, 2, 8, 12, CHECK, 1>(g, P, st);
-    case 23: return launch_gather_s4<GT, 4, 4, 12, 16, CHECK>(g, P, st);
-    case 24: return launch_gather_s4<GT, 4, 2, 8, 16, CHECK>(g, P, st);
-    case 25: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK>(g, P, st);
-    case 26: return launch_gather_s3<GT, 4, 2, 4, 16, CHECK>(g, P, st);
-    case 27: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 2>(g, P, st);
-    case 28: return launch_gather_s3<GT, 4, 3, 8, 16, CHECK, 2>(g, P, st);
-    case 29: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, 3>(g, P, st);
-    case 30: return launch_gather_s3<GT, 4, 2, 8, 12, CHECK, 3>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }

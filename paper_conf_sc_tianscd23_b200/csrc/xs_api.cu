@@ -579,7 +579,9 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!g || !name) return fail(XS_ERR_INVALID_ARG, "NULL argument");
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
-    if (value < 0 || value > 30) return fail(XS_ERR_INVALID_ARG, "variant in [0,30]");
+    if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
+          (value >= 17 && value <= 20)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12 or 17-20");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
