@@ -52,13 +52,6 @@ struct Sample {
 };
 
 // lookup id -> (p, mat): s = FF(seed, 2 id); p = draw; roll = draw (R4)
-__device__ __forceinline__ Sample sample_from_state(uint64_t s) {
-  s = lcg_next(s);
-  const double p = lcg_double(s);
-  s = lcg_next(s);
-  return Sample{p, pick_material(lcg_double(s))};
-}
-
 __device__ __forceinline__ Sample sample_lookup(uint64_t seed, uint64_t id) {
   uint64_t s = fast_forward(seed, 2 * id);
   s = lcg_next(s);
@@ -93,6 +86,7 @@ struct Params {
   // workspace
   uint32_t* counts;
   uint32_t* cursor;
+  uint32_t* task_next;  // dynamic task counter of the staged gather (zeroed per call)
   LookupRec* recs;
   uint32_t* bins;   // [(n_mats + 1) * kEnergyBins] histogram -> cursors (A2)
   LookupRec* tmp;   // [count] records in batch order
@@ -188,7 +182,7 @@ __device__ __forceinline__ int32_t union_upper_tab(const Params& P, double p) {
 }
 
 // k_sample: A1 + A3 in batch order.  Thread t of a block handles lookups
-// c0 + it*256 + t, it < kPrepItems; their unionized searches run in
+// c0 + kPrepItems*t + it, it < kPrepItems; their unionized searches run in
 // lockstep (kPrepItems independent probes in flight per thread).  Writes
 // the 16-B record tmp[i] = {p, i, u|b}, the material mat8[i] and the
 // histogram: per material (plain) or per (material, energy bin) (A2).
@@ -211,18 +205,27 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
     Sample smp[kPrepItems];
     bool ok[kPrepItems];
     int64_t lo[kPrepItems], hi[kPrepItems];
+    // thread t owns the kPrepItems consecutive lookups c0 + kPrepItems*t + it:
+    // one jump to the first, then two LCG steps per lookup (R4: lookup i+1's
+    // stream starts where lookup i's two draws end)
+    uint64_t st = 0;
+    if (!P.in_energy) st = fast_forward(s_state, 2ull * kPrepItems * threadIdx.x);
 #pragma unroll
     for (int it = 0; it < kPrepItems; ++it) {
-      const uint64_t k = static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
+      const uint64_t k = static_cast<uint64_t>(kPrepItems) * threadIdx.x + it;
       const uint64_t i = c0 + k;
       ok[it] = i < P.count;
-      if (P.in_energy)
+      if (P.in_energy) {
         smp[it] = ok[it] ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
-      else
-        smp[it] = sample_from_state(fast_forward(s_state, 2 * k));
+      } else {
+        st = lcg_next(st);
+        const double pe = lcg_double(st);
+        st = lcg_next(st);
+        smp[it] = Sample{pe, pick_material(lcg_double(st))};
+      }
       lo[it] = 0;
       hi[it] = P.NU - 1;
-      if (GT == XS_GRID_UNIONIZED) {
+      if (GT == XS_GRID_UNIONIZED && P.need_gidx) {
         // A3 search range from the equal-width table: u in [UB[b]-1, UB[b+1]]
         const double q = smp[it].p * static_cast<double>(P.UBn);
         const int32_t b = q > 0.0 ? (q < static_cast<double>(P.UBn) ? static_cast<int32_t>(q)
@@ -268,8 +271,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
 #pragma unroll
     for (int it = 0; it < kPrepItems; ++it) {
       if (!ok[it]) continue;
-      const uint32_t i = static_cast<uint32_t>(c0 + static_cast<uint64_t>(it) * kPrepThreads +
-                                               threadIdx.x);
+      const uint32_t i = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPrepItems) * threadIdx.x +
+                                               it);
       const int32_t m = smp[it].mat;
       const double p = smp[it].p;
       const bool valid = m < P.n_mats;
@@ -1358,7 +1361,7 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
   for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK>
+template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   constexpr int kTask = 32 * R;
   constexpr int S = 2 * D;               // window slots per warp
@@ -1416,7 +1419,11 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 
   unsigned long long acc_v = 0, acc_n = 0;
   int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+  // tasks: the first by warp index, later ones from a global counter (fuel
+  // tasks, ~25x the work of the others, come first), fetched one task ahead
+  uint32_t next = 0;
+  if (DYN && lane == 0) next = nwarps + atomicAdd(P.task_next, 1u);
+  for (uint32_t task = gw; task < total_tasks;) {
     while (task >= G.toff[m + 1]) ++m;
     const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
     double p[R];
@@ -1559,6 +1566,12 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 #pragma unroll
         for (int c = 0; c < 5; ++c) o[c] = M[r][c];
       }
+    }
+    if (DYN) {
+      task = __shfl_sync(0xffffffffu, next, 0);
+      if (lane == 0 && task < total_tasks) next = nwarps + atomicAdd(P.task_next, 1u);
+    } else {
+      task += nwarps;
     }
   }
 #pragma unroll
@@ -1793,14 +1806,14 @@ static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK>
+template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false>
 static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * kIvDoubles * 8;
   const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
   const size_t smem = sizeof(GatherSmem) +
                       static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
                       NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
-  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK>;
+  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK, DYN>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -1836,6 +1849,9 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 18: return launch_gather_s3<GT, 4, 4, 8, 16, CHECK>(g, P, st);
     case 19: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK>(g, P, st);
     case 20: return launch_gather_s3<GT, 2, 2, 8, 24, CHECK>(g, P, st);
+    case 21: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, true>(g, P, st);
+    case 22: return launch_gather_s3<GT, 4, 1, 8, 16, CHECK, true>(g, P, st);
+    case 23: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK, true>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
@@ -1864,6 +1880,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.in_mat = a.in_mat;
   P.counts = ws.counts;
   P.cursor = ws.cursor;
+  P.task_next = ws.cursor + (kMaxMats + 1);
   P.recs = ws.recs;
   P.out_M = a.out.macro_xs;
   P.out_E = a.out.energy;
@@ -1887,7 +1904,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     mark(3);
     return cudaGetLastError();
   }
-  e = cudaMemsetAsync(ws.counts, 0, 2 * (kMaxMats + 1) * sizeof(uint32_t), st);
+  e = cudaMemsetAsync(ws.counts, 0, (2 * (kMaxMats + 1) + 1) * sizeof(uint32_t), st);
   if (e != cudaSuccess) return e;
   const bool binned = a.flags & XS_FLAG_SORT;
   const unsigned nb = grid_cap(a.count, kPrepThreads * kPrepItems, g.sm_count, 16);

@@ -79,7 +79,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
     off += align256(bytes);
     return o;
   };
-  const size_t o_counts = take(2 * (kMaxMats + 1) * sizeof(uint32_t));
+  const size_t o_counts = take((2 * (kMaxMats + 1) + 1) * sizeof(uint32_t));
   const size_t o_recs = take(count * sizeof(LookupRec));
   const size_t o_tmp = take(count * sizeof(LookupRec));
   const size_t o_mat8 = take(count);
@@ -580,8 +580,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
-          (value >= 17 && value <= 20)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12 or 17-20");
+          (value >= 17 && value <= 23)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12 or 17-23");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");

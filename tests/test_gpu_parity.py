@@ -71,7 +71,7 @@ def _compare(out, ref, mode_index=True):
 @pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
                                      "sort-v1", "sort-v3", "sort-v4", "sort-v9", "sort-v10",
                                      "sort-v11", "sort-v12", "sort-v17", "sort-v18", "sort-v19",
-                                     "sort-v20"])
+                                     "sort-v20", "sort-v21", "sort-v22", "sort-v23"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -101,7 +101,7 @@ def test_tiny_other_grids(X, grid_type, bins, sort):
 
 
 @pytest.mark.parametrize("grid_type,bins", [("hash", 97), ("hash", 8192), ("nuclide", 0)])
-@pytest.mark.parametrize("variant", [9, 17, 19, 20])
+@pytest.mark.parametrize("variant", [9, 17, 19, 20, 21])
 def test_tiny_other_grids_staged(X, grid_type, bins, variant):
     """The TMA-staged sorted gathers on the hash and nuclide grids."""
     g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
