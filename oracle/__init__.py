@@ -26,6 +26,7 @@ _SOURCES = [os.path.join(_HERE, "xs_oracle.c"), os.path.join(_HERE, "xs_oracle.h
             os.path.join(_ROOT, "gen", "xs_gen.cpp"), os.path.join(_ROOT, "gen", "xs_gen.h")]
 
 UNIONIZED, NUCLIDE, HASH = 0, 1, 2
+F32 = 0x10   # OR into a mode: the fp32 variant (R18)
 _lock = threading.Lock()
 _lib = None
 
@@ -88,6 +89,8 @@ def lib() -> C.CDLL:
                 "oracle_micro_xs": (None, [P, i32, i64, d, P]),
                 "oracle_macro_xs": (None, [P, d, i32, C.c_int, P, P]),
                 "oracle_verify": (C.c_int, [P]),
+                "oracle_micro_xs_f32": (None, [P, i32, i64, d, P]),
+                "oracle_macro_xs_f32": (None, [P, d, i32, C.c_int, P, P]),
                 "oracle_lookup": (None, [P, u64, C.c_int, P, P, P, P, P]),
                 "oracle_run": (u64, [P, u64, u64, C.c_int, C.c_int, P, P, P, P, P]),
                 "oracle_run_explicit": (u64, [P, P, P, u64, C.c_int, C.c_int, P, P]),
@@ -267,10 +270,19 @@ class Oracle:
         lib().oracle_micro_xs(self._h, n, k, p, _ptr(xs))
         return xs
 
+    def micro_xs_f32(self, n: int, k: int, p: float) -> np.ndarray:
+        xs = np.zeros(5, np.float32)
+        lib().oracle_micro_xs_f32(self._h, n, k, p, _ptr(xs))
+        return xs
+
     def macro_xs(self, p: float, mat: int, mode: int = UNIONIZED):
+        """mode may include F32 (the fp32 variant; M is the binary32 result widened)."""
         M = np.zeros(5, np.float64)
         gi = C.c_int64(0)
-        lib().oracle_macro_xs(self._h, p, mat, mode, _ptr(M), C.byref(gi))
+        if mode & F32:
+            lib().oracle_macro_xs_f32(self._h, p, mat, mode & 0xF, _ptr(M), C.byref(gi))
+        else:
+            lib().oracle_macro_xs(self._h, p, mat, mode, _ptr(M), C.byref(gi))
         return M, gi.value
 
     def lookup(self, i: int, mode: int = UNIONIZED):

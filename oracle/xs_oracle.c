@@ -397,6 +397,54 @@ void oracle_macro_xs(const oracle_ctx* c, double p, int32_t mat, int mode, doubl
   if (grid_index) *grid_index = idx;
 }
 
+/* R18 (fp32 variant, north_star "1e-5 if an fp32 variant is offered";
+ * SURVEY §8(f) NEXT-2): energies stay binary64, so the search and every
+ * bracket are those of R5-R9; f is the binary64 quotient of R10, rounded once
+ * to binary32; the channel values and concentrations are the binary64 data
+ * rounded once to binary32; then, each a separate IEEE binary32 operation:
+ *   d = hi.c - lo.c;  t = f * d;  x = hi.c - t;  w = x * conc;  M_c = M_c + w,
+ * M starting at +0.0f, nuclides in list order.                           */
+void oracle_micro_xs_f32(const oracle_ctx* c, int32_t n, int64_t k, double p, float xs[5]) {
+  const double* lo = c->grid + ((int64_t)n * c->N + k) * 6;
+  const double* hi = lo + 6;
+  double f64 = (hi[0] - p) / (hi[0] - lo[0]);
+  float f = (float)f64;
+  for (int ch = 0; ch < 5; ch++) {
+    float h = (float)hi[1 + ch];
+    float l = (float)lo[1 + ch];
+    float d = h - l;
+    float t = f * d;
+    xs[ch] = h - t;
+  }
+}
+
+void oracle_macro_xs_f32(const oracle_ctx* c, double p, int32_t mat, int mode, double M[5],
+                         int64_t* grid_index) {
+  int64_t idx = -1;
+  float Mf[5] = {0.0f, 0.0f, 0.0f, 0.0f, 0.0f};
+  if (mode == ORACLE_UNIONIZED) idx = oracle_union_index(c, p);
+  if (mode == ORACLE_HASH) idx = oracle_hash_bin(c, p);
+  for (int32_t j = 0; j < c->num_nucs[mat]; j++) {
+    int32_t n = c->mats[mat * c->max_nucs + j];
+    float conc = (float)c->concs[mat * c->max_nucs + j];
+    int64_t k;
+    if (mode == ORACLE_UNIONIZED)
+      k = oracle_index_grid_entry(c, idx, n);
+    else if (mode == ORACLE_HASH)
+      k = oracle_hash_bracket(c, idx, n, p);
+    else
+      k = oracle_nuclide_bracket(c, n, p);
+    float xs[5];
+    oracle_micro_xs_f32(c, n, k, p, xs);
+    for (int ch = 0; ch < 5; ch++) {
+      float w = xs[ch] * conc;
+      Mf[ch] = Mf[ch] + w;
+    }
+  }
+  for (int ch = 0; ch < 5; ch++) M[ch] = (double)Mf[ch]; /* exact widening */
+  if (grid_index) *grid_index = idx;
+}
+
 /* R12: v = 1 + argmax_c M_c with max initialised to -1.0, strict '>', so the
  * first of equal maxima wins and all M_c <= -1 gives v = 1.             */
 int oracle_verify(const double M[5]) {
@@ -417,7 +465,10 @@ void oracle_lookup(const oracle_ctx* c, uint64_t id, int mode, double* p, int32_
   int32_t m;
   double Ml[5];
   oracle_sample(c->lookup_seed, id, &pe, &m);
-  oracle_macro_xs(c, pe, m, mode, Ml, grid_index);
+  if (mode & ORACLE_F32)
+    oracle_macro_xs_f32(c, pe, m, mode & 0xF, Ml, grid_index);
+  else
+    oracle_macro_xs(c, pe, m, mode, Ml, grid_index);
   if (p) *p = pe;
   if (mat) *mat = m;
   if (M) memcpy(M, Ml, sizeof(Ml));
@@ -442,6 +493,8 @@ typedef struct {
 static void* run_range(void* va) {
   run_arg* a = (run_arg*)va;
   uint64_t s = 0;
+  const int grid_mode = a->mode & 0xF;
+  const int f32 = (a->mode & ORACLE_F32) != 0;
   for (uint64_t i = a->begin; i < a->end; i++) {
     double pe, Ml[5];
     int32_t m;
@@ -449,11 +502,13 @@ static void* run_range(void* va) {
     if (a->in_p) {
       pe = a->in_p[i];
       m = a->in_mat[i];
-      oracle_macro_xs(a->c, pe, m, a->mode, Ml, &gi);
     } else {
       oracle_sample(a->c->lookup_seed, a->first + i, &pe, &m);
-      oracle_macro_xs(a->c, pe, m, a->mode, Ml, &gi);
     }
+    if (f32)
+      oracle_macro_xs_f32(a->c, pe, m, grid_mode, Ml, &gi);
+    else
+      oracle_macro_xs(a->c, pe, m, grid_mode, Ml, &gi);
     int vv = oracle_verify(Ml);
     s += (uint64_t)vv;
     if (a->p) a->p[i] = pe;

@@ -6,7 +6,8 @@
  * never links or imports it and shares no code with it; the only shared
  * module is the seeded input generator gen/xs_gen.h.
  *
- * Plain, serial-per-lookup, fp64, compiled with -O2 -ffp-contract=off (no
+ * Plain, serial-per-lookup, fp64 (plus the fp32 variant of R18, selected
+ * by ORACLE_F32), compiled with -O2 -ffp-contract=off (no
  * FMA contraction, no fast-math), one function per step of the method, each
  * citing the passage it follows.  PAPER.md states only what is computed
  * ("continuous energy macroscopic neutron cross-section lookup",
@@ -26,6 +27,8 @@ extern "C" {
 #endif
 
 enum { ORACLE_UNIONIZED = 0, ORACLE_NUCLIDE = 1, ORACLE_HASH = 2 };
+/* OR'ed into `mode` of oracle_lookup / oracle_run*: the fp32 variant (R18) */
+enum { ORACLE_F32 = 0x10 };
 
 typedef struct oracle_ctx oracle_ctx;
 
@@ -86,6 +89,11 @@ void oracle_micro_xs(const oracle_ctx* c, int32_t n, int64_t k, double p, double
 void oracle_macro_xs(const oracle_ctx* c, double p, int32_t mat, int mode, double M[5],
                      int64_t* grid_index);
 int  oracle_verify(const double M[5]);
+/* R18: the fp32 variant (binary64 search and f, binary32 channels,
+ * concentrations and accumulation); M is the binary32 result widened. */
+void oracle_micro_xs_f32(const oracle_ctx* c, int32_t n, int64_t k, double p, float xs[5]);
+void oracle_macro_xs_f32(const oracle_ctx* c, double p, int32_t mat, int mode, double M[5],
+                         int64_t* grid_index);
 
 /* One lookup id end to end; any output pointer may be NULL. */
 void oracle_lookup(const oracle_ctx* c, uint64_t id, int mode, double* p, int32_t* mat,

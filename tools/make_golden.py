@@ -42,6 +42,8 @@ def main():
     ap.add_argument("--configs", default="tiny,small,large,large-hash,xl")
     ap.add_argument("--threads", type=int, default=os.cpu_count())
     ap.add_argument("--out", default=os.path.join(ROOT, "tests", "golden", "oracle_hashes.json"))
+    ap.add_argument("--f32-only", action="store_true",
+                    help="only add the fp32-variant sums (R18) to existing entries")
     a = ap.parse_args()
     out = {}
     if os.path.exists(a.out):
@@ -54,14 +56,25 @@ def main():
                                     material_rule=c["rule"], lookup_seed=1070,
                                     hash_bins=c["bins"], nthreads=a.threads)
         t1 = time.time()
+        if a.f32_only:
+            S32 = o.run(0, c["L"], mode=oracle.HASH | oracle.F32, nthreads=a.threads)
+            out[name]["sum_v_f32"] = int(S32)
+            out[name]["hash_f32"] = int(oracle.hash_finalize(S32))
+            print(name, "f32", S32, flush=True)
+            del o
+            with open(a.out, "w") as f:
+                json.dump(out, f, indent=1, sort_keys=True)
+            continue
         S = o.run(0, c["L"], mode=oracle.HASH, nthreads=a.threads)
         t2 = time.time()
+        S32 = o.run(0, c["L"], mode=oracle.HASH | oracle.F32, nthreads=a.threads)
         # P11 regression fingerprints of the generated inputs (first 1 MiB of
         # the grid + the whole material tables)
         g = o.grid()
         entry = dict(n_isotopes=c["I"], n_gridpoints=c["N"], material_rule=c["rule"],
                      lookups=c["L"], grid_seed=42, conc_seed=CONC_SEED, lookup_seed=1070,
                      sum_v=int(S), hash=int(oracle.hash_finalize(S)),
+                     sum_v_f32=int(S32), hash_f32=int(oracle.hash_finalize(S32)),
                      oracle_route=f"hash, {c['bins']} bins (P9: route-independent)",
                      fnv_grid_head=fnv1a(g.ravel()[:131072].tobytes()),
                      fnv_mats=fnv1a(o.mats().tobytes()), fnv_concs=fnv1a(o.concs().tobytes()),
