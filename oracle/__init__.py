@@ -42,7 +42,8 @@ def build(force: bool = False) -> str:
     flags = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC"]
     subprocess.check_call(["gcc", *flags, "-std=c11", "-c", _SOURCES[0], "-o", tmp_o])
     subprocess.check_call(["g++", *flags, "-std=c++17", "-c", _SOURCES[2], "-o", tmp_g])
-    subprocess.check_call(["g++", "-shared", "-o", LIB_PATH + ".tmp", tmp_o, tmp_g, "-lpthread"])
+    subprocess.check_call(["g++", "-shared", "-o", LIB_PATH + ".tmp", tmp_o, tmp_g, "-lpthread",
+                           "-lm"])
     os.replace(LIB_PATH + ".tmp", LIB_PATH)
     for f in (tmp_o, tmp_g):
         os.remove(f)

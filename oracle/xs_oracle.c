@@ -401,8 +401,9 @@ void oracle_macro_xs(const oracle_ctx* c, double p, int32_t mat, int mode, doubl
  * SURVEY §8(f) NEXT-2): energies stay binary64, so the search and every
  * bracket are those of R5-R9; f is the binary64 quotient of R10, rounded once
  * to binary32; the channel values and concentrations are the binary64 data
- * rounded once to binary32; then, each a separate IEEE binary32 operation:
- *   d = hi.c - lo.c;  t = f * d;  x = hi.c - t;  w = x * conc;  M_c = M_c + w,
+ * rounded once to binary32; then, in binary32 with fused multiply-adds
+ * (fmaf: one rounding each):
+ *   d = hi.c - lo.c;  x = fmaf(-f, d, hi.c);  M_c = fmaf(x, conc, M_c),
  * M starting at +0.0f, nuclides in list order.                           */
 void oracle_micro_xs_f32(const oracle_ctx* c, int32_t n, int64_t k, double p, float xs[5]) {
   const double* lo = c->grid + ((int64_t)n * c->N + k) * 6;
@@ -413,8 +414,7 @@ void oracle_micro_xs_f32(const oracle_ctx* c, int32_t n, int64_t k, double p, fl
     float h = (float)hi[1 + ch];
     float l = (float)lo[1 + ch];
     float d = h - l;
-    float t = f * d;
-    xs[ch] = h - t;
+    xs[ch] = fmaf(-f, d, h);
   }
 }
 
@@ -436,10 +436,7 @@ void oracle_macro_xs_f32(const oracle_ctx* c, double p, int32_t mat, int mode, d
       k = oracle_nuclide_bracket(c, n, p);
     float xs[5];
     oracle_micro_xs_f32(c, n, k, p, xs);
-    for (int ch = 0; ch < 5; ch++) {
-      float w = xs[ch] * conc;
-      Mf[ch] = Mf[ch] + w;
-    }
+    for (int ch = 0; ch < 5; ch++) Mf[ch] = fmaf(xs[ch], conc, Mf[ch]);
   }
   for (int ch = 0; ch < 5; ch++) M[ch] = (double)Mf[ch]; /* exact widening */
   if (grid_index) *grid_index = idx;

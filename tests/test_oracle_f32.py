@@ -2,7 +2,8 @@
 fp32 variant is offered").
 
 R18 keeps the binary64 search and interpolation weight and runs the channel
-arithmetic, the concentrations and the accumulation in binary32.  Pins that
+arithmetic, the concentrations and the accumulation in binary32 with fused
+multiply-adds (x = fma(-f, d, hi), M = fma(x, conc, M)).  Pins that
 do not re-type the formula:
   * the hand-worked two-nuclide example (dyadic with few
     significant bits, so every value is exact in binary32 as well): the fp32
