@@ -44,6 +44,9 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     ap.add_argument("--no-sort", action="store_true", help="skip A2 (material/energy binning)")
+    ap.add_argument("--f32", action="store_true",
+                    help="the fp32 variant (XS_FLAG_F32, DESIGN.md R18; hash vs the oracle's "
+                         "fp32 golden sum)")
     ap.add_argument("--lookups", type=int, default=0, help="override lookups per GPU (weak)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -125,6 +128,7 @@ def measured_peaks():
 GATHER_KERNEL = {True: "k_gather_s3 (A4-A8, TMA-staged interval-table windows)",
                  False: "k_gather (A4-A8, 3 lanes per lookup)"}
 FP64_OPS_PER_LOOKUP_NUCLIDE = 24
+FP64_OPS_F32_VARIANT = 5
 FP64_LANES_PER_SM = 64   # B200: 37 TFLOP/s FP64 (FMA = 2) = 148 SMs x 64 lanes x 2 x 1.965 GHz
 
 
@@ -173,12 +177,12 @@ def cpu_info():
     return name
 
 
-def oracle_sample_rate(pre, target_s: float, first: int = 0):
+def oracle_sample_rate(pre, target_s: float, first: int = 0, f32: bool = False):
     """Time the CPU oracle (as it stands) on a bounded sample of the workload
     on all host cores.  Returns (lookups/s, cores, description, sum_v)."""
     import oracle
     cores = os.cpu_count() or 1
-    mode = ORACLE_MODE[pre["grid_type"]]
+    mode = ORACLE_MODE[pre["grid_type"]] | (oracle.F32 if f32 else 0)
     o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"], conc_seed=1070 * 1070,
                                 material_rule=pre["material_rule"],
                                 hash_bins=pre.get("hash_bins", 0), nthreads=cores)
@@ -205,10 +209,10 @@ def run_reference(a, pre, cfg):
     # size each step to a bounded sample so the whole run takes a few minutes
     budget = 150.0
     per_step = max(1.0, min(a.cpu_seconds, budget / max(1, a.steps + a.warmup)))
-    rate0, cores, _, _, _ = oracle_sample_rate(pre, per_step / 4)
+    rate0, cores, _, _, _ = oracle_sample_rate(pre, per_step / 4, f32=a.f32)
     n = int(min(pre["lookups"], max(10_000, rate0 * per_step)))
     import oracle
-    mode = ORACLE_MODE[pre["grid_type"]]
+    mode = ORACLE_MODE[pre["grid_type"]] | (oracle.F32 if a.f32 else 0)
     o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"], conc_seed=1070 * 1070,
                                 material_rule=pre["material_rule"],
                                 hash_bins=pre.get("hash_bins", 0), nthreads=cores)
@@ -225,7 +229,8 @@ def run_reference(a, pre, cfg):
     line = {"impl": "reference", "metric": "XS lookups/sec", "value": value,
             "unit": "lookups/s", "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
             "ms_per_step": 1e3 * tot / a.steps, "higher_is_better": True,
-            "scaling": a.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "scaling": a.scaling, "vs_baseline": None, "dtype": "f32" if a.f32 else "f64",
+            "data": "synthetic",
             "config": cfg,
             "cpu_baseline": {"value": value, "unit": "lookups/s", "cores": cores,
                              "kind": "oracle",
@@ -269,7 +274,8 @@ def run_ours(a, pre, cfg):
 
     # untimed: per-material counts of this shard (exact algorithmic bytes)
     # and the inputs of the end-to-end leg
-    vs0, res0 = g.lookup(first, L, sort=sort, want=("mat", "energy"))
+    f32 = a.f32
+    vs0, res0 = g.lookup(first, L, sort=sort, want=("mat", "energy"), f32=f32)
     torch.cuda.synchronize()
     mats = torch.bincount(res0["mat"].long(), minlength=g.info.n_mats).cpu().tolist()
     num_nucs = g.table(X.XS_TABLE_NUM_NUCS).tolist()
@@ -282,13 +288,14 @@ def run_ours(a, pre, cfg):
     gold = golden().get(a.config)
     hash_check = None
     if gold and first == 0 and L == gold["lookups"]:
-        hash_check = int(vs0[0]) == gold["sum_v"] and int(vs0[1]) == L
+        hash_check = (int(vs0[0]) == gold["sum_v_f32" if f32 else "sum_v"] and
+                      int(vs0[1]) == L)
 
     vsum = torch.zeros(2, dtype=torch.int64, device=dev)
 
     def step():
         vsum.zero_()
-        g.lookup(first, L, sort=sort, vsum=vsum)
+        g.lookup(first, L, sort=sort, vsum=vsum, f32=f32)
         if world > 1:
             if a.backend == "nccl":
                 D.combine_vsum(vsum)      # A9 over NCCL (NVLink / NVSwitch)
@@ -340,18 +347,21 @@ def run_ours(a, pre, cfg):
         # energy-sorted batches re-read each record pair from shared memory for
         # ~40 lookups: the staged gather is bound by the FP64 pipe
         fp64_peak, fp64_src = fp64_pipe_peak()
-        ops = nuc_lookups * FP64_OPS_PER_LOOKUP_NUCLIDE
+        per = FP64_OPS_F32_VARIANT if f32 else FP64_OPS_PER_LOOKUP_NUCLIDE
+        ops = nuc_lookups * per
         fp64_achieved = ops / (gather_ms / 1e3) / 1e12
         roofline = {"bound": "alu", "kernel": GATHER_KERNEL[sort], "achieved": fp64_achieved,
                     "peak": fp64_peak, "unit": "TFLOP/s", "frac": fp64_achieved / fp64_peak,
                     "traffic": roofline_hbm["traffic"], "peak_source": fp64_src,
                     "algorithmic_fp64_ops_per_launch": ops,
                     "gather_ms_per_launch": gather_ms, "traffic_source": traffic_src,
-                    "note": "FP64 pipe operations (DADD/DMUL/DFMA count one each): "
-                            f"{FP64_OPS_PER_LOOKUP_NUCLIDE} per (lookup, nuclide) = f (1 sub "
-                            "+ 3 for the correctly rounded division by a precomputed "
-                            "reciprocal) + 5 channels x (mul, sub, mul, add); traffic = DRAM "
-                            "bytes per launch from ncu"}
+                    "note": ("FP64 pipe operations (DADD/DMUL/DFMA count one each): "
+                             f"{per} per (lookup, nuclide) = f (1 sub + 3 for the correctly "
+                             "rounded division by a precomputed reciprocal) + " +
+                             ("1 conversion to binary32; the channels run as binary32 "
+                              "FFMA2 (2 per channel pair of lookups)" if f32 else
+                              "5 channels x (mul, sub, mul, add)") +
+                             "; traffic = DRAM bytes per launch from ncu")}
     else:
         roofline = roofline_hbm
     step_frac = balg_per_lookup * (value / world) / 8e12
@@ -359,7 +369,7 @@ def run_ours(a, pre, cfg):
     line = {"metric": "XS lookups/sec", "value": value, "unit": "lookups/s", "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps,
             "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None,
-            "dtype": "f64", "data": "synthetic", "config": cfg,
+            "dtype": "f32" if f32 else "f64", "data": "synthetic", "config": cfg,
             "roofline": roofline,
             "roofline_hbm": roofline_hbm,
             "hbm_gather_roofline_frac_8TBs": step_frac,
@@ -375,13 +385,13 @@ def run_ours(a, pre, cfg):
         e_host = res0["energy"].cpu().pin_memory()
         m_host = res0["mat"].cpu().pin_memory()
         vs_h = torch.zeros(2, dtype=torch.int64).pin_memory()
-        g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)      # warm-up
+        g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h, f32=f32)  # warm-up
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
         for _ in range(a.e2e_steps):
             vs_h.zero_()
-            g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)  # H2D, lookup, D2H
+            g.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h, f32=f32)  # H2D, lookup, D2H
         dt = time.perf_counter() - t0
         dt = D.max_over_ranks(dt, device=dev if a.backend == "nccl" else None)
         e2e_total = L * world * a.e2e_steps if a.scaling == "weak" else L_cfg * a.e2e_steps
@@ -394,7 +404,7 @@ def run_ours(a, pre, cfg):
     line["clocks"] = clk.summary()
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         try:
-            rate, cores, desc, S, n = oracle_sample_rate(pre, a.cpu_seconds)
+            rate, cores, desc, S, n = oracle_sample_rate(pre, a.cpu_seconds, f32=f32)
             line["cpu_baseline"] = {"value": rate, "unit": "lookups/s", "cores": cores,
                                     "kind": "oracle", "sample": desc, "cpu": cpu_info()}
         except Exception as e:  # the oracle is test infrastructure; report, don't fail
@@ -419,6 +429,8 @@ def main():
            else None, "lookups_total": per_gpu if a.scaling == "strong" else per_gpu * a.gpus,
            "sort": ("A2 material+energy binning (2^18 energy bins per material)"
                     if not a.no_sort else "none"),
+           "precision": ("fp32 variant (R18: binary64 search and weight, binary32 channels "
+                         "and accumulation)" if a.f32 else "binary64 (R10, R11)"),
            "l2": "not flushed: the resident tables (GBs, see grid_device_bytes) far exceed "
                  "the 126 MB L2",
            "parallelism": f"dp{a.gpus} (lookup shards, grid replicated)"}

@@ -148,6 +148,13 @@ typedef struct {
 #define XS_FLAG_HOST_IO 0x2u  /* inputs/outputs are host pointers               */
 #define XS_FLAG_BASELINE 0x4u /* thread-per-lookup, unbucketed kernel (XSBench's
                                  CUDA baseline shape; for comparison only)     */
+#define XS_FLAG_F32 0x8u      /* the fp32 variant (R18; north_star "1e-5
+                                 if an fp32 variant is offered"): energies, the
+                                 search and f stay binary64; channel values,
+                                 concentrations and the accumulation are
+                                 binary32 with fused multiply-adds.  macro_xs
+                                 receives the binary32 results widened.  Not
+                                 combinable with XS_FLAG_BASELINE.             */
 
 /* tables for xs_get_table (element type in brackets) */
 #define XS_TABLE_NUCLIDE_GRID 0 /* [double] I*N*6                               */

@@ -5,6 +5,7 @@
 //   K0b  IG[e][n] = clamp(ub(E_n, U[e]) - 1, 0, N-2)   (chunked search + sweep)
 //   K0c  HG[b][n] = clamp(ub(E_n, b du) - 1, 0, N-2)   (one search per entry)
 //   K0d  IV[n][k]  = interval terms of record pair (k, k+1) (see below)
+//   K0e  IV32[n][k] = the same for the fp32 variant (R18)
 // Definitions: DESIGN.md R6, R7 (north_star: "the unionized (or
 // hash-accelerated) energy grid").
 #include "common.cuh"
@@ -215,6 +216,44 @@ __global__ void k_build_intervals(const double* __restrict__ grid, uint64_t tota
       o[5 + 2 * c] = dsub(hi[1 + c], lo[1 + c]);
     }
   }
+}
+
+// K0e: fp32-variant interval table (R18), 80-B entries:
+// {E[k+1], gap} {recip(gap), 0} then float4 {h0, d0, h1, d1} {h2, d2, h3, d3}
+// {h4, d4, 0, 0} with h = (float) hi.c and d = h - (float) lo.c (binary32).
+__global__ void k_build_intervals32(const double* __restrict__ grid, uint64_t total, int64_t N,
+                                    double* __restrict__ IV) {
+  for (uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; t < total;
+       t += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    double* o = IV + t * kIv32Doubles;
+    float* of = reinterpret_cast<float*>(o + 4);
+    if (static_cast<int64_t>(t % static_cast<uint64_t>(N)) == N - 1) {
+      for (int q = 0; q < kIv32Doubles; ++q) o[q] = 0.0;
+      continue;
+    }
+    const double* lo = grid + t * 6;
+    const double* hi = lo + 6;
+    const double bd = dsub(hi[0], lo[0]);
+    o[0] = hi[0];
+    o[1] = bd;
+    o[2] = recip_nr(bd);
+    o[3] = 0.0;
+    for (int c = 0; c < 5; ++c) {
+      const float h = __double2float_rn(hi[1 + c]);
+      const float l = __double2float_rn(lo[1 + c]);
+      of[2 * c] = h;
+      of[2 * c + 1] = __fsub_rn(h, l);
+    }
+    of[10] = 0.0f;
+    of[11] = 0.0f;
+  }
+}
+
+cudaError_t build_intervals32(const DeviceGrid& g, cudaStream_t st) {
+  const uint64_t total = static_cast<uint64_t>(g.I) * g.N;
+  k_build_intervals32<<<grid_for(total, 256, g.sm_count), 256, 0, st>>>(g.grid, total, g.N,
+                                                                        g.iv32);
+  return cudaGetLastError();
 }
 
 cudaError_t build_intervals(const DeviceGrid& g, cudaStream_t st) {

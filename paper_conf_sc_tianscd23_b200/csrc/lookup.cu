@@ -64,6 +64,7 @@ struct Params {
   // grid
   const double* grid;
   const double* iv;         // interval table [I][N][kIvDoubles] (K0d)
+  const double* iv32;       // fp32-variant interval table [I][N][kIv32Doubles] (K0e)
   int32_t I;
   int64_t N;
   const double* U;
@@ -1318,13 +1319,101 @@ __device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R]
   }
 }
 
+// fp32 variant (R18): paired binary32 fused multiply-add (sm_100a FFMA2),
+// one rounding per element.  Plain mul/add pairs are avoided on purpose:
+// ptxas contracts f32x2 mul + add into FFMA2 even with .rn.
+__device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
+  uint64_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;"
+      : "=l"(d)
+      : "l"(*reinterpret_cast<uint64_t*>(&a)), "l"(*reinterpret_cast<uint64_t*>(&b)),
+        "l"(*reinterpret_cast<uint64_t*>(&c)));
+  return *reinterpret_cast<float2*>(&d);
+}
+
+// Accumulators of the staged gather: M for R lookups and the A6 + A7 update
+// from one interval-table entry q for lookups r in [r0, r1).
+template <int R, bool CHECK>
+struct AccF64 {  // binary64 (R10, R11): entry = K0d, 7 x 16 B
+  static constexpr int kE = kIvDoubles / 2;
+  double M[R][5];
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+  }
+  __device__ __forceinline__ double get(int r, int c) const { return M[r][c]; }
+  template <bool SHARED>
+  __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
+                                         int r1) {
+    iv_interp<R, CHECK, SHARED>(q, p, conc, M, r0, r1);
+  }
+};
+
+template <int R, bool CHECK>
+struct AccF32 {  // binary32 variant (R18): entry = K0e, 5 x 16 B
+  static_assert(R % 2 == 0, "fp32 accumulators pair lookups");
+  static constexpr int kE = kIv32Doubles / 2;
+  float2 M[R / 2][5];  // {lookup 2q, lookup 2q+1}
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int q = 0; q < R / 2; ++q)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) M[q][c] = make_float2(0.0f, 0.0f);
+  }
+  __device__ __forceinline__ double get(int r, int c) const {
+    return static_cast<double>((r & 1) ? M[r >> 1][c].y : M[r >> 1][c].x);
+  }
+  template <bool SHARED>
+  __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
+                                         int r1) {
+    auto ld = [&](int u) -> double2 { return SHARED ? q[u] : __ldg(q + u); };
+    auto ldf = [&](int u) -> float4 {
+      const float4* f4 = reinterpret_cast<const float4*>(q + u);
+      return SHARED ? *f4 : __ldg(f4);
+    };
+    const double2 a0 = ld(0), a1 = ld(1);
+    float nf[R];  // -f, f = binary64 weight rounded once to binary32
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (r < r0 || r >= r1) continue;
+      const double an = dsub(a0.x, p[r]);
+      double f = div_by_recip(an, a0.y, a1.x);
+      if (CHECK && !div_in_range(an, a0.y)) f = ddiv(an, a0.y);
+      nf[r] = -__double2float_rn(f);
+    }
+    const float cf = __double2float_rn(conc);
+    const float4 t0 = ldf(2), t1 = ldf(3), t2 = ldf(4);
+    const float hh[5] = {t0.x, t0.z, t1.x, t1.z, t2.x};
+    const float dd[5] = {t0.y, t0.w, t1.y, t1.w, t2.y};
+#pragma unroll
+    for (int c = 0; c < 5; ++c) {
+#pragma unroll
+      for (int qq = 0; qq < R / 2; ++qq) {
+        const int ra = 2 * qq, rb = 2 * qq + 1;
+        const bool ia = ra >= r0 && ra < r1, ib = rb >= r0 && rb < r1;
+        if (ia && ib) {
+          const float2 x = ffma2(make_float2(nf[ra], nf[rb]), make_float2(dd[c], dd[c]),
+                                 make_float2(hh[c], hh[c]));
+          M[qq][c] = ffma2(x, make_float2(cf, cf), M[qq][c]);
+        } else if (ia) {
+          M[qq][c].x = __fmaf_rn(__fmaf_rn(nf[ra], dd[c], hh[c]), cf, M[qq][c].x);
+        } else if (ib) {
+          M[qq][c].y = __fmaf_rn(__fmaf_rn(nf[rb], dd[c], hh[c]), cf, M[qq][c].y);
+        }
+      }
+    }
+  }
+};
+
 // One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
 // i(p) = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p} by binary lifting
 // (warp-uniform trip count; loads clamped so the loop has no branches).
-template <int R, bool CHECK, bool SHARED>
+template <int R, bool SHARED, class Acc>
 __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
-                                                 const double (&p)[R], double (&M)[R][5]) {
-  constexpr int kE = kIvDoubles / 2;
+                                                 const double (&p)[R], Acc& acc) {
+  constexpr int kE = Acc::kE;
   // E[k_lo + t] = first double of entry t - 1
   auto E = [&](int t) -> double {
     const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
@@ -1339,7 +1428,7 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     if (tL <= n_int && eL <= p[R - 1]) iL = tL;
   }
   if (__all_sync(0xffffffffu, i0 == iL)) {
-    iv_interp<R, CHECK, SHARED>(win + i0 * kE, p, conc, M, 0, R);
+    acc.template interp<SHARED>(win + i0 * kE, p, conc, 0, R);
     return;
   }
   int i[R];
@@ -1358,14 +1447,16 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     }
   }
 #pragma unroll
-  for (int r = 0; r < R; ++r) iv_interp<R, CHECK, SHARED>(win + i[r] * kE, p, conc, M, r, r + 1);
+  for (int r = 0; r < R; ++r) acc.template interp<SHARED>(win + i[r] * kE, p, conc, r, r + 1);
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false>
+template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false, bool F32 = false>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
+  using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
   constexpr int kTask = 32 * R;
   constexpr int S = 2 * D;               // window slots per warp
-  constexpr int kEntry = kIvDoubles * 8;  // bytes per interval entry
+  constexpr int kE = Acc::kE;            // 16-B units per interval entry
+  constexpr int kEntry = kE * 16;        // bytes per interval entry
   static_assert(S <= 32, "slots");
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GatherSmem& G = *reinterpret_cast<GatherSmem*>(smem_raw);
@@ -1414,7 +1505,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   const uint32_t total_tasks = G.toff[P.n_mats];
   const uint32_t gw = blockIdx.x * NW + warp;
   const uint32_t nwarps = gridDim.x * NW;
-  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(P.iv);
+  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(F32 ? P.iv32 : P.iv);
   uint32_t phase = 0;  // parity bit per slot
 
   unsigned long long acc_v = 0, acc_n = 0;
@@ -1510,9 +1601,9 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
         const int2 kk = s_k[j];
         const int32_t w = kk.y - kk.x + 1;
         if (w <= W) {
-          const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
+          const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
           mbar_arrive_expect_tx(&s_bar[slot], static_cast<uint32_t>(w) * kEntry);
-          bulk_copy_g2s(s_win + slot * W * (kIvDoubles / 2), src, static_cast<uint32_t>(w) * kEntry,
+          bulk_copy_g2s(s_win + slot * W * kE, src, static_cast<uint32_t>(w) * kEntry,
                         &s_bar[slot]);
         } else {
           mbar_arrive_expect_tx(&s_bar[slot], 0u);  // read in place from global memory
@@ -1522,11 +1613,8 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
     issue_group(0);
     issue_group(1);
 
-    double M[R][5];
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
+    Acc acc;
+    acc.zero();
 
     for (int j = 0; j < nn; ++j) {
       const int slot = j % S;
@@ -1540,10 +1628,10 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
       if (n_int < W) {
-        stage_nuclide_iv<R, CHECK, true>(s_win + slot * W * (kIvDoubles / 2), n_int, conc, p, M);
+        stage_nuclide_iv<R, true>(s_win + slot * W * kE, n_int, conc, p, acc);
       } else {
-        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * (kIvDoubles / 2);
-        stage_nuclide_iv<R, CHECK, false>(g2, n_int, conc, p, M);
+        const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
+        stage_nuclide_iv<R, false>(g2, n_int, conc, p, acc);
       }
     }
     __syncwarp();
@@ -1554,8 +1642,8 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       int vi = 0;
 #pragma unroll
       for (int c = 0; c < 5; ++c)
-        if (M[r][c] > mx) {
-          mx = M[r][c];
+        if (acc.get(r, c) > mx) {
+          mx = acc.get(r, c);
           vi = c;
         }
       acc_v += static_cast<unsigned long long>(vi + 1);
@@ -1564,7 +1652,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       if (P.out_M) {
         double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
 #pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = M[r][c];
+        for (int c = 0; c < 5; ++c) o[c] = acc.get(r, c);
       }
     }
     if (DYN) {
@@ -1710,6 +1798,7 @@ static Params make_params(const DeviceGrid& g) {
   Params P{};
   P.grid = g.grid;
   P.iv = g.iv;
+  P.iv32 = g.iv32;
   P.I = g.I;
   P.N = g.N;
   P.U = g.U;
@@ -1806,14 +1895,14 @@ static cudaError_t launch_gather_s(const DeviceGrid& g, const Params& P, cudaStr
   return cudaGetLastError();
 }
 
-template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false>
+template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false, bool F32 = false>
 static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * kIvDoubles * 8;
+  constexpr size_t win_bytes = static_cast<size_t>(2 * D) * W * (F32 ? kIv32Doubles : kIvDoubles) * 8;
   const size_t k_bytes = ((static_cast<size_t>(g.max_nucs) * 8 + 15) / 16) * 16;
   const size_t smem = sizeof(GatherSmem) +
                       static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry) +
                       NW * (win_bytes + k_bytes + ((2 * D * 8 + 15) / 16) * 16);
-  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK, DYN>;
+  auto kern = k_gather_s3<GT, R, D, W, NW, CHECK, DYN, F32>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return e;
@@ -1856,14 +1945,28 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   }
 }
 
-// Kernel choice: energy-sorted batches use the thread-per-lookup kernel;
-// unsorted batches the 3-lanes-per-lookup kernel, which needs the row
-// layout of the unionized index grid (a column-only grid falls back to the
-// thread-per-lookup kernel).
+// fp32 variant (R18): the staged interval-table gather for every batch
+// (variants 31-33 select its shape; any other value the default).
+template <int GT, bool CHECK>
+static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  switch (g.unroll) {
+    case 32: return launch_gather_s3<GT, 8, 2, 8, 16, CHECK, false, true>(g, P, st);
+    case 33: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, true, true>(g, P, st);
+    default: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, false, true>(g, P, st);
+  }
+}
+
+// Kernel choice: energy-sorted batches use the staged gather (variant
+// table in launch_gather_tv); unsorted batches the 3-lanes-per-lookup
+// kernel, which needs the row layout of the unionized index grid (a
+// column-only grid uses the staged gather); the fp32 variant always runs
+// the staged gather.
 template <int GT>
-static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool sorted,
+static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool sorted, bool f32,
                                    cudaStream_t st) {
   const bool check = P.in_energy != nullptr || !g.dyadic63;
+  if (f32)
+    return check ? launch_gather_f32<GT, true>(g, P, st) : launch_gather_f32<GT, false>(g, P, st);
   const bool thread_kernel = sorted || (GT == XS_GRID_UNIONIZED && !g.index);
   if (thread_kernel)
     return check ? launch_gather_tv<GT, true>(g, P, st) : launch_gather_tv<GT, false>(g, P, st);
@@ -1911,7 +2014,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   // the staged gather (default for sorted batches) only needs u at each task's
   // extreme energies; per-lookup u is searched when reported or otherwise used
   const int variant = g.unroll;
-  P.need_gidx = (!binned || a.out.grid_index || (variant != 0 && variant < 9)) ? 1 : 0;
+  P.need_gidx = (!binned || a.out.grid_index ||
+                 (!(a.flags & XS_FLAG_F32) && variant != 0 && variant < 9)) ? 1 : 0;
   P.tmp = ws.tmp;
   P.mat8 = ws.mat8;
   if (binned) {
@@ -1936,7 +2040,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   }
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   mark(2);
-  e = launch_gather_u<GT>(g, P, binned, st);
+  e = launch_gather_u<GT>(g, P, binned, (a.flags & XS_FLAG_F32) != 0, st);
   launched(1);
   mark(3);
   return e;

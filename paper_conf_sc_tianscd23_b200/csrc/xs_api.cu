@@ -247,6 +247,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   auto cleanup = [&]() {
     cudaFree(G.grid);
     cudaFree(G.iv);
+    cudaFree(G.iv32);
     cudaFree(G.U);
     cudaFree(G.UB);
     cudaFree(G.index);
@@ -263,6 +264,8 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
                                             6 * sizeof(double), st);
   const size_t iv_bytes = static_cast<size_t>(I) * N * kIvDoubles * sizeof(double);
   if (e == cudaSuccess) e = cudaMalloc(&G.iv, iv_bytes);
+  const size_t iv32_bytes = static_cast<size_t>(I) * N * kIv32Doubles * sizeof(double);
+  if (e == cudaSuccess) e = cudaMalloc(&G.iv32, iv32_bytes);
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.U, G.NU * sizeof(double));
   if (e == cudaSuccess && G.NU) e = cudaMalloc(&G.UB, (static_cast<size_t>(G.UBn) + 1) * 4);
   if (e == cudaSuccess && G.index_len && (G.index_layout & XS_INDEX_ROW))
@@ -276,13 +279,14 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cleanup();
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
-  G.device_bytes = grid_bytes + iv_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
+  G.device_bytes = grid_bytes + iv_bytes + iv32_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
   e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.mats, d->mats, tab * 4, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.concs, d->concs, tab * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = build_intervals(G, st);
+  if (e == cudaSuccess) e = build_intervals32(G, st);
   if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
     e = build_union_grid(G, G.U, st);
     if (e == cudaSuccess) e = build_union_table(G, st);
@@ -394,8 +398,10 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
   if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
   if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
-  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE))
+  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE | XS_FLAG_F32))
     return fail(XS_ERR_INVALID_ARG, "unknown flag bits");
+  if ((flags & XS_FLAG_F32) && (flags & XS_FLAG_BASELINE))
+    return fail(XS_ERR_UNSUPPORTED, "XS_FLAG_F32 cannot be combined with XS_FLAG_BASELINE");
   if (count == 0) return XS_OK;
   const size_t need = total_workspace(count, flags, g->d.n_mats);
   if (!workspace || ws_bytes < need)
@@ -580,8 +586,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
-          (value >= 17 && value <= 23)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12 or 17-23");
+          (value >= 17 && value <= 23) || (value >= 31 && value <= 33)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-23 or 31-33");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
@@ -637,6 +643,7 @@ void xs_free_grid(xs_grid* g) {
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   cudaFree(g->d.grid);
   cudaFree(g->d.iv);
+  cudaFree(g->d.iv32);
   cudaFree(g->d.U);
   cudaFree(g->d.UB);
   cudaFree(g->d.index);

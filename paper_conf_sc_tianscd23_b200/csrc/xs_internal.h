@@ -19,6 +19,7 @@ struct alignas(16) LookupRec {
 constexpr int kMaxMats = 64;  // materials supported by the bucketed kernels
 constexpr uint32_t kEnergyBins = 1u << 18;  // A2: energy bins per material
 constexpr int kIvDoubles = 14;  // interval-table entry (112 B; grid_build.cu K0d)
+constexpr int kIv32Doubles = 10;  // fp32-variant entry (80 B; grid_build.cu K0e)
 
 struct DeviceGrid {
   int device = 0;
@@ -32,6 +33,7 @@ struct DeviceGrid {
   int64_t NU = 0, index_len = 0;
   double* grid = nullptr;    // [I][N][6]
   double* iv = nullptr;      // [I][N][kIvDoubles] interval table (K0d), or null
+  double* iv32 = nullptr;    // [I][N][kIv32Doubles] fp32-variant interval table (K0e)
   double* U = nullptr;       // [NU]
   int32_t* UB = nullptr;     // [UBn + 1]: UB[b] = ub(U, b / UBn)  (A3 search table)
   int32_t UBn = 0;           // power of two
@@ -84,6 +86,7 @@ cudaError_t build_index_grid_t(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_intervals(const DeviceGrid& g, cudaStream_t st);
+cudaError_t build_intervals32(const DeviceGrid& g, cudaStream_t st);
 cudaError_t init_constants();
 
 // lookup.cu

@@ -20,7 +20,7 @@ LIB_PATH = os.path.join(HERE, "libxs.so")
 
 XS_ABI_VERSION = 1
 XS_GRID_UNIONIZED, XS_GRID_NUCLIDE, XS_GRID_HASH = 0, 1, 2
-XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE = 0x1, 0x2, 0x4
+XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE, XS_FLAG_F32 = 0x1, 0x2, 0x4, 0x8
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
  XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T) = range(7)
 XS_INDEX_AUTO, XS_INDEX_ROW, XS_INDEX_COL, XS_INDEX_BOTH = 0, 1, 2, 3
@@ -304,11 +304,13 @@ class Grid:
         return o, res
 
     def lookup(self, first_id: int, count: int, sort: bool = False, baseline: bool = False,
-               want=(), vsum=None, stream=None):
-        """A1-A8 for lookup ids [first_id, first_id+count) on the current stream.
+               want=(), vsum=None, stream=None, f32: bool = False):
+        """A1-A8 for lookup ids [first_id, first_id+count) on the current stream
+        (f32: the fp32 variant, XS_FLAG_F32).
         Returns (vsum tensor [2] uint64-as-int64 on device, dict of outputs)."""
         import torch
-        flags = (XS_FLAG_SORT if sort else 0) | (XS_FLAG_BASELINE if baseline else 0)
+        flags = ((XS_FLAG_SORT if sort else 0) | (XS_FLAG_BASELINE if baseline else 0) |
+                 (XS_FLAG_F32 if f32 else 0))
         if vsum is None:
             vsum = torch.zeros(2, dtype=torch.int64, device=self.device)
         o, res = self._outputs(count, want, vsum)
@@ -317,13 +319,15 @@ class Grid:
         xs_lookup_batch(self._h, first_id, count, flags, o, ws.data_ptr(), ws.numel(), st)
         return vsum, res
 
-    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, stream=None):
+    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, stream=None,
+                        f32: bool = False):
         """A2-A8 for caller-given (energy, material).  energy/mat are CUDA
         tensors (float64 / int32), or CPU tensors (then XS_FLAG_HOST_IO: staged
         copies inside the call, outputs returned on the host)."""
         import torch
         host = not energy.is_cuda
-        flags = (XS_FLAG_SORT if sort else 0) | (XS_FLAG_HOST_IO if host else 0)
+        flags = ((XS_FLAG_SORT if sort else 0) | (XS_FLAG_HOST_IO if host else 0) |
+                 (XS_FLAG_F32 if f32 else 0))
         count = energy.numel()
         if vsum is None:
             vsum = torch.zeros(2, dtype=torch.int64, device="cpu" if host else self.device)
