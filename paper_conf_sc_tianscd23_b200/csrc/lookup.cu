@@ -455,8 +455,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
     for (int it = 0; it < kPrepItems; ++it) {
       const uint64_t i = c0 + static_cast<uint64_t>(it) * kPrepThreads + threadIdx.x;
       if (i < P.count) {
-        if (BINNED)
-          P.perm[rank[it]] = static_cast<uint32_t>(i);  // 4-B writes into an L2-resident array
+        if (BINNED) P.perm[rank[it]] = static_cast<uint32_t>(i);  // 4-B writes, L2-resident array
         else
           P.recs[s_base[mm[it]] + rank[it]] = rec[it];
       }
@@ -1419,8 +1418,12 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
     return SHARED ? q[0] : __ldg(q);
   };
+  if (n_int == 0) {  // one entry: every lookup of the task lies in it (warp-uniform)
+    acc.template interp<SHARED>(win, p, conc, 0, R);
+    return;
+  }
   int i0 = 0, iL = 0;
-  const int top = n_int > 0 ? 1 << (31 - __clz(n_int)) : 0;
+  const int top = 1 << (31 - __clz(n_int));
   for (int step = top; step > 0; step >>= 1) {
     const int t0 = i0 + step, tL = iL + step;
     const double e0 = E(t0 <= n_int ? t0 : n_int), eL = E(tL <= n_int ? tL : n_int);

@@ -420,3 +420,18 @@ def test_explicit_host_io_chunked(X, sort):
         assert vs.tolist() == [S, p.size]
         assert np.array_equal(res["macro_xs"].numpy(), M)
         assert np.array_equal(res["verification"].numpy(), v)
+
+
+@pytest.mark.parametrize("variant", [0, 9, 17, 19, 20, 21])
+@pytest.mark.parametrize("grid_type,bins", [("unionized", 0), ("hash", 97)])
+def test_vsum_only_sorted(X, variant, grid_type, bins):
+    """Sorted batches with only vsum requested take the staged gather's fast
+    record path (energies read in task order, no per-lookup u)."""
+    g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
+    g.set_param("variant", variant)
+    mode = oracle.HASH if grid_type == "hash" else oracle.UNIONIZED
+    for first, count in [(0, 100_000), (77, 4099), (5, 1)]:
+        S = oracle_for("tiny", hash_bins=bins).run(first, count, mode=mode, nthreads=NT)
+        vs, _ = g.lookup(first, count, sort=True)
+        torch.cuda.synchronize()
+        assert [int(x) for x in vs.cpu()] == [S, count]
