@@ -1944,18 +1944,22 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 21: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, true>(g, P, st);
     case 22: return launch_gather_s3<GT, 4, 1, 8, 16, CHECK, true>(g, P, st);
     case 23: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK, true>(g, P, st);
+    case 24: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
 
 // fp32 variant (R18): the staged interval-table gather for every batch
-// (variants 31-33 select its shape; any other value the default).
+// (variants 31-34 select its shape; any other value the default, 24 warps
+// per block: binary32 accumulators leave room for 80 registers per thread).
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   switch (g.unroll) {
     case 32: return launch_gather_s3<GT, 8, 2, 8, 16, CHECK, false, true>(g, P, st);
     case 33: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, true, true>(g, P, st);
-    default: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, false, true>(g, P, st);
+    case 31: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, false, true>(g, P, st);
+    case 34: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK, false, true>(g, P, st);
+    default: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
   }
 }
 

@@ -586,8 +586,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
-          (value >= 17 && value <= 23) || (value >= 31 && value <= 33)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-23 or 31-33");
+          (value >= 17 && value <= 24) || (value >= 31 && value <= 35)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-24 or 31-35");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
