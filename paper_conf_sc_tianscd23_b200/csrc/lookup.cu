@@ -1422,13 +1422,20 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     acc.template interp<SHARED>(win, p, conc, 0, R);
     return;
   }
-  int i0 = 0, iL = 0;
+  int i0, iL;
   const int top = 1 << (31 - __clz(n_int));
-  for (int step = top; step > 0; step >>= 1) {
-    const int t0 = i0 + step, tL = iL + step;
-    const double e0 = E(t0 <= n_int ? t0 : n_int), eL = E(tL <= n_int ? tL : n_int);
-    if (t0 <= n_int && e0 <= p[0]) i0 = t0;
-    if (tL <= n_int && eL <= p[R - 1]) iL = tL;
+  if (n_int == 1) {  // two entries (the common multi-entry case): one shared probe
+    const double e = E(1);
+    i0 = e <= p[0] ? 1 : 0;
+    iL = e <= p[R - 1] ? 1 : 0;
+  } else {
+    i0 = iL = 0;
+    for (int step = top; step > 0; step >>= 1) {
+      const int t0 = i0 + step, tL = iL + step;
+      const double e0 = E(t0 <= n_int ? t0 : n_int), eL = E(tL <= n_int ? tL : n_int);
+      if (t0 <= n_int && e0 <= p[0]) i0 = t0;
+      if (tL <= n_int && eL <= p[R - 1]) iL = tL;
+    }
   }
   if (__all_sync(0xffffffffu, i0 == iL)) {
     acc.template interp<SHARED>(win + i0 * kE, p, conc, 0, R);
