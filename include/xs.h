@@ -155,6 +155,9 @@ typedef struct {
                                  binary32 with fused multiply-adds.  macro_xs
                                  receives the binary32 results widened.  Not
                                  combinable with XS_FLAG_BASELINE.             */
+#define XS_FLAG_MAT_U8 0x10u  /* xs_lookup_explicit: `mat` points to uint8_t[count]
+                                 (a material id per byte) instead of int32_t —
+                                 a quarter of the material bytes to upload    */
 
 /* tables for xs_get_table (element type in brackets) */
 #define XS_TABLE_NUCLIDE_GRID 0 /* [double] I*N*6                               */

@@ -84,6 +84,7 @@ struct Params {
   uint32_t count;
   const double* in_energy;
   const int32_t* in_mat;
+  const uint8_t* in_mat8;   // XS_FLAG_MAT_U8 (else null)
   // workspace
   uint32_t* counts;
   uint32_t* cursor;
@@ -107,7 +108,7 @@ struct Params {
 
 __device__ __forceinline__ Sample get_lookup(const Params& P, uint32_t i) {
   if (P.in_energy) {
-    int32_t m = P.in_mat[i];
+    int32_t m = P.in_mat8 ? static_cast<int32_t>(P.in_mat8[i]) : P.in_mat[i];
     if (m < 0 || m >= P.n_mats) m = P.n_mats;  // invalid bucket
     return Sample{P.in_energy[i], m};
   }
@@ -289,7 +290,9 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
       P.tmp[i] = r;
       P.mat8[i] = static_cast<uint8_t>(m);
       if (P.out_E) P.out_E[i] = p;
-      if (P.out_mat) P.out_mat[i] = valid ? m : (P.in_mat ? P.in_mat[i] : -1);
+      if (P.out_mat)
+        P.out_mat[i] = valid ? m : (P.in_mat8 ? static_cast<int32_t>(P.in_mat8[i])
+                                    : (P.in_mat ? P.in_mat[i] : -1));
       if (P.out_gidx) P.out_gidx[i] = valid ? gi : -1;
       if (!valid) write_invalid(P, i);
     }
@@ -1708,7 +1711,8 @@ __global__ void __launch_bounds__(256) k_baseline(Params P) {
     const Sample s = get_lookup(P, i);
     if (s.mat >= P.n_mats) {
       write_invalid(P, i);
-      if (P.out_mat) P.out_mat[i] = P.in_mat ? P.in_mat[i] : -1;
+      if (P.out_mat)
+        P.out_mat[i] = P.in_mat8 ? static_cast<int32_t>(P.in_mat8[i]) : (P.in_mat ? P.in_mat[i] : -1);
       if (P.out_gidx) P.out_gidx[i] = -1;
       if (P.out_E) P.out_E[i] = s.p;
       continue;
@@ -1995,6 +1999,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.count = a.count;
   P.in_energy = a.in_energy;
   P.in_mat = a.in_mat;
+  P.in_mat8 = a.in_mat8;
   P.counts = ws.counts;
   P.cursor = ws.cursor;
   P.task_next = ws.cursor + (kMaxMats + 1);

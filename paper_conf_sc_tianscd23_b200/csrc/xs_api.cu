@@ -398,8 +398,12 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
   if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
   if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
-  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE | XS_FLAG_F32))
+  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE | XS_FLAG_F32 | XS_FLAG_MAT_U8))
     return fail(XS_ERR_INVALID_ARG, "unknown flag bits");
+  if ((flags & XS_FLAG_MAT_U8) && !energy)
+    return fail(XS_ERR_INVALID_ARG, "XS_FLAG_MAT_U8 applies to explicit lookups only");
+  const bool mat8 = (flags & XS_FLAG_MAT_U8) != 0;
+  const size_t mat_es = mat8 ? 1 : 4;  // bytes per material id
   if ((flags & XS_FLAG_F32) && (flags & XS_FLAG_BASELINE))
     return fail(XS_ERR_UNSUPPORTED, "XS_FLAG_F32 cannot be combined with XS_FLAG_BASELINE");
   if (count == 0) return XS_OK;
@@ -418,7 +422,8 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   a.count = static_cast<uint32_t>(count);
   a.flags = flags;
   a.in_energy = energy;
-  a.in_mat = mat;
+  a.in_mat = mat8 ? nullptr : mat;
+  a.in_mat8 = mat8 ? reinterpret_cast<const uint8_t*>(mat) : nullptr;
   a.out = *out;
   a.launches = &g->d.launches;
   if (g->timing) {
@@ -443,11 +448,12 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
     staging_layout(count, static_cast<char*>(workspace) + wbytes, &sg);
     if (energy && !chunked) {
       XS_TRY(cudaMemcpyAsync(sg.energy, energy, count * 8, cudaMemcpyHostToDevice, st), "H2D energy");
-      XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * 4, cudaMemcpyHostToDevice, st), "H2D mat");
+      XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * mat_es, cudaMemcpyHostToDevice, st), "H2D mat");
     }
     if (energy) {
       a.in_energy = sg.energy;
-      a.in_mat = sg.mat;
+      a.in_mat = mat8 ? nullptr : sg.mat;
+      a.in_mat8 = mat8 ? reinterpret_cast<const uint8_t*>(sg.mat) : nullptr;
     }
     XS_TRY(cudaMemcpyAsync(sg.vsum, out->vsum, 16, cudaMemcpyHostToDevice, st), "H2D vsum");
     a.out.vsum = sg.vsum;
@@ -476,7 +482,9 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
       const uint64_t b = k * chunk, n = std::min(chunk, count - b);
       XS_TRY(cudaMemcpyAsync(sg.energy + b, energy + b, n * 8, cudaMemcpyHostToDevice,
                              g->copy_stream), "H2D energy");
-      XS_TRY(cudaMemcpyAsync(sg.mat + b, mat + b, n * 4, cudaMemcpyHostToDevice, g->copy_stream),
+      XS_TRY(cudaMemcpyAsync(reinterpret_cast<char*>(sg.mat) + b * mat_es,
+                             reinterpret_cast<const char*>(mat) + b * mat_es, n * mat_es,
+                             cudaMemcpyHostToDevice, g->copy_stream),
              "H2D mat");
       XS_TRY(cudaEventRecord(g->chunk_ev[k], g->copy_stream), "event");
     }
@@ -487,7 +495,8 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
       XS_TRY(cudaStreamWaitEvent(st, g->chunk_ev[k], 0), "wait");
       c.count = static_cast<uint32_t>(n);
       c.in_energy = sg.energy + b;
-      c.in_mat = sg.mat + b;
+      c.in_mat = mat8 ? nullptr : sg.mat + b;
+      c.in_mat8 = mat8 ? reinterpret_cast<const uint8_t*>(sg.mat) + b : nullptr;
       c.out.macro_xs = a.out.macro_xs ? a.out.macro_xs + b * 5 : nullptr;
       c.out.energy = a.out.energy ? a.out.energy + b : nullptr;
       c.out.mat = a.out.mat ? a.out.mat + b : nullptr;

@@ -59,6 +59,7 @@ struct LookupArgs {
   uint32_t flags = 0;
   const double* in_energy = nullptr;  // explicit mode (device)
   const int32_t* in_mat = nullptr;
+  const uint8_t* in_mat8 = nullptr;   // XS_FLAG_MAT_U8 (explicit mode, device)
   xs_outputs out{};                    // device pointers
   cudaEvent_t* ev = nullptr;           // [4] phase events (optional)
   uint64_t* launches = nullptr;        // incremented per kernel launch

@@ -21,6 +21,7 @@ LIB_PATH = os.path.join(HERE, "libxs.so")
 XS_ABI_VERSION = 1
 XS_GRID_UNIONIZED, XS_GRID_NUCLIDE, XS_GRID_HASH = 0, 1, 2
 XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE, XS_FLAG_F32 = 0x1, 0x2, 0x4, 0x8
+XS_FLAG_MAT_U8 = 0x10
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
  XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T) = range(7)
 XS_INDEX_AUTO, XS_INDEX_ROW, XS_INDEX_COL, XS_INDEX_BOTH = 0, 1, 2, 3
@@ -322,12 +323,14 @@ class Grid:
     def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, stream=None,
                         f32: bool = False):
         """A2-A8 for caller-given (energy, material).  energy/mat are CUDA
-        tensors (float64 / int32), or CPU tensors (then XS_FLAG_HOST_IO: staged
-        copies inside the call, outputs returned on the host)."""
+        tensors (float64 / int32 or uint8 -> XS_FLAG_MAT_U8), or CPU tensors
+        (then XS_FLAG_HOST_IO: staged copies inside the call, outputs returned
+        on the host)."""
         import torch
         host = not energy.is_cuda
         flags = ((XS_FLAG_SORT if sort else 0) | (XS_FLAG_HOST_IO if host else 0) |
-                 (XS_FLAG_F32 if f32 else 0))
+                 (XS_FLAG_F32 if f32 else 0) |
+                 (XS_FLAG_MAT_U8 if mat.dtype == torch.uint8 else 0))
         count = energy.numel()
         if vsum is None:
             vsum = torch.zeros(2, dtype=torch.int64, device="cpu" if host else self.device)

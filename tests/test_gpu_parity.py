@@ -413,9 +413,9 @@ def test_explicit_host_io_chunked(X, sort):
     p = rng.random(50_003)
     m = rng.integers(0, 12, p.size).astype(np.int32)
     S, M, v = o.run_explicit(p, m, mode=oracle.UNIONIZED, nthreads=NT)
-    for chunk in (1 << 22, 7_001, 1_024):
+    for chunk, mt in [(1 << 22, m), (7_001, m), (1_024, m), (7_001, m.astype(np.uint8))]:
         g.set_param("host_chunk", chunk)
-        vs, res = g.lookup_explicit(torch.tensor(p), torch.tensor(m), sort=sort,
+        vs, res = g.lookup_explicit(torch.tensor(p), torch.tensor(mt), sort=sort,
                                     want=("macro_xs", "verification"))
         assert vs.tolist() == [S, p.size]
         assert np.array_equal(res["macro_xs"].numpy(), M)
@@ -425,8 +425,8 @@ def test_explicit_host_io_chunked(X, sort):
 @pytest.mark.parametrize("variant", [0, 9, 17, 19, 20, 21])
 @pytest.mark.parametrize("grid_type,bins", [("unionized", 0), ("hash", 97)])
 def test_vsum_only_sorted(X, variant, grid_type, bins):
-    """Sorted batches with only vsum requested take the staged gather's fast
-    record path (energies read in task order, no per-lookup u)."""
+    """Sorted batches with only vsum requested (no per-lookup outputs: the
+    staged gathers search U only at each task's extreme energies)."""
     g = X.Grid.from_preset("tiny", grid_type=grid_type, hash_bins=bins)
     g.set_param("variant", variant)
     mode = oracle.HASH if grid_type == "hash" else oracle.UNIONIZED
@@ -435,3 +435,29 @@ def test_vsum_only_sorted(X, variant, grid_type, bins):
         vs, _ = g.lookup(first, count, sort=True)
         torch.cuda.synchronize()
         assert [int(x) for x in vs.cpu()] == [S, count]
+
+
+@pytest.mark.parametrize("host", [False, True])
+@pytest.mark.parametrize("sort", [False, True])
+def test_explicit_lookups_u8_materials(X, host, sort):
+    """XS_FLAG_MAT_U8: one byte per material id, same results as int32 ids;
+    ids >= n_mats (e.g. 255) are invalid lookups."""
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    rng = np.random.default_rng(21)
+    p = rng.random(30_001)
+    m = rng.integers(0, 12, p.size).astype(np.uint8)
+    m[3] = 255
+    m[9] = 12
+    ok = m < 12
+    S, M, v = o.run_explicit(np.where(ok, p, 0.5), np.where(ok, m, 0).astype(np.int32),
+                             mode=oracle.UNIONIZED, nthreads=NT)
+    dev = "cpu" if host else "cuda"
+    vs, res = g.lookup_explicit(torch.tensor(p, device=dev), torch.tensor(m, device=dev),
+                                sort=sort, want=("macro_xs", "verification", "mat"))
+    torch.cuda.synchronize()
+    Mg, vg = res["macro_xs"].cpu().numpy(), res["verification"].cpu().numpy()
+    assert np.array_equal(Mg[ok], M[ok]) and np.array_equal(vg[ok], v[ok])
+    assert np.all(vg[~ok] == 0)
+    assert np.array_equal(res["mat"].cpu().numpy(), m.astype(np.int32))
+    assert [int(x) for x in vs.cpu()] == [int(v[ok].sum()), int(ok.sum())]

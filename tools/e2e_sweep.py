@@ -13,7 +13,7 @@ g = X.Grid.from_preset("large")
 L = 17_000_000
 _, res = g.lookup(0, L, sort=True, want=("energy", "mat"))
 e = res["energy"].cpu().pin_memory()
-m = res["mat"].cpu().pin_memory()
+m = res["mat"].cpu().to(torch.uint8).pin_memory()
 vs = torch.zeros(2, dtype=torch.int64).pin_memory()
 for chunk in [int(a) for a in (sys.argv[1:] or ["17000000", "8500000", "4250000", "2125000"])]:
     g.set_param("host_chunk", chunk)
