@@ -4,7 +4,7 @@ import paper_conf_sc_tianscd23_b200.xs as X
 for cfg in ["large", "small", "large-hash"]:
     g = X.Grid.from_preset(cfg)
     L = 17_000_000
-    for f32, var in [(False, 0), (True, 0)]:
+    for f32, var in [(False, 0), (True, 0), (True, 36)]:
         g.set_param("variant", var)
         vs = torch.zeros(2, dtype=torch.int64, device="cuda")
         g.lookup(0, L, sort=True, vsum=vs, f32=f32); torch.cuda.synchronize()

@@ -1936,9 +1936,9 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // blocks); 9-12 TMA-staged record windows (R, stages D, window W records,
   // warps per block); 17-20 TMA-staged interval-table windows (R, group
   // size D, window W entries, warps per block).  Measured best on B200 (large,
-  // large-hash, small): k_gather_s3 (4, 2, 8, 16) = variant 19.
+  // large-hash, small): k_gather_s3 (4, 4, 6, 16) = variant 25.
   int v = g.unroll;
-  if (v == 0) v = 19;
+  if (v == 0) v = 25;
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
@@ -1956,6 +1956,10 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 22: return launch_gather_s3<GT, 4, 1, 8, 16, CHECK, true>(g, P, st);
     case 23: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK, true>(g, P, st);
     case 24: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK>(g, P, st);
+    case 25: return launch_gather_s3<GT, 4, 4, 6, 16, CHECK>(g, P, st);
+    case 26: return launch_gather_s3<GT, 4, 3, 6, 16, CHECK>(g, P, st);
+    case 27: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK>(g, P, st);
+    case 28: return launch_gather_s3<GT, 4, 4, 4, 16, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
@@ -1970,6 +1974,7 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
     case 33: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, true, true>(g, P, st);
     case 31: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, false, true>(g, P, st);
     case 34: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK, false, true>(g, P, st);
+    case 36: return launch_gather_s3<GT, 4, 4, 6, 24, CHECK, false, true>(g, P, st);
     default: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
   }
 }

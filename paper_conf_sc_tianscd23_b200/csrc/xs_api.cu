@@ -595,8 +595,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
-          (value >= 17 && value <= 24) || (value >= 31 && value <= 35)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-24 or 31-35");
+          (value >= 17 && value <= 28) || (value >= 31 && value <= 36)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28 or 31-36");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");

@@ -66,7 +66,7 @@ def test_tiny_f32_parity(X, grid_type, bins, sort):
     assert np.quantile(rel, 0.999) < 1e-5
 
 
-@pytest.mark.parametrize("variant", [0, 31, 32, 33, 34])
+@pytest.mark.parametrize("variant", [0, 31, 32, 33, 34, 36])
 @pytest.mark.parametrize("first,count", [(0, 1), (5, 31), (999_999, 4097), (3, 70_001)])
 def test_f32_shapes_and_ragged(X, variant, first, count):
     g = X.Grid.from_preset("tiny")
