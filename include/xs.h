@@ -219,9 +219,11 @@ xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t
 xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
                        void* host_dst);
 
-/* Tuning knobs: "variant" (gather kernel: 0 = default, 1-12 = the kernel
- * shapes listed in DESIGN.md §4), "blocks_per_sm" (0 = occupancy calculator)
- * and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in
+/* Tuning knobs: "variant" (gather kernel: 0 = default, 1-4, 9-12, 17-28,
+ * 31-36 = the kernel shapes listed in DESIGN.md §4), "blocks_per_sm"
+ * (0 = occupancy calculator), "legacy_sort" (1: XS_FLAG_SORT through the
+ * global-atomic bins and a permutation instead of the partitioned counting
+ * sort; comparison only) and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in
  * chunks of this many lookups, overlapped with the lookups of the previous
  * chunk; default 10^7, split evenly).  INVALID_ARG for an
  * unknown name or value.  Never changes results. */

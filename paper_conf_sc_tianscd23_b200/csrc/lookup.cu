@@ -97,6 +97,14 @@ struct Params {
   uint32_t* perm;      // A2: batch positions in (material, energy) order (else null)
   int need_gidx;       // k_sample must search u per lookup (else the staged gather
                        // searches only each task's extreme energies)
+  // partitioned A2 (k_part_*): H[block][key] lives in bins
+  int cbits;            // coarse energy bits per material
+  uint32_t* key_tot;    // [nkeys] lookups per coarse key
+  uint32_t* key_start;  // [nkeys] first position of the key
+  double* sp_tmp;       // [count] energies in coarse-key order
+  uint32_t* sidx_tmp;   // [count] their batch positions (null: no per-lookup outputs)
+  double* sp;           // [count] energies in (material, energy bin) order
+  uint32_t* sidx;       // [count] their batch positions, or null
   // outputs
   double* out_M;
   double* out_E;
@@ -337,6 +345,36 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* excl) 
   return total;
 }
 
+// the same for NT threads (a multiple of 32, at most 1024)
+template <int NT>
+__device__ __forceinline__ uint32_t block_excl_scan_n(uint32_t v, uint32_t* excl) {
+  constexpr int kW = NT / 32;
+  __shared__ uint32_t s_w[kW];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t t = lane < kW ? s_w[lane] : 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, t, o);
+      if (lane >= o) t += y;
+    }
+    if (lane < kW) s_w[lane] = t;
+  }
+  __syncthreads();
+  *excl = (w ? s_w[w - 1] : 0u) + x - v;
+  const uint32_t total = s_w[kW - 1];
+  __syncthreads();
+  return total;
+}
+
 __global__ void __launch_bounds__(1024) k_scan_partial(Params P) {
   const uint32_t* c = P.bins + static_cast<uint64_t>(blockIdx.x) * kScanChunk;
   uint32_t v = 0;
@@ -467,6 +505,267 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
   }
 }
 
+// ----------------------------------------------- A2, partitioned variant ---
+// The A2 of the staged gather (its default): a two-level counting sort that
+// moves only the energy (8 B) and, when per-lookup outputs are requested, the
+// batch position (4 B).  The key is the same (material, energy bin of width
+// 2^-18) as above, split into a coarse part (material, top cbits of the bin;
+// a small fan-out, so that every tile writes runs of whole sectors) and a
+// fine part (the remaining 18 - cbits bits):
+//   k_part_count    A1 (+ per-lookup A3 outputs) in batch order; per-tile
+//                   histogram of coarse keys in shared memory -> H[tile][key]
+//   k_part_colscan  per key: exclusive scan of H over tiles, key totals
+//   k_part_keyscan  exclusive scan of the key totals -> key starts; material counts
+//   k_part_place    A1 again, tile by tile; position = key start + tile offset +
+//                   shared-memory rank (energies in coarse-key order)
+//   k_part_fine     one block per coarse key: counting sort of its segment by
+//                   the fine key (shared-memory histogram, segment L2-resident)
+// Only shared-memory atomics.  Order inside a fine bin is arbitrary: results
+// never depend on it.
+constexpr int kPartItems = kPrepItems;
+constexpr uint32_t kPartChunk = kPrepThreads * kPartItems;  // lookups per block round
+constexpr uint32_t kPartMaxTiles = 4000;  // H [tiles][nkeys] fits the A2 bin area
+
+__host__ __device__ __forceinline__ uint32_t part_tile_chunks(uint64_t count) {
+  const uint64_t chunks = (count + kPartChunk - 1) / kPartChunk;
+  const uint64_t per = (chunks + kPartMaxTiles - 1) / kPartMaxTiles;
+  return static_cast<uint32_t>(per < 8 ? 8 : per);
+}
+
+// LCG^n as an affine map (A, C) from the constant-memory jump table
+__device__ __forceinline__ void affine_pow(uint64_t n, uint64_t& A, uint64_t& C) {
+  A = 1;
+  C = 0;
+  int b = 0;
+  while (n) {
+    if (n & 1ULL) {
+      A = (A * c_jump.A[b]) & kMask63;
+      C = (C * c_jump.A[b] + c_jump.C[b]) & kMask63;
+    }
+    n >>= 1;
+    ++b;
+  }
+}
+
+__device__ __forceinline__ uint32_t part_key(const Params& P, const Sample& s) {
+  return (static_cast<uint32_t>(s.mat) << P.cbits) | (energy_bin(s.p) >> (18 - P.cbits));
+}
+
+// The kPartItems lookups of thread t in the chunk starting at c0 (the same
+// assignment in k_part_count and k_part_place).  sc = stream state at the
+// chunk's first lookup, tA, tC = LCG^(2 kPartItems t).
+__device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint64_t sc, uint64_t tA,
+                                             uint64_t tC, Sample (&smp)[kPartItems],
+                                             bool (&ok)[kPartItems]) {
+  uint64_t st = (tA * sc + tC) & kMask63;
+#pragma unroll
+  for (int it = 0; it < kPartItems; ++it) {
+    const uint64_t i = c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it;
+    ok[it] = i < P.count;
+    if (P.in_energy) {
+      smp[it] = ok[it] ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
+    } else {
+      st = lcg_next(st);
+      const double pe = lcg_double(st);
+      st = lcg_next(st);
+      smp[it] = Sample{pe, pick_material(lcg_double(st))};
+    }
+  }
+}
+
+// Stream constants of a k_part_* thread: the chunk-to-chunk jump and the
+// thread's offset inside a chunk; the state at a tile's first lookup is one
+// fast-forward per tile.
+struct PartStream {
+  uint64_t cA, cC, tA, tC;
+  __device__ __forceinline__ void init(const Params& P) {
+    cA = tA = 1;
+    cC = tC = 0;
+    if (P.in_energy) return;
+    affine_pow(2ull * kPartChunk, cA, cC);
+    affine_pow(2ull * kPartItems * threadIdx.x, tA, tC);
+  }
+  __device__ __forceinline__ uint64_t at(const Params& P, uint64_t first) const {
+    return P.in_energy ? 0 : fast_forward(P.seed, 2 * (P.first_id + first));
+  }
+  __device__ __forceinline__ uint64_t next(uint64_t sc) const { return (cA * sc + cC) & kMask63; }
+};
+
+template <int GT>
+__global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
+  extern __shared__ uint32_t s_h[];  // [nkeys]
+  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
+  const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
+  const bool outputs = P.out_E || P.out_mat || P.out_gidx || P.out_M || P.out_v;
+  PartStream ps;
+  ps.init(P);
+  for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
+    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) s_h[t] = 0;
+    __syncthreads();
+    uint64_t sc = ps.at(P, tl * tlen);
+    for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
+      const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
+      if (c0 >= P.count) break;
+      Sample smp[kPartItems];
+      bool ok[kPartItems];
+      part_samples(P, c0, sc, ps.tA, ps.tC, smp, ok);
+#pragma unroll
+      for (int it = 0; it < kPartItems; ++it) {
+        if (!ok[it]) continue;
+        atomicAdd(&s_h[part_key(P, smp[it])], 1u);
+        if (!outputs) continue;
+        const uint32_t i = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
+        const bool valid = smp[it].mat < P.n_mats;
+        if (P.out_E) P.out_E[i] = smp[it].p;
+        if (P.out_mat)
+          P.out_mat[i] = valid ? smp[it].mat
+                               : (P.in_mat8 ? static_cast<int32_t>(P.in_mat8[i]) : (P.in_mat ? P.in_mat[i] : -1));
+        if (P.out_gidx) {
+          int32_t gi = -1;
+          if (GT == XS_GRID_UNIONIZED) gi = union_index_tab(P, smp[it].p);
+          if (GT == XS_GRID_HASH) gi = hash_bin(smp[it].p, P.du, P.B);
+          P.out_gidx[i] = valid ? gi : -1;
+        }
+        if (!valid) write_invalid(P, i);
+      }
+    }
+    __syncthreads();
+    uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
+    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) row[t] = s_h[t];
+    __syncthreads();
+  }
+}
+
+// H[t][key] -> exclusive prefix over tiles t (per key); key totals.  Block =
+// 32 keys x 32 slices of the tiles.
+__global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
+  __shared__ uint32_t s_p[32][33];
+  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int key = blockIdx.x * 32 + threadIdx.x;
+  const int sl = threadIdx.y;
+  const int per = (nb + 31) / 32;
+  const int b0 = sl * per, b1 = min(nb, b0 + per);
+  uint32_t sum = 0;
+  if (key < nkeys)
+    for (int b = b0; b < b1; ++b) sum += P.bins[static_cast<uint64_t>(b) * nkeys + key];
+  s_p[sl][threadIdx.x] = sum;
+  __syncthreads();
+  if (sl == 0) {
+    uint32_t run = 0;
+    for (int q = 0; q < 32; ++q) {
+      const uint32_t v = s_p[q][threadIdx.x];
+      s_p[q][threadIdx.x] = run;
+      run += v;
+    }
+    if (key < nkeys) P.key_tot[key] = run;
+  }
+  __syncthreads();
+  if (key < nkeys) {
+    uint32_t run = s_p[sl][threadIdx.x];
+    for (int b = b0; b < b1; ++b) {
+      uint32_t* h = P.bins + static_cast<uint64_t>(b) * nkeys + key;
+      const uint32_t v = *h;
+      *h = run;
+      run += v;
+    }
+  }
+}
+
+// key_start = exclusive scan of key_tot (one block); counts[m] per material
+__global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
+  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int per = (nkeys + 1023) / 1024;
+  const int k0 = threadIdx.x * per, k1 = min(nkeys, k0 + per);
+  uint32_t sum = 0;
+  for (int k = k0; k < k1; ++k) sum += P.key_tot[k];
+  uint32_t ex;
+  const uint32_t total = block_excl_scan(sum, &ex);
+  for (int k = k0; k < k1; ++k) {
+    P.key_start[k] = ex;
+    ex += P.key_tot[k];
+  }
+  __syncthreads();
+  for (int m = threadIdx.x; m <= P.n_mats; m += blockDim.x) {
+    const uint32_t s = P.key_start[m << P.cbits];
+    const uint32_t e = m < P.n_mats ? P.key_start[(m + 1) << P.cbits] : total;
+    P.counts[m] = e - s;
+  }
+}
+
+template <int GT>
+__global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
+  extern __shared__ uint32_t s_cur[];  // [nkeys]
+  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
+  const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
+  PartStream ps;
+  ps.init(P);
+  for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
+    const uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
+    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) s_cur[t] = P.key_start[t] + row[t];
+    __syncthreads();
+    uint64_t sc = ps.at(P, tl * tlen);
+    for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
+      const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
+      if (c0 >= P.count) break;
+      Sample smp[kPartItems];
+      bool ok[kPartItems];
+      part_samples(P, c0, sc, ps.tA, ps.tC, smp, ok);
+#pragma unroll
+      for (int it = 0; it < kPartItems; ++it) {
+        if (!ok[it] || smp[it].mat >= P.n_mats) continue;  // invalid lookups are not gathered
+        const uint32_t pos = atomicAdd(&s_cur[part_key(P, smp[it])], 1u);
+        P.sp_tmp[pos] = smp[it].p;
+        if (P.sidx_tmp)
+          P.sidx_tmp[pos] = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// one block per coarse key of a valid material: counting sort of the
+// segment by the fine key (the low 18 - cbits bits of the energy bin)
+constexpr int kFineThreads = 1024;
+__global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
+  extern __shared__ uint32_t s_f[];  // [nf]
+  const int key = blockIdx.x;
+  const uint32_t s = P.key_start[key], n = P.key_tot[key];
+  if (n == 0) return;
+  const int fb = 18 - P.cbits;
+  const uint32_t nf = 1u << fb, fmask = nf - 1u;
+  for (uint32_t t = threadIdx.x; t < nf; t += blockDim.x) s_f[t] = 0;
+  __syncthreads();
+  const double* src = P.sp_tmp + s;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&s_f[energy_bin(src[i]) & fmask], 1u);
+  __syncthreads();
+  // exclusive scan of s_f: each thread a run of nf / kFineThreads bins (nf >= 64)
+  const uint32_t per = (nf + kFineThreads - 1) / kFineThreads;
+  const uint32_t f0 = threadIdx.x * per;
+  uint32_t sum = 0;
+  for (uint32_t f = f0; f < f0 + per && f < nf; ++f) sum += s_f[f];
+  uint32_t ex;
+  block_excl_scan_n<kFineThreads>(sum, &ex);
+  for (uint32_t f = f0; f < f0 + per && f < nf; ++f) {
+    const uint32_t v = s_f[f];
+    s_f[f] = ex;
+    ex += v;
+  }
+  __syncthreads();
+  double* dst = P.sp + s;
+  const uint32_t* isrc = P.sidx_tmp ? P.sidx_tmp + s : nullptr;
+  uint32_t* idst = P.sidx ? P.sidx + s : nullptr;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const double p = src[i];
+    const uint32_t pos = atomicAdd(&s_f[energy_bin(p) & fmask], 1u);
+    dst[pos] = p;
+    if (idst) idst[pos] = isrc[i];
+  }
+}
+
 // ------------------------------------------------------------- A4 -- A8 ---
 // Bracket index k_n for the lookup's energy through the grid's structure.
 template <int GT>
@@ -486,6 +785,13 @@ constexpr int kLPT = 32 / kG;         // lookups per warp task (10)
 // Record at bucket position pos: A2 batches go through the permutation
 // (tmp holds the bin rank in idx; the batch index is the permutation value).
 __device__ __forceinline__ LookupRec load_rec(const Params& P, uint32_t pos) {
+  if (P.sp) {  // partitioned A2: energies (and positions) in sorted order, no u
+    LookupRec r;
+    r.p = P.sp[pos];
+    r.idx = P.sidx ? P.sidx[pos] : 0u;
+    r.gidx = 0;
+    return r;
+  }
   if (P.perm) {
     const uint32_t i = __ldg(P.perm + pos);
     LookupRec r = P.tmp[i];
@@ -1425,13 +1731,22 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     acc.template interp<SHARED>(win, p, conc, 0, R);
     return;
   }
-  int i0, iL;
-  const int top = 1 << (31 - __clz(n_int));
   if (n_int == 1) {  // two entries (the common multi-entry case): one shared probe
     const double e = E(1);
-    i0 = e <= p[0] ? 1 : 0;
-    iL = e <= p[R - 1] ? 1 : 0;
-  } else {
+    int i[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) i[r] = e <= p[r] ? 1 : 0;
+    if (__all_sync(0xffffffffu, i[0] == i[R - 1])) {  // p sorted within the lane
+      acc.template interp<SHARED>(win + i[0] * kE, p, conc, 0, R);
+      return;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) acc.template interp<SHARED>(win + i[r] * kE, p, conc, r, r + 1);
+    return;
+  }
+  int i0, iL;
+  const int top = 1 << (31 - __clz(n_int));
+  {
     i0 = iL = 0;
     for (int step = top; step > 0; step >>= 1) {
       const int t0 = i0 + step, tL = iL + step;
@@ -1605,22 +1920,26 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       s_k[j] = make_int2(klo, khi);
     }
     __syncwarp();
-    // A5 producer: lanes 0..D-1 stage the entries k_lo .. k_hi of nuclides
-    // g*D .. g*D+D-1
+    // A5 producer: lane 0 stages the entries k_lo .. k_hi of nuclides
+    // g*D .. g*D+D-1 into their slots; one mbarrier per group (two groups in
+    // flight), its transaction count raised per copy before the copy
     auto issue_group = [&](int g) {
-      const int j = g * D + lane;
-      if (lane < D && j < nn) {
-        const int slot = j % S;
-        const int2 kk = s_k[j];
-        const int32_t w = kk.y - kk.x + 1;
-        if (w <= W) {
-          const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
-          mbar_arrive_expect_tx(&s_bar[slot], static_cast<uint32_t>(w) * kEntry);
-          bulk_copy_g2s(s_win + slot * W * kE, src, static_cast<uint32_t>(w) * kEntry,
-                        &s_bar[slot]);
-        } else {
-          mbar_arrive_expect_tx(&s_bar[slot], 0u);  // read in place from global memory
+      if (lane == 0 && g * D < nn) {
+        uint64_t* bar = &s_bar[g & 1];
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+          const int j = g * D + d;
+          if (j < nn) {
+            const int2 kk = s_k[j];
+            const uint32_t bytes = static_cast<uint32_t>(kk.y - kk.x + 1) * kEntry;
+            if (bytes <= static_cast<uint32_t>(W * kEntry)) {
+              const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
+              mbar_expect_tx(bar, bytes);
+              bulk_copy_g2s(s_win + (j % S) * W * kE, src, bytes, bar);
+            }
+          }
         }
+        mbar_arrive(bar);
       }
     };
     issue_group(0);
@@ -1631,12 +1950,15 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 
     for (int j = 0; j < nn; ++j) {
       const int slot = j % S;
-      if (j >= D && j % D == 0) {
-        __syncwarp();  // every lane is done with the slots of group j/D - 1
-        issue_group(j / D + 1);
+      if (j % D == 0) {
+        const int g = j / D;
+        if (g >= 1) {
+          __syncwarp();  // every lane is done with the slots of group g - 1
+          issue_group(g + 1);
+        }
+        mbar_wait(&s_bar[g & 1], (phase >> (g & 1)) & 1u);
+        phase ^= 1u << (g & 1);
       }
-      mbar_wait(&s_bar[slot], (phase >> slot) & 1u);
-      phase ^= 1u << slot;
       const double conc = row[j].conc;
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
@@ -1996,6 +2318,12 @@ static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool so
   return check ? launch_gather_v<GT, true>(g, P, st) : launch_gather_v<GT, false>(g, P, st);
 }
 
+static uint32_t part_tiles(uint64_t count) {
+  const uint64_t tlen = static_cast<uint64_t>(part_tile_chunks(count)) * kPartChunk;
+  const uint64_t t = (count + tlen - 1) / tlen;
+  return static_cast<uint32_t>(t < 1 ? 1 : t);
+}
+
 template <int GT>
 static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                                 cudaStream_t st) {
@@ -2042,7 +2370,34 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
                  (!(a.flags & XS_FLAG_F32) && variant != 0 && variant < 9)) ? 1 : 0;
   P.tmp = ws.tmp;
   P.mat8 = ws.mat8;
-  if (binned) {
+  const bool f32 = (a.flags & XS_FLAG_F32) != 0;
+  const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28);
+  if (binned && staged && !g.legacy_sort) {
+    // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
+    // positions when per-lookup results are written) in sorted order
+    P.need_gidx = 0;
+    P.cbits = 6;  // 64 coarse energy bins per material
+    const int nkeys = (g.n_mats + 1) << P.cbits;
+    const uint32_t ntiles = part_tiles(a.count);
+    const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;
+    P.bins = ws.bins;  // H [ntiles][nkeys]
+    P.key_tot = ws.bins + static_cast<size_t>(ntiles) * nkeys;
+    P.key_start = P.key_tot + nkeys;
+    const bool per_lookup = a.out.macro_xs || a.out.verification;
+    P.sp_tmp = reinterpret_cast<double*>(ws.tmp);
+    P.sidx_tmp = per_lookup ? reinterpret_cast<uint32_t*>(P.sp_tmp + a.count) : nullptr;
+    double* sp = reinterpret_cast<double*>(ws.recs);
+    P.sp = sp;
+    P.sidx = per_lookup ? reinterpret_cast<uint32_t*>(sp + a.count) : nullptr;
+    const size_t hs = static_cast<size_t>(nkeys) * 4;
+    k_part_count<GT><<<nb, kPrepThreads, hs, st>>>(P);
+    mark(1);
+    k_part_colscan<<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));
+    k_part_keyscan<<<1, 1024, 0, st>>>(P);
+    k_part_place<GT><<<nb, kPrepThreads, hs, st>>>(P);
+    k_part_fine<<<g.n_mats << P.cbits, kFineThreads, (1u << (18 - P.cbits)) * 4, st>>>(P);
+    launched(5);
+  } else if (binned) {
     P.bins = ws.bins;
     e = cudaMemsetAsync(ws.bins, 0, static_cast<size_t>(g.n_mats + 1) * kEnergyBins * 4, st);
     if (e != cudaSuccess) return e;

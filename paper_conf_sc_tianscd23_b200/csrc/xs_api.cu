@@ -604,6 +604,9 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   } else if (!std::strcmp(name, "blocks_per_sm")) {
     if (value < 0 || value > 32) return fail(XS_ERR_INVALID_ARG, "blocks_per_sm in [0,32]");
     G.blocks_per_sm = static_cast<int>(value);
+  } else if (!std::strcmp(name, "legacy_sort")) {
+    if (value < 0 || value > 1) return fail(XS_ERR_INVALID_ARG, "legacy_sort is 0 or 1");
+    G.legacy_sort = static_cast<int>(value);
   } else {
     return fail(XS_ERR_INVALID_ARG, std::string("unknown parameter ") + name);
   }

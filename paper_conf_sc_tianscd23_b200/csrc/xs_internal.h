@@ -48,6 +48,7 @@ struct DeviceGrid {
   // tuning
   int unroll = 0;          // gather variant (0 = default; see launch_gather_u)
   int blocks_per_sm = 0;   // 0 = occupancy calculator
+  int legacy_sort = 0;     // 1: A2 through the global-atomic bins + permutation (comparison)
   // instrumentation (host side)
   uint64_t launches = 0;   // kernels launched by lookup calls
 };
