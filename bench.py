@@ -56,6 +56,12 @@ def parse():
                          "of the multi-rank path; ranks then share GPUs round-robin)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0,
                     help="target CPU seconds of the oracle sample")
+    ap.add_argument("--mode", default="event", choices=["event", "history"],
+                    help="event (default; the paper's XSBench -m event) or history "
+                         "(DESIGN.md R19: particles x chained lookups)")
+    ap.add_argument("--particles", type=int, default=500_000,
+                    help="history mode: particles per GPU (weak) / in total (strong)")
+    ap.add_argument("--lookups-per-particle", type=int, default=34)
     return ap.parse_args()
 
 
@@ -240,6 +246,140 @@ def run_reference(a, pre, cfg):
                     "d2h_bytes_per_step": 0},
             "wall_s": round(time.time() - t_start, 1)}
     print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------- history mode --
+def run_history(a, pre, cfg):
+    """History mode (R19): one step = all chained lookups of this
+    rank's particles (lookups_per_particle rounds of the event pipeline)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_tianscd23_b200 import dist as D
+    from paper_conf_sc_tianscd23_b200 import xs as X
+
+    rank, world, local = D.env_rank()
+    local = local % torch.cuda.device_count()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl" if a.backend == "nccl" else "gloo",
+                                **({"device_id": dev} if a.backend == "nccl" else {}))
+    Lp = a.lookups_per_particle
+    first, n = D.shard_range(rank, world, a.particles, a.scaling)
+    # each round is a batch of n independent lookups at random energies: the
+    # material-bucketed gather beats per-round energy binning there (measured:
+    # large 1.14 vs 0.27 G lookups/s), so history rounds skip A2
+    sort = False
+    t0 = time.time()
+    g = X.Grid.from_preset(a.config, device=local)
+    torch.cuda.synchronize()
+    init_s = time.time() - t0
+    stream = torch.cuda.current_stream(dev)
+    vsum = torch.zeros(2, dtype=torch.int64, device=dev)
+
+    def step():
+        vsum.zero_()
+        g.lookup_history(first, n, Lp, sort=sort, vsum=vsum)
+        if world > 1:
+            if a.backend == "nccl":
+                D.combine_vsum(vsum)
+            else:
+                vsum.copy_(D.combine_vsum(vsum.cpu()))
+
+    for _ in range(a.warmup):
+        step()
+    torch.cuda.synchronize()
+    g.timing(True)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(a.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms_local = ev0.elapsed_time(ev1)
+    tm = g.timing_read()
+    g.timing(False)
+    ms = D.max_over_ranks(ms_local, device=dev if a.backend == "nccl" else None)
+    total = (n * world if a.scaling == "weak" else a.particles) * Lp * a.steps
+    value = total / (ms / 1e3)
+    vglob = [int(x) for x in vsum.cpu()]
+    gold = golden().get(a.config, {}).get("history")
+    hash_check = None
+    if gold and world == 1 and first == 0 and n == gold["particles"] and \
+            Lp == gold["lookups_per_particle"]:
+        hash_check = vglob == [gold["sum_v"], n * Lp]
+    # whole-step roofline against HBM: every round is an unsorted-or-binned
+    # gather of n lookups; algorithmic bytes = sum over chained lookups of
+    # n_nuclides(mat) x (4 + 96) B (E[n] from the material distribution)
+    num_nucs = g.table(X.XS_TABLE_NUM_NUCS).tolist()
+    en = sum(p * k for p, k in zip(MAT_PROB, num_nucs))
+    balg = en * 100 + (8 * math.ceil(math.log2(max(2, g.info.n_union - 1)))
+                       if pre["grid_type"] == "unionized" else 0)
+    peak, peak_src = measured_peaks()
+    achieved = balg * value / world / 1e9
+    line = {"metric": "XS lookups/sec", "mode": "history", "value": value,
+            "unit": "lookups/s", "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+            "ms_per_step": ms / a.steps, "higher_is_better": True, "scaling": a.scaling,
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": dict(cfg, mode="history", particles_per_gpu=n,
+                           lookups_per_particle=Lp,
+                           sort="material buckets per round (no energy binning)"),
+            "roofline": {"bound": "hbm", "kernel": "whole step (lookups_per_particle rounds)",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "note": f"algorithmic bytes per chained lookup = {balg:.0f} "
+                                 "(E[n] x (4 + 96) B + unionized search probes)"},
+            "gpu_launches": int(tm["kernel_launches"]),
+            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
+            "clocks": clk.summary()}
+    # e2e: the public call from a host program (nothing to upload: particles
+    # are generated on the device), vsum read back every step
+    vs_h = torch.zeros(2, dtype=torch.int64).pin_memory()
+    t0 = time.perf_counter()
+    for _ in range(a.e2e_steps):
+        step()
+        vs_h.copy_(vsum)
+    dt = time.perf_counter() - t0
+    dt = D.max_over_ranks(dt, device=dev if a.backend == "nccl" else None)
+    line["e2e"] = {"value": (n * world if a.scaling == "weak" else a.particles) * Lp *
+                   a.e2e_steps / dt, "unit": "lookups/s", "h2d_bytes_per_step": 0,
+                   "d2h_bytes_per_step": 16,
+                   "api": "xs_lookup_history + vsum D2H, wall clock", "steps": a.e2e_steps}
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        import oracle
+        cores = os.cpu_count() or 1
+        o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"],
+                                    conc_seed=1070 * 1070, material_rule=pre["material_rule"],
+                                    hash_bins=pre.get("hash_bins", 0), nthreads=cores)
+        mode = ORACLE_MODE[pre["grid_type"]]
+        pilot = 500
+        t0 = time.perf_counter()
+        o.run_history(0, pilot, Lp, mode=mode, nthreads=cores)
+        rate = pilot / max(time.perf_counter() - t0, 1e-6)
+        m = int(min(n, max(pilot, rate * a.cpu_seconds)))
+        t0 = time.perf_counter()
+        o.run_history(0, m, Lp, mode=mode, nthreads=cores)
+        dt = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": m * Lp / dt, "unit": "lookups/s", "cores": cores,
+                                "kind": "oracle",
+                                "sample": f"particles [0, {m}) x {Lp} chained lookups, oracle "
+                                          f"route '{pre['grid_type']}', {cores} threads, "
+                                          f"{dt:.1f} s", "cpu": cpu_info()}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
     return 0
 
 
@@ -437,6 +577,8 @@ def main():
            "parallelism": f"dp{a.gpus} (lookup shards, grid replicated)"}
     if a.impl == "reference":
         return run_reference(a, pre, cfg)
+    if a.mode == "history":
+        return run_history(a, pre, cfg)
     return run_ours(a, pre, cfg)
 
 

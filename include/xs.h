@@ -203,6 +203,27 @@ xs_status xs_lookup_explicit(xs_grid* g, const double* energy, const int32_t* ma
                              uint64_t count, uint32_t flags, const xs_outputs* out,
                              void* workspace, size_t workspace_bytes, void* cuda_stream);
 
+/* History mode (XSBench "-m history"; R19; SURVEY.md §8(f)
+ * NEXT-3 — the paper runs the event driver).  Particles
+ * q in [first_particle, first_particle + n_particles) each carry one stream
+ * of the lookup LCG through `lookups` chained lookups: s = LCG^(10 lookups q)
+ * (lookup_seed), draw (p, mat); per lookup: M = A3-A8 at (p, mat), v =
+ * 1 + argmax M, skip n_forward = #{c : M_c > 1.0} draws, draw the next
+ * (p, mat).  Outputs (DEVICE pointers, any NULL except vsum): macro_xs
+ * [n][lookups][5], energy / mat / verification [n][lookups] (lookup i of
+ * particle q at q * lookups + i); grid_index must be NULL (XS_ERR_UNSUPPORTED).
+ * vsum += {sum v, n_particles * lookups}.  flags: 0 or XS_FLAG_SORT (each
+ * round's batch through A2).  Requires n_mats == 12, 1 <= lookups,
+ * n_particles < 2^32; workspace from xs_history_workspace_size (256-B
+ * aligned, caller-owned, alive until the stream passes the call).  Enqueued
+ * on the stream: lookups rounds of the event pipeline plus one state-update
+ * kernel each. */
+xs_status xs_history_workspace_size(const xs_grid* g, uint64_t n_particles, uint32_t flags,
+                                    size_t* bytes);
+xs_status xs_lookup_history(xs_grid* g, uint64_t first_particle, uint64_t n_particles,
+                            int32_t lookups, uint32_t flags, const xs_outputs* out,
+                            void* workspace, size_t workspace_bytes, void* cuda_stream);
+
 /* A8 alone on stored results: vsum += {sum_i (1 + argmax_c macro_xs[i][c]), count}
  * (device pointers). */
 xs_status xs_verify(const xs_grid* g, const double* macro_xs, uint64_t count, uint64_t* vsum,

@@ -95,6 +95,7 @@ def lib() -> C.CDLL:
                 "oracle_lookup": (None, [P, u64, C.c_int, P, P, P, P, P]),
                 "oracle_run": (u64, [P, u64, u64, C.c_int, C.c_int, P, P, P, P, P]),
                 "oracle_run_explicit": (u64, [P, P, P, u64, C.c_int, C.c_int, P, P]),
+                "oracle_run_history": (u64, [P, u64, u64, i32, C.c_int, C.c_int, P, P, P, P]),
                 "oracle_hash_finalize": (u64, [u64]),
                 "xsgen_num_nucs": (C.c_int, [i32, i32, P]),
                 "xsgen_max_num_nucs": (i32, [i32, i32]),
@@ -307,6 +308,22 @@ class Oracle:
         S = lib().oracle_run(self._h, first, count, mode, nthreads, _ptr(p), _ptr(mat), _ptr(gi),
                              _ptr(M), _ptr(v))
         return S, dict(p=p, mat=mat, grid_index=gi, M=M, v=v)
+
+    def run_history(self, first_particle: int, n_particles: int, lookups: int,
+                    mode: int = UNIONIZED, nthreads: int = 1, outputs: bool = False):
+        """History mode (R19): particles [first, first+n), `lookups`
+        chained lookups each.  Returns S or (S, dict of [n*lookups] arrays)."""
+        if not outputs:
+            return lib().oracle_run_history(self._h, first_particle, n_particles, lookups, mode,
+                                            nthreads, None, None, None, None)
+        n = n_particles * lookups
+        p = np.empty(n, np.float64)
+        mat = np.empty(n, np.int32)
+        M = np.empty((n, 5), np.float64)
+        v = np.empty(n, np.int32)
+        S = lib().oracle_run_history(self._h, first_particle, n_particles, lookups, mode,
+                                     nthreads, _ptr(p), _ptr(mat), _ptr(M), _ptr(v))
+        return S, dict(p=p, mat=mat, M=M, v=v)
 
     def run_explicit(self, p: np.ndarray, mat: np.ndarray, mode: int = UNIONIZED,
                      nthreads: int = 1):

@@ -563,3 +563,104 @@ uint64_t oracle_run_explicit(const oracle_ctx* c, const double* p, const int32_t
 }
 
 uint64_t oracle_hash_finalize(uint64_t S) { return S % 999983ULL; }
+
+/* ------------------------------------------------- history mode (R19) --
+ * XSBench's other driver ("-m history"; PAPER.md:835 names the event driver
+ * the paper runs): particle q carries one stream
+ * of the lookup LCG through `lookups` chained lookups.  In step order
+ * (R19):
+ *   s = FF(lookup_seed, 10 * lookups * q)      (2 draws per lookup + up to 5
+ *                                               extra, inside 10 per lookup)
+ *   p = draw(s); mat = pick_mat(draw(s))        (R2, R3)
+ *   for i in 0 .. lookups-1:
+ *     M = macro_xs(p, mat)                      (R5-R11)
+ *     v = verify(M); S += v                     (R12)
+ *     n = #{c : M_c > 1.0}; s = FF(s, n)        (the chain's data dependence)
+ *     p = draw(s); mat = pick_mat(draw(s))
+ * Per-lookup arrays are indexed [q * lookups + i] (relative to the first
+ * particle of the call). */
+typedef struct {
+  const oracle_ctx* c;
+  uint64_t first, begin, end;
+  int32_t lookups;
+  int mode;
+  double* p;
+  int32_t* mat;
+  double* M;
+  int32_t* v;
+  uint64_t sum;
+} hist_arg;
+
+/* one draw: s <- LCG(s), return s / 2^63 (R2) */
+static double draw(uint64_t* s) {
+  *s = oracle_lcg_step(*s);
+  return oracle_lcg_to_double(*s);
+}
+
+static void* hist_range(void* va) {
+  hist_arg* a = (hist_arg*)va;
+  uint64_t S = 0;
+  const int grid_mode = a->mode & 0xF;
+  const int f32 = (a->mode & ORACLE_F32) != 0;
+  for (uint64_t q = a->begin; q < a->end; q++) {
+    const uint64_t part = a->first + q;
+    uint64_t s = oracle_fast_forward(a->c->lookup_seed, 10ULL * (uint64_t)a->lookups * part);
+    double pe = draw(&s);
+    int32_t m = oracle_pick_mat(draw(&s));
+    for (int32_t i = 0; i < a->lookups; i++) {
+      double Ml[5];
+      int64_t gi;
+      if (f32)
+        oracle_macro_xs_f32(a->c, pe, m, grid_mode, Ml, &gi);
+      else
+        oracle_macro_xs(a->c, pe, m, grid_mode, Ml, &gi);
+      const int vv = oracle_verify(Ml);
+      S += (uint64_t)vv;
+      const uint64_t o = q * (uint64_t)a->lookups + (uint64_t)i;
+      if (a->p) a->p[o] = pe;
+      if (a->mat) a->mat[o] = m;
+      if (a->M) memcpy(a->M + 5 * o, Ml, sizeof(Ml));
+      if (a->v) a->v[o] = vv;
+      uint64_t n_forward = 0;
+      for (int c = 0; c < 5; c++)
+        if (Ml[c] > 1.0) n_forward++;
+      if (n_forward > 0) s = oracle_fast_forward(s, n_forward);
+      pe = draw(&s);
+      m = oracle_pick_mat(draw(&s));
+    }
+  }
+  a->sum = S;
+  return NULL;
+}
+
+uint64_t oracle_run_history(const oracle_ctx* c, uint64_t first_particle, uint64_t n_particles,
+                            int32_t lookups, int mode, int nthreads, double* p, int32_t* mat,
+                            double* M, int32_t* v) {
+  if (nthreads < 1) nthreads = 1;
+  if (n_particles == 0 || lookups <= 0) return 0;
+  if ((uint64_t)nthreads > n_particles) nthreads = (int)n_particles;
+  hist_arg* args = (hist_arg*)calloc((size_t)nthreads, sizeof(hist_arg));
+  pthread_t* th = (pthread_t*)calloc((size_t)nthreads, sizeof(pthread_t));
+  for (int t = 0; t < nthreads; t++) {
+    args[t].c = c;
+    args[t].first = first_particle;
+    args[t].begin = n_particles * (uint64_t)t / (uint64_t)nthreads;
+    args[t].end = n_particles * (uint64_t)(t + 1) / (uint64_t)nthreads;
+    args[t].lookups = lookups;
+    args[t].mode = mode;
+    args[t].p = p;
+    args[t].mat = mat;
+    args[t].M = M;
+    args[t].v = v;
+    if (t > 0) pthread_create(&th[t], NULL, hist_range, &args[t]);
+  }
+  hist_range(&args[0]);
+  uint64_t S = args[0].sum;
+  for (int t = 1; t < nthreads; t++) {
+    pthread_join(th[t], NULL);
+    S += args[t].sum;
+  }
+  free(args);
+  free(th);
+  return S;
+}

@@ -108,6 +108,14 @@ uint64_t oracle_run(const oracle_ctx* c, uint64_t first, uint64_t count, int mod
 uint64_t oracle_run_explicit(const oracle_ctx* c, const double* p, const int32_t* mat,
                              uint64_t count, int mode, int nthreads, double* M, int32_t* v);
 
+/* History mode (R19): particles
+ * [first_particle, first_particle + n_particles), each `lookups` chained
+ * lookups; returns S = sum of v.  Per-lookup arrays (NULL allowed) are
+ * indexed [q * lookups + i], q relative to first_particle. */
+uint64_t oracle_run_history(const oracle_ctx* c, uint64_t first_particle, uint64_t n_particles,
+                            int32_t lookups, int mode, int nthreads, double* p, int32_t* mat,
+                            double* M, int32_t* v);
+
 /* hash = S mod 999983, once, after the global sum (R13). */
 uint64_t oracle_hash_finalize(uint64_t S);
 

@@ -2279,8 +2279,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 23: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK, true>(g, P, st);
     case 24: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK>(g, P, st);
     case 25: return launch_gather_s3<GT, 4, 4, 6, 16, CHECK>(g, P, st);
-    case 26: return launch_gather_s3<GT, 4, 3, 6, 16, CHECK>(g, P, st);
-    case 27: return launch_gather_s3<GT, 4, 2, 6, 16, CHECK>(g, P, st);
+    case 26: return launch_gather_s3<GT, 4, 4, 6, 20, CHECK>(g, P, st);
+    case 27: return launch_gather_s3<GT, 4, 2, 6, 24, CHECK>(g, P, st);
     case 28: return launch_gather_s3<GT, 4, 4, 4, 16, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
@@ -2432,6 +2432,86 @@ cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace
     case XS_GRID_HASH: return run_lookup_t<XS_GRID_HASH>(g, a, ws, st);
     default: return run_lookup_t<XS_GRID_NUCLIDE>(g, a, ws, st);
   }
+}
+
+// ------------------------------------------------- history mode (R19) ---
+// XSBench's history driver: particle q carries one
+// LCG stream through L chained lookups; after each lookup the stream skips
+// n_forward = #{c : M_c > 1.0} draws, then draws the next energy and
+// material.  On the device the chain runs as L rounds: every round is one
+// explicit-lookup batch over all particles (A2-A8 through run_lookup: the
+// same kernels as event mode, material-bucketed), then k_hist_advance applies
+// the data dependence.  Results are those of the serial chain (each lookup
+// depends only on its own energy and material).
+__global__ void k_hist_init(uint64_t seed, uint64_t first, uint32_t n, int32_t L, uint64_t* st,
+                            double* E, int32_t* mat) {
+  for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) {
+    uint64_t s = fast_forward(seed, 10ull * static_cast<uint64_t>(L) * (first + q));
+    s = lcg_next(s);
+    E[q] = lcg_double(s);
+    s = lcg_next(s);
+    mat[q] = pick_material(lcg_double(s));
+    st[q] = s;
+  }
+}
+
+__global__ void k_hist_advance(HistoryArgs h, int32_t i) {
+  for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < h.n_particles;
+       q += gridDim.x * blockDim.x) {
+    double M[5];
+#pragma unroll
+    for (int c = 0; c < 5; ++c) M[c] = h.hist_M[static_cast<uint64_t>(q) * 5 + c];
+    const uint64_t o = static_cast<uint64_t>(q) * h.lookups + i;
+    if (h.out.macro_xs)
+      for (int c = 0; c < 5; ++c) h.out.macro_xs[o * 5 + c] = M[c];
+    if (h.out.energy) h.out.energy[o] = h.hist_energy[q];
+    if (h.out.mat) h.out.mat[o] = h.hist_mat[q];
+    if (h.out.verification) {
+      double mx = -1.0;
+      int vi = 0;
+      for (int c = 0; c < 5; ++c)
+        if (M[c] > mx) {
+          mx = M[c];
+          vi = c;
+        }
+      h.out.verification[o] = vi + 1;
+    }
+    int nf = 0;
+#pragma unroll
+    for (int c = 0; c < 5; ++c) nf += M[c] > 1.0 ? 1 : 0;
+    uint64_t s = h.hist_state[q];
+    for (int k = 0; k < nf; ++k) s = lcg_next(s);
+    s = lcg_next(s);
+    h.hist_energy[q] = lcg_double(s);
+    s = lcg_next(s);
+    h.hist_mat[q] = pick_material(lcg_double(s));
+    h.hist_state[q] = s;
+  }
+}
+
+cudaError_t run_history(const DeviceGrid& g, const HistoryArgs& h, const Workspace& ws,
+                        cudaStream_t st) {
+  const unsigned nb = grid_cap(h.n_particles, 256, g.sm_count, 8);
+  k_hist_init<<<nb, 256, 0, st>>>(g.lookup_seed, h.first_particle, h.n_particles, h.lookups,
+                                  h.hist_state, h.hist_energy, h.hist_mat);
+  if (h.launches) *h.launches += 1;
+  cudaError_t e = cudaGetLastError();
+  for (int32_t i = 0; i < h.lookups && e == cudaSuccess; ++i) {
+    LookupArgs a;
+    a.count = h.n_particles;
+    a.flags = h.flags & XS_FLAG_SORT;
+    a.in_energy = h.hist_energy;
+    a.in_mat = h.hist_mat;
+    a.out.macro_xs = h.hist_M;
+    a.out.vsum = h.out.vsum;
+    a.launches = h.launches;
+    e = run_lookup(g, a, ws, st);
+    if (e != cudaSuccess) break;
+    k_hist_advance<<<nb, 256, 0, st>>>(h, i);
+    if (h.launches) *h.launches += 1;
+    e = cudaGetLastError();
+  }
+  return e;
 }
 
 cudaError_t run_verify(const DeviceGrid& g, const double* M, uint64_t count, uint64_t* vsum,

@@ -538,6 +538,71 @@ xs_status xs_lookup_explicit(xs_grid* g, const double* energy, const int32_t* ma
                        cuda_stream);
 }
 
+// history mode (R19): event workspace for one round of n lookups
+// (flags & XS_FLAG_SORT) + per-particle state
+static size_t history_layout(uint64_t n, void* base, HistoryArgs* h) {
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off += align256(bytes);
+    return o;
+  };
+  const size_t o_s = take(n * 8), o_e = take(n * 8), o_m = take(n * 4), o_M = take(n * 40);
+  if (h) {
+    char* b = static_cast<char*>(base);
+    h->hist_state = reinterpret_cast<uint64_t*>(b + o_s);
+    h->hist_energy = reinterpret_cast<double*>(b + o_e);
+    h->hist_mat = reinterpret_cast<int32_t*>(b + o_m);
+    h->hist_M = reinterpret_cast<double*>(b + o_M);
+  }
+  return off;
+}
+
+xs_status xs_history_workspace_size(const xs_grid* g, uint64_t n_particles, uint32_t flags,
+                                    size_t* bytes) {
+  if (!g || !bytes) return fail(XS_ERR_INVALID_ARG, "NULL argument");
+  const uint32_t f = flags & XS_FLAG_SORT;
+  *bytes = workspace_layout(n_particles, f, g->d.n_mats, nullptr, nullptr) +
+           history_layout(n_particles, nullptr, nullptr);
+  return XS_OK;
+}
+
+xs_status xs_lookup_history(xs_grid* g, uint64_t first_particle, uint64_t n_particles,
+                            int32_t lookups, uint32_t flags, const xs_outputs* out,
+                            void* workspace, size_t workspace_bytes, void* cuda_stream) {
+  if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
+  if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
+  if (out->grid_index)
+    return fail(XS_ERR_UNSUPPORTED, "history mode does not report grid indices");
+  if (flags & ~XS_FLAG_SORT) return fail(XS_ERR_INVALID_ARG, "history mode takes XS_FLAG_SORT only");
+  if (lookups < 1) return fail(XS_ERR_INVALID_ARG, "lookups per particle must be >= 1");
+  if (n_particles >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "n_particles must be < 2^32");
+  if (g->d.n_mats != XSGEN_N_MATS)
+    return fail(XS_ERR_UNSUPPORTED, "history mode samples the 12 XSBench materials");
+  if (n_particles == 0) return XS_OK;
+  size_t need = 0;
+  xs_history_workspace_size(g, n_particles, flags, &need);
+  if (!workspace || workspace_bytes < need)
+    return fail(XS_ERR_INVALID_ARG, "workspace too small: need " + std::to_string(need) + " bytes");
+  if (reinterpret_cast<uintptr_t>(workspace) & 255)
+    return fail(XS_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
+  DeviceGuard guard(g->d.device);
+  if (!guard.ok) return fail(XS_ERR_CUDA, "cudaSetDevice failed");
+  Workspace ws;
+  const size_t wbytes = workspace_layout(n_particles, flags, g->d.n_mats, workspace, &ws);
+  HistoryArgs h;
+  history_layout(n_particles, static_cast<char*>(workspace) + wbytes, &h);
+  h.first_particle = first_particle;
+  h.n_particles = static_cast<uint32_t>(n_particles);
+  h.lookups = lookups;
+  h.flags = flags;
+  h.out = *out;
+  h.launches = &g->d.launches;
+  const cudaError_t e = run_history(g->d, h, ws, static_cast<cudaStream_t>(cuda_stream));
+  if (e != cudaSuccess) return fail(XS_ERR_CUDA, "history launch", e);
+  return XS_OK;
+}
+
 xs_status xs_verify(const xs_grid* g, const double* macro_xs, uint64_t count, uint64_t* vsum,
                     void* cuda_stream) {
   if (!g || !vsum || (count && !macro_xs)) return fail(XS_ERR_INVALID_ARG, "NULL argument");

@@ -94,6 +94,22 @@ cudaError_t init_constants();
 // lookup.cu
 cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                        cudaStream_t st);
+// history mode (R19): `lookups` rounds of explicit lookups over
+// the particle population, the per-particle stream state in hist_* arrays
+struct HistoryArgs {
+  uint64_t first_particle = 0;
+  uint32_t n_particles = 0;
+  int32_t lookups = 0;
+  uint32_t flags = 0;                  // XS_FLAG_SORT only
+  xs_outputs out{};                    // per-lookup arrays [n][lookups], vsum
+  uint64_t* hist_state = nullptr;      // [n] LCG state after the last draw
+  double* hist_energy = nullptr;       // [n] energy of the particle's next lookup
+  int32_t* hist_mat = nullptr;         // [n] its material
+  double* hist_M = nullptr;            // [n][5] macroscopic XS of the current round
+  uint64_t* launches = nullptr;
+};
+cudaError_t run_history(const DeviceGrid& g, const HistoryArgs& h, const Workspace& ws,
+                        cudaStream_t st);
 cudaError_t run_verify(const DeviceGrid& g, const double* M, uint64_t count, uint64_t* vsum,
                        cudaStream_t st);
 cudaError_t run_nuclide_index(const DeviceGrid& g, const double* energy, const int32_t* nuc,

@@ -76,7 +76,8 @@ class xs_outputs(C.Structure):
 EXPORTS = ["xs_abi_version", "xs_init_grid", "xs_init_grid_data", "xs_grid_get_info",
            "xs_workspace_size", "xs_lookup_batch", "xs_lookup_explicit", "xs_verify",
            "xs_nuclide_index", "xs_get_table", "xs_set_param", "xs_hash_finalize",
-           "xs_free_grid", "xs_last_error", "xs_timing_enable", "xs_timing_read"]
+           "xs_free_grid", "xs_last_error", "xs_timing_enable", "xs_timing_read",
+           "xs_history_workspace_size", "xs_lookup_history"]
 
 
 def _load() -> C.CDLL:
@@ -104,6 +105,9 @@ def _load() -> C.CDLL:
         "xs_last_error": (C.c_char_p, []),
         "xs_timing_enable": (st, [P, C.c_int]),
         "xs_timing_read": (st, [P, C.POINTER(xs_timing)]),
+        "xs_history_workspace_size": (st, [P, u64, u32, C.POINTER(C.c_size_t)]),
+        "xs_lookup_history": (st, [P, u64, u64, i32, u32, C.POINTER(xs_outputs), P, C.c_size_t,
+                                   P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -160,6 +164,18 @@ def xs_lookup_explicit(g, energy, mat, count, flags, out: xs_outputs, workspace,
                        stream):
     _check(lib.xs_lookup_explicit(g, energy, mat, count, flags, C.byref(out), workspace,
                                   ws_bytes, stream))
+
+
+def xs_history_workspace_size(g: int, n_particles: int, flags: int) -> int:
+    n = C.c_size_t()
+    _check(lib.xs_history_workspace_size(g, n_particles, flags, C.byref(n)))
+    return n.value
+
+
+def xs_lookup_history(g, first_particle, n_particles, lookups, flags, out: xs_outputs, workspace,
+                      ws_bytes, stream):
+    _check(lib.xs_lookup_history(g, first_particle, n_particles, lookups, flags, C.byref(out),
+                                 workspace, ws_bytes, stream))
 
 
 def xs_verify(g, macro_xs, count, vsum, stream):
@@ -339,6 +355,24 @@ class Grid:
         st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
         xs_lookup_explicit(self._h, energy.data_ptr(), mat.data_ptr(), count, flags, o,
                            ws.data_ptr(), ws.numel(), st)
+        return vsum, res
+
+    def lookup_history(self, first_particle: int, n_particles: int, lookups: int = 34,
+                       sort: bool = False, want=(), vsum=None, stream=None):
+        """History mode (R19): n_particles x lookups chained lookups.
+        Per-lookup outputs in `want` (macro_xs, energy, mat, verification) are
+        [n_particles * lookups] (lookup i of particle q at q * lookups + i)."""
+        import torch
+        flags = XS_FLAG_SORT if sort else 0
+        if vsum is None:
+            vsum = torch.zeros(2, dtype=torch.int64, device=self.device)
+        o, res = self._outputs(n_particles * lookups, want, vsum)
+        n = xs_history_workspace_size(self._h, n_particles, flags)
+        if self._ws is None or self._ws.numel() < n:
+            self._ws = torch.empty(max(n, 256), dtype=torch.uint8, device=self.device)
+        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
+        xs_lookup_history(self._h, first_particle, n_particles, lookups, flags, o,
+                          self._ws.data_ptr(), self._ws.numel(), st)
         return vsum, res
 
     def verify(self, macro_xs, vsum=None):

@@ -27,6 +27,8 @@ CONFIGS = {
     "xl": dict(I=355, N=238847, rule=0, L=170_000_000, bins=131072),
 }
 CONC_SEED = 1070 * 1070
+HIST_PARTICLES, HIST_LOOKUPS = 500_000, 34   # XSBench history-mode defaults (R19)
+HIST_PARTICLES_TINY = 3_000
 
 
 def fnv1a(buf: bytes) -> str:
@@ -42,6 +44,9 @@ def main():
     ap.add_argument("--configs", default="tiny,small,large,large-hash,xl")
     ap.add_argument("--threads", type=int, default=os.cpu_count())
     ap.add_argument("--out", default=os.path.join(ROOT, "tests", "golden", "oracle_hashes.json"))
+    ap.add_argument("--history-only", action="store_true",
+                    help="only add the history-mode sums (R19: 500,000 particles x 34 "
+                         "lookups, XSBench's history defaults) to existing entries")
     ap.add_argument("--f32-only", action="store_true",
                     help="only add the fp32-variant sums (R18) to existing entries")
     a = ap.parse_args()
@@ -56,6 +61,16 @@ def main():
                                     material_rule=c["rule"], lookup_seed=1070,
                                     hash_bins=c["bins"], nthreads=a.threads)
         t1 = time.time()
+        if a.history_only:
+            P, L = (HIST_PARTICLES_TINY, 34) if name == "tiny" else (HIST_PARTICLES, HIST_LOOKUPS)
+            Sh = o.run_history(0, P, L, mode=oracle.HASH, nthreads=a.threads)
+            out[name]["history"] = dict(particles=P, lookups_per_particle=L, sum_v=int(Sh),
+                                        hash=int(oracle.hash_finalize(Sh)))
+            print(name, "history", P, L, Sh, flush=True)
+            del o
+            with open(a.out, "w") as f:
+                json.dump(out, f, indent=1, sort_keys=True)
+            continue
         if a.f32_only:
             S32 = o.run(0, c["L"], mode=oracle.HASH | oracle.F32, nthreads=a.threads)
             out[name]["sum_v_f32"] = int(S32)
