@@ -694,19 +694,45 @@ __global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
   }
 }
 
+// k_part_place: A1 again, tile by tile.  Every lookup of the tile first goes
+// to its rank inside the tile's coarse-key order in shared memory (the tile's
+// per-key counts are the differences of the scanned H rows), then the tile
+// leaves as runs of consecutive positions (coalesced stores).
 template <int GT>
 __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
-  extern __shared__ uint32_t s_cur[];  // [nkeys]
+  extern __shared__ __align__(16) unsigned char smem_pl[];
   const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int nvalid = P.n_mats << P.cbits;
   const uint32_t tchunks = part_tile_chunks(P.count);
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
+  uint32_t* s_ls = reinterpret_cast<uint32_t*>(smem_pl);   // [nkeys + 1] local starts
+  uint32_t* s_lc = s_ls + nkeys + 1;                       // [nkeys] local cursors
+  uint32_t* s_gb = s_lc + nkeys;                           // [nkeys] global bases
+  double* s_p = reinterpret_cast<double*>(smem_pl + ((3 * static_cast<size_t>(nkeys) + 1) * 4 + 15) / 16 * 16);
+  uint16_t* s_k = reinterpret_cast<uint16_t*>(s_p + tlen);
+  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_k + tlen);
   PartStream ps;
   ps.init(P);
   for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
     const uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
-    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) s_cur[t] = P.key_start[t] + row[t];
+    const uint32_t* nxt = tl + 1 < ntiles ? row + nkeys : nullptr;
+    // local exclusive scan of the tile's per-key counts (keys in order; the
+    // invalid material's keys come last)
+    const int per = (nkeys + kPrepThreads - 1) / kPrepThreads;
+    const int k0 = threadIdx.x * per, k1 = min(nkeys, k0 + per);
+    uint32_t sum = 0;
+    for (int k = k0; k < k1; ++k) sum += (nxt ? nxt[k] : P.key_tot[k]) - row[k];
+    uint32_t ex;
+    block_excl_scan_n<kPrepThreads>(sum, &ex);
+    for (int k = k0; k < k1; ++k) {
+      s_ls[k] = ex;
+      s_lc[k] = ex;
+      s_gb[k] = P.key_start[k] + row[k];
+      ex += (nxt ? nxt[k] : P.key_tot[k]) - row[k];
+    }
     __syncthreads();
+    const uint32_t nloc = s_ls[nvalid];  // valid lookups of the tile
     uint64_t sc = ps.at(P, tl * tlen);
     for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
       const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
@@ -717,11 +743,20 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
         if (!ok[it] || smp[it].mat >= P.n_mats) continue;  // invalid lookups are not gathered
-        const uint32_t pos = atomicAdd(&s_cur[part_key(P, smp[it])], 1u);
-        P.sp_tmp[pos] = smp[it].p;
+        const uint32_t key = part_key(P, smp[it]);
+        const uint32_t q = atomicAdd(&s_lc[key], 1u);
+        s_p[q] = smp[it].p;
+        s_k[q] = static_cast<uint16_t>(key);
         if (P.sidx_tmp)
-          P.sidx_tmp[pos] = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
+          s_i[q] = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
       }
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < nloc; i += kPrepThreads) {
+      const uint32_t k = s_k[i];
+      const uint32_t d = s_gb[k] + (i - s_ls[k]);
+      P.sp_tmp[d] = s_p[i];
+      if (P.sidx_tmp) P.sidx_tmp[d] = s_i[i];
     }
     __syncthreads();
   }
@@ -2372,7 +2407,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28);
-  if (binned && staged && !g.legacy_sort) {
+  if (binned && staged && !g.legacy_sort &&
+      part_tile_chunks(a.count) <= 12) {  // k_part_place stages a tile in shared memory
     // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
     // positions when per-lookup results are written) in sorted order
     P.need_gidx = 0;
@@ -2394,7 +2430,15 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     mark(1);
     k_part_colscan<<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));
     k_part_keyscan<<<1, 1024, 0, st>>>(P);
-    k_part_place<GT><<<nb, kPrepThreads, hs, st>>>(P);
+    {
+      const size_t tlen = static_cast<size_t>(part_tile_chunks(a.count)) * kPartChunk;
+      const size_t pl_smem = ((3 * static_cast<size_t>(nkeys) + 1) * 4 + 15) / 16 * 16 +
+                             tlen * (per_lookup ? 14 : 10);
+      e = cudaFuncSetAttribute(k_part_place<GT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               static_cast<int>(pl_smem));
+      if (e != cudaSuccess) return e;
+      k_part_place<GT><<<nb, kPrepThreads, pl_smem, st>>>(P);
+    }
     k_part_fine<<<g.n_mats << P.cbits, kFineThreads, (1u << (18 - P.cbits)) * 4, st>>>(P);
     launched(5);
   } else if (binned) {
