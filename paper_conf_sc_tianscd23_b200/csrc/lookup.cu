@@ -762,42 +762,95 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
   }
 }
 
-// one block per coarse key of a valid material: counting sort of the
-// segment by the fine key (the low 18 - cbits bits of the energy bin)
-constexpr int kFineThreads = 1024;
+// k_part_fine: one block per coarse key of a valid material: counting sort
+// of its segment by the fine key (the low 18 - cbits bits of the energy
+// bin).  The histogram is scanned once; the output is then produced in
+// windows of consecutive fine bins holding at most kFineCap lookups: each
+// window re-reads the segment (L2-resident after the first pass), places its
+// lookups in shared memory and stores the window as one coalesced run.
+constexpr int kFineThreads = 1024, kFineCap = 12288, kFineBinsMax = 4096;
 __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
-  extern __shared__ uint32_t s_f[];  // [nf]
+  extern __shared__ __align__(16) unsigned char smem_fine[];
+  uint32_t* s_st = reinterpret_cast<uint32_t*>(smem_fine);            // [nf + 1] bin starts
+  uint32_t* s_cu = s_st + kFineBinsMax + 1;                            // [nf] cursors
+  double* s_p = reinterpret_cast<double*>(s_cu + kFineBinsMax + 3);    // [kFineCap]
+  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_p + kFineCap);         // [kFineCap]
+  __shared__ uint32_t s_win[2];
   const int key = blockIdx.x;
   const uint32_t s = P.key_start[key], n = P.key_tot[key];
   if (n == 0) return;
   const int fb = 18 - P.cbits;
   const uint32_t nf = 1u << fb, fmask = nf - 1u;
-  for (uint32_t t = threadIdx.x; t < nf; t += blockDim.x) s_f[t] = 0;
+  const int t = threadIdx.x;
+  for (uint32_t f = t; f < nf; f += kFineThreads) s_cu[f] = 0;
   __syncthreads();
   const double* src = P.sp_tmp + s;
-  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&s_f[energy_bin(src[i]) & fmask], 1u);
+  const uint32_t* isrc = P.sidx_tmp ? P.sidx_tmp + s : nullptr;
+  for (uint32_t i = t; i < n; i += kFineThreads) atomicAdd(&s_cu[energy_bin(src[i]) & fmask], 1u);
   __syncthreads();
-  // exclusive scan of s_f: each thread a run of nf / kFineThreads bins (nf >= 64)
+  // exclusive scan -> s_st (nf / kFineThreads bins per thread)
   const uint32_t per = (nf + kFineThreads - 1) / kFineThreads;
-  const uint32_t f0 = threadIdx.x * per;
+  const uint32_t f0 = t * per;
   uint32_t sum = 0;
-  for (uint32_t f = f0; f < f0 + per && f < nf; ++f) sum += s_f[f];
+  for (uint32_t f = f0; f < f0 + per && f < nf; ++f) sum += s_cu[f];
   uint32_t ex;
   block_excl_scan_n<kFineThreads>(sum, &ex);
   for (uint32_t f = f0; f < f0 + per && f < nf; ++f) {
-    const uint32_t v = s_f[f];
-    s_f[f] = ex;
-    ex += v;
+    s_st[f] = ex;
+    ex += s_cu[f];
   }
+  if (t == 0) s_st[nf] = n;
   __syncthreads();
   double* dst = P.sp + s;
-  const uint32_t* isrc = P.sidx_tmp ? P.sidx_tmp + s : nullptr;
   uint32_t* idst = P.sidx ? P.sidx + s : nullptr;
-  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
-    const double p = src[i];
-    const uint32_t pos = atomicAdd(&s_f[energy_bin(p) & fmask], 1u);
-    dst[pos] = p;
-    if (idst) idst[pos] = isrc[i];
+  uint32_t lo = 0;  // first bin of the window
+  while (lo < nf) {
+    if (t == 0) {
+      // last bin hi with s_st[hi + 1] - s_st[lo] <= kFineCap (at least lo)
+      const uint32_t o = s_st[lo];
+      uint32_t a = lo, b = nf;  // invariant: bins [lo, a] fit
+      while (b - a > 1) {
+        const uint32_t m = (a + b) >> 1;
+        if (s_st[m + 1] - o <= static_cast<uint32_t>(kFineCap)) a = m; else b = m;
+      }
+      s_win[0] = a;
+      s_win[1] = s_st[a + 1] - o <= static_cast<uint32_t>(kFineCap) ? 1u : 0u;
+    }
+    __syncthreads();
+    const uint32_t hi = s_win[0];
+    const bool fits = s_win[1] != 0;
+    const uint32_t o = s_st[lo], wn = s_st[hi + 1] - o;
+    if (fits) {
+      for (uint32_t f = lo + t; f <= hi; f += kFineThreads) s_cu[f] = s_st[f] - o;
+      __syncthreads();
+      for (uint32_t i = t; i < n; i += kFineThreads) {
+        const double p = src[i];
+        const uint32_t f = energy_bin(p) & fmask;
+        if (f >= lo && f <= hi) {
+          const uint32_t q = atomicAdd(&s_cu[f], 1u);
+          s_p[q] = p;
+          if (idst) s_i[q] = isrc[i];
+        }
+      }
+      __syncthreads();
+      for (uint32_t i = t; i < wn; i += kFineThreads) {
+        dst[o + i] = s_p[i];
+        if (idst) idst[o + i] = s_i[i];
+      }
+    } else {  // one bin larger than the window (skewed explicit inputs): in place
+      if (t == 0) s_cu[lo] = o;
+      __syncthreads();
+      for (uint32_t i = t; i < n; i += kFineThreads) {
+        const double p = src[i];
+        if ((energy_bin(p) & fmask) == lo) {
+          const uint32_t q = atomicAdd(&s_cu[lo], 1u);
+          dst[q] = p;
+          if (idst) idst[q] = isrc[i];
+        }
+      }
+    }
+    __syncthreads();
+    lo = hi + 1;
   }
 }
 
@@ -2439,7 +2492,14 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       if (e != cudaSuccess) return e;
       k_part_place<GT><<<nb, kPrepThreads, pl_smem, st>>>(P);
     }
-    k_part_fine<<<g.n_mats << P.cbits, kFineThreads, (1u << (18 - P.cbits)) * 4, st>>>(P);
+    {
+      const size_t fine_smem = (2 * static_cast<size_t>(kFineBinsMax) + 4) * 4 +
+                               static_cast<size_t>(kFineCap) * (per_lookup ? 12 : 8);
+      e = cudaFuncSetAttribute(k_part_fine, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               static_cast<int>(fine_smem));
+      if (e != cudaSuccess) return e;
+      k_part_fine<<<g.n_mats << P.cbits, kFineThreads, fine_smem, st>>>(P);
+    }
     launched(5);
   } else if (binned) {
     P.bins = ws.bins;
