@@ -2465,7 +2465,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
     // positions when per-lookup results are written) in sorted order
     P.need_gidx = 0;
-    P.cbits = 6;  // 64 coarse energy bins per material
+    P.cbits = 7;  // 128 coarse energy bins per material
     const int nkeys = (g.n_mats + 1) << P.cbits;
     const uint32_t ntiles = part_tiles(a.count);
     const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;
