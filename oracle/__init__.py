@@ -23,7 +23,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _ROOT = os.path.dirname(_HERE)
 LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _SOURCES = [os.path.join(_HERE, "xs_oracle.c"), os.path.join(_HERE, "xs_oracle.h"),
-            os.path.join(_ROOT, "gen", "xs_gen.cpp"), os.path.join(_ROOT, "gen", "xs_gen.h")]
+            os.path.join(_ROOT, "gen", "xs_gen.cpp"), os.path.join(_ROOT, "gen", "xs_gen.h"),
+            os.path.join(_HERE, "rs_oracle.c"), os.path.join(_HERE, "rs_oracle.h"),
+            os.path.join(_ROOT, "gen", "rs_gen.cpp"), os.path.join(_ROOT, "gen", "rs_gen.h")]
 
 UNIONIZED, NUCLIDE, HASH = 0, 1, 2
 F32 = 0x10   # OR into a mode: the fp32 variant (R18)
@@ -37,15 +39,15 @@ def build(force: bool = False) -> str:
         os.path.getmtime(s) > os.path.getmtime(LIB_PATH) for s in _SOURCES)
     if not stale:
         return LIB_PATH
-    tmp_o = LIB_PATH + ".oracle.o"
-    tmp_g = LIB_PATH + ".gen.o"
+    objs = [LIB_PATH + s for s in (".oracle.o", ".gen.o", ".rs_oracle.o", ".rs_gen.o")]
     flags = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC"]
-    subprocess.check_call(["gcc", *flags, "-std=c11", "-c", _SOURCES[0], "-o", tmp_o])
-    subprocess.check_call(["g++", *flags, "-std=c++17", "-c", _SOURCES[2], "-o", tmp_g])
-    subprocess.check_call(["g++", "-shared", "-o", LIB_PATH + ".tmp", tmp_o, tmp_g, "-lpthread",
-                           "-lm"])
+    subprocess.check_call(["gcc", *flags, "-std=c11", "-c", _SOURCES[0], "-o", objs[0]])
+    subprocess.check_call(["g++", *flags, "-std=c++17", "-c", _SOURCES[2], "-o", objs[1]])
+    subprocess.check_call(["gcc", *flags, "-std=c11", "-c", _SOURCES[4], "-o", objs[2]])
+    subprocess.check_call(["g++", *flags, "-std=c++17", "-c", _SOURCES[6], "-o", objs[3]])
+    subprocess.check_call(["g++", "-shared", "-o", LIB_PATH + ".tmp", *objs, "-lpthread", "-lm"])
     os.replace(LIB_PATH + ".tmp", LIB_PATH)
-    for f in (tmp_o, tmp_g):
+    for f in objs:
         os.remove(f)
     return LIB_PATH
 
@@ -102,6 +104,36 @@ def lib() -> C.CDLL:
                 "xsgen_mats": (C.c_int, [i32, i32, i32, P]),
                 "xsgen_concs": (C.c_int, [u64, P, i32, P]),
                 "xsgen_nuclide_grid": (C.c_int, [i32, i64, u64, P, C.c_int]),
+                # RSBench oracle (rs_oracle.h, R20-R27)
+                "rs_oracle_fast_exp": (d, [d]),
+                "rs_oracle_fast_cexp": (None, [d, d, P, P]),
+                "rs_oracle_faddeeva": (None, [d, d, P, P]),
+                "rs_oracle_sigT_factors": (None, [P, d, P, P]),
+                "rs_oracle_abrarov": (None, [d, d, d, d, P, P]),
+                "rs_oracle_asymptotic": (None, [d, d, P, P]),
+                "rs_oracle_abrarov_constants": (None, [P, P, P, P]),
+                "rs_oracle_create": (P, [i32, i32, i32, i32, i32, u64, u64, i32, P]),
+                "rs_oracle_free": (None, [P]),
+                "rs_oracle_n_nuclides": (i32, [P]),
+                "rs_oracle_max_num_nucs": (i32, [P]),
+                "rs_oracle_max_poles": (i32, [P]),
+                "rs_oracle_max_windows": (i32, [P]),
+                "rs_oracle_num_nucs": (P, [P]),
+                "rs_oracle_mats": (P, [P]),
+                "rs_oracle_concs": (P, [P]),
+                "rs_oracle_n_poles": (P, [P]),
+                "rs_oracle_n_windows": (P, [P]),
+                "rs_oracle_poles": (P, [P]),
+                "rs_oracle_l_value": (P, [P]),
+                "rs_oracle_windows": (P, [P]),
+                "rs_oracle_wrange": (P, [P]),
+                "rs_oracle_k0rs": (P, [P]),
+                "rs_oracle_window": (i32, [P, i32, d]),
+                "rs_oracle_micro_xs": (None, [P, i32, d, P]),
+                "rs_oracle_macro_xs": (None, [P, d, i32, P]),
+                "rs_oracle_verify": (C.c_int, [P]),
+                "rs_oracle_lookup": (None, [P, u64, P, P, P, P]),
+                "rs_oracle_run": (u64, [P, u64, u64, C.c_int, P, P, P, P]),
             }
             for name, (res, args) in sig.items():
                 f = getattr(L, name)
@@ -334,3 +366,158 @@ class Oracle:
         S = lib().oracle_run_explicit(self._h, _ptr(p), _ptr(mat), len(p), mode, nthreads,
                                       _ptr(M), _ptr(v))
         return S, M, v
+
+
+# ------------------------------------------------------------ RSBench oracle
+def rs_fast_exp(x: float) -> float:
+    return lib().rs_oracle_fast_exp(x)
+
+
+def rs_fast_cexp(z: complex) -> complex:
+    r, i = C.c_double(), C.c_double()
+    lib().rs_oracle_fast_cexp(z.real, z.imag, C.byref(r), C.byref(i))
+    return complex(r.value, i.value)
+
+
+def rs_faddeeva(z: complex) -> complex:
+    """RSBench's fast_nuclear_W(z) (R24)."""
+    r, i = C.c_double(), C.c_double()
+    lib().rs_oracle_faddeeva(z.real, z.imag, C.byref(r), C.byref(i))
+    return complex(r.value, i.value)
+
+
+def rs_abrarov(z: complex, e: complex) -> complex:
+    """The |z| < 6 branch of fast_nuclear_W with e = e^{12 i z} supplied (R24)."""
+    r, i = C.c_double(), C.c_double()
+    lib().rs_oracle_abrarov(z.real, z.imag, e.real, e.imag, C.byref(r), C.byref(i))
+    return complex(r.value, i.value)
+
+
+def rs_abrarov_constants():
+    """(a_n, (-1)^n, (n pi)^2, tau^2/sqrt(pi)) as the oracle holds them."""
+    an, sg, dl = (np.zeros(10, np.float64) for _ in range(3))
+    pf = C.c_double()
+    lib().rs_oracle_abrarov_constants(_ptr(an), _ptr(sg), _ptr(dl), C.byref(pf))
+    return an, sg, dl, pf.value
+
+
+def rs_asymptotic(z: complex) -> complex:
+    """The |z| >= 6 branch of fast_nuclear_W (R24)."""
+    r, i = C.c_double(), C.c_double()
+    lib().rs_oracle_asymptotic(z.real, z.imag, C.byref(r), C.byref(i))
+    return complex(r.value, i.value)
+
+
+def rs_sigT_factors(k0, E: float) -> np.ndarray:
+    """The four phase factors (cos 2phi_l, -sin 2phi_l) as complex (R23)."""
+    k0 = np.ascontiguousarray(k0, np.float64)
+    fr = np.zeros(4, np.float64)
+    fi = np.zeros(4, np.float64)
+    lib().rs_oracle_sigT_factors(_ptr(k0), E, _ptr(fr), _ptr(fi))
+    return fr + 1j * fi
+
+
+class RSOracle:
+    """RSBench problem data (gen/rs_gen.h) + the serial multipole lookup
+    (oracle/rs_oracle.c, R20-R27)."""
+
+    def __init__(self, n_nuclides=355, avg_n_poles=1000, avg_n_windows=100, numL=4,
+                 material_rule=0, seed=42, lookup_seed=1070, doppler=1):
+        err = C.c_int(0)
+        self._h = lib().rs_oracle_create(n_nuclides, avg_n_poles, avg_n_windows, numL,
+                                         material_rule, seed, lookup_seed, doppler, C.byref(err))
+        if not self._h:
+            raise ValueError(f"rs_oracle_create failed (err {err.value})")
+        L = lib()
+        self.I = n_nuclides
+        self.numL = numL
+        self.doppler = doppler
+        self.max_num_nucs = L.rs_oracle_max_num_nucs(self._h)
+        self.P = L.rs_oracle_max_poles(self._h)
+        self.W = L.rs_oracle_max_windows(self._h)
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and lib is not None:
+            try:
+                lib().rs_oracle_free(h)
+            except Exception:
+                pass
+
+    def _view(self, fn, ctype, shape):
+        a = np.ctypeslib.as_array(C.cast(getattr(lib(), fn)(self._h), C.POINTER(ctype)),
+                                  shape=(int(np.prod(shape)),))
+        return a.reshape(shape)
+
+    # copies of the inputs; the writable views let pins edit the data in place
+    def num_nucs(self):
+        return self._view("rs_oracle_num_nucs", C.c_int32, (12,)).copy()
+
+    def mats(self):
+        return self._view("rs_oracle_mats", C.c_int32, (12, self.max_num_nucs)).copy()
+
+    def concs(self):
+        return self._view("rs_oracle_concs", C.c_double, (12, self.max_num_nucs)).copy()
+
+    def n_poles(self):
+        return self._view("rs_oracle_n_poles", C.c_int32, (self.I,)).copy()
+
+    def n_windows(self):
+        return self._view("rs_oracle_n_windows", C.c_int32, (self.I,)).copy()
+
+    def poles(self, writable=False):
+        v = self._view("rs_oracle_poles", C.c_double, (self.I, self.P, 8))
+        return v if writable else v.copy()
+
+    def l_value(self, writable=False):
+        v = self._view("rs_oracle_l_value", C.c_int32, (self.I, self.P))
+        return v if writable else v.copy()
+
+    def windows(self, writable=False):
+        v = self._view("rs_oracle_windows", C.c_double, (self.I, self.W, 3))
+        return v if writable else v.copy()
+
+    def wrange(self, writable=False):
+        v = self._view("rs_oracle_wrange", C.c_int32, (self.I, self.W, 2))
+        return v if writable else v.copy()
+
+    def k0rs(self, writable=False):
+        v = self._view("rs_oracle_k0rs", C.c_double, (self.I, self.numL))
+        return v if writable else v.copy()
+
+    # steps
+    def window(self, nuc: int, E: float) -> int:
+        return lib().rs_oracle_window(self._h, nuc, E)
+
+    def micro_xs(self, nuc: int, E: float) -> np.ndarray:
+        m = np.zeros(4, np.float64)
+        lib().rs_oracle_micro_xs(self._h, nuc, E, _ptr(m))
+        return m
+
+    def macro_xs(self, E: float, mat: int) -> np.ndarray:
+        M = np.zeros(4, np.float64)
+        lib().rs_oracle_macro_xs(self._h, E, mat, _ptr(M))
+        return M
+
+    @staticmethod
+    def verify(M) -> int:
+        M = np.ascontiguousarray(M, np.float64)
+        return lib().rs_oracle_verify(_ptr(M))
+
+    def lookup(self, i: int):
+        E, m, v = C.c_double(), C.c_int32(), C.c_int32()
+        M = np.zeros(4, np.float64)
+        lib().rs_oracle_lookup(self._h, i, C.byref(E), C.byref(m), _ptr(M), C.byref(v))
+        return dict(E=E.value, mat=m.value, M=M, v=v.value)
+
+    def run(self, first: int, count: int, nthreads: int = 1, outputs: bool = False):
+        """Lookups [first, first+count).  Returns S (= sum v) or (S, dict)."""
+        if not outputs:
+            return lib().rs_oracle_run(self._h, first, count, nthreads, None, None, None, None)
+        E = np.empty(count, np.float64)
+        mat = np.empty(count, np.int32)
+        M = np.empty((count, 4), np.float64)
+        v = np.empty(count, np.int32)
+        S = lib().rs_oracle_run(self._h, first, count, nthreads, _ptr(E), _ptr(mat), _ptr(M),
+                                _ptr(v))
+        return S, dict(E=E, mat=mat, M=M, v=v)
