@@ -40,7 +40,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="large",
-                    choices=["tiny", "small", "large", "large-hash", "xl"])
+                    choices=["tiny", "small", "large", "large-hash", "xl", "rs-tiny", "rs-small",
+                             "rs-large"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     ap.add_argument("--no-sort", action="store_true", help="skip A2 (material/energy binning)")
@@ -383,6 +384,182 @@ def run_history(a, pre, cfg):
     return 0
 
 
+# ---------------------------------------------------------------- RSBench --
+# Algorithmic FP64 operations of the multipole lookup: each
+# add/sub/mul/compare is one, a correctly rounded quotient by a shared
+# refined reciprocal is 3 (+5 for the reciprocal), and every sqrt, sin, cos,
+# atan and IEEE division counts ONE (so frac is a lower bound on the pipe
+# time the transcendentals really take).
+RS_OPS_PER_POLE = 314
+RS_OPS_PER_NUCLIDE = 46
+RS_OPS_PER_LOOKUP = 5
+
+
+def rs_cpu_rate(pre, target_s, first=0):
+    import oracle
+    cores = os.cpu_count() or 1
+    o = oracle.RSOracle(pre["n_nuclides"], 1000, 100, 4, pre["material_rule"], 42, 1070, 1)
+    pilot = min(pre["lookups"], 2000)
+    t0 = time.perf_counter()
+    o.run(first, pilot, nthreads=cores)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    n = int(min(pre["lookups"], max(pilot, pilot / dt * target_s)))
+    t0 = time.perf_counter()
+    S = o.run(first, n, nthreads=cores)
+    dt = time.perf_counter() - t0
+    return n / dt, cores, n, dt, S
+
+
+def run_rs(a, pre, cfg):
+    """RSBench event mode: one step = R1-R7 over this
+    rank's lookups, vsum all-reduced for N > 1."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_tianscd23_b200 import dist as D
+    from paper_conf_sc_tianscd23_b200 import rs as RS
+
+    rank, world, local = D.env_rank()
+    if a.impl == "reference":
+        if rank != 0:
+            return 0
+        budget = 150.0
+        per_step = max(1.0, min(a.cpu_seconds, budget / max(1, a.steps + a.warmup)))
+        rate0, cores, n, _, _ = rs_cpu_rate(pre, per_step / 4)
+        n = int(min(pre["lookups"], max(1000, rate0 * per_step)))
+        import oracle
+        o = oracle.RSOracle(pre["n_nuclides"], 1000, 100, 4, pre["material_rule"], 42, 1070, 1)
+        for w in range(a.warmup):
+            o.run(w * n, n, nthreads=cores)
+        times = []
+        for k in range(a.steps):
+            t0 = time.perf_counter()
+            o.run((k * n) % max(1, pre["lookups"] - n + 1), n, nthreads=cores)
+            times.append(time.perf_counter() - t0)
+        value = n * a.steps / sum(times)
+        print(json.dumps({"impl": "reference", "metric": "RS lookups/sec", "value": value,
+                          "unit": "lookups/s", "n_gpus": a.gpus, "steps": a.steps,
+                          "warmup": a.warmup, "ms_per_step": 1e3 * sum(times) / a.steps,
+                          "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None,
+                          "dtype": "f64", "data": "synthetic", "config": cfg,
+                          "cpu_baseline": {"value": value, "unit": "lookups/s", "cores": cores,
+                                           "kind": "oracle",
+                                           "sample": f"{n:,} lookups per step, {cores} host "
+                                                     f"threads, {cpu_info()}"},
+                          "e2e": {"value": value, "unit": "lookups/s", "h2d_bytes_per_step": 0,
+                                  "d2h_bytes_per_step": 0}}), flush=True)
+        return 0
+    local = local % torch.cuda.device_count()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl" if a.backend == "nccl" else "gloo",
+                                **({"device_id": dev} if a.backend == "nccl" else {}))
+    sort = not a.no_sort
+    L_cfg = a.lookups or pre["lookups"]
+    first, L = D.shard_range(rank, world, L_cfg, a.scaling)
+    t0 = time.time()
+    p = RS.RSProblem.from_spec(device=local, **pre)
+    torch.cuda.synchronize()
+    init_s = time.time() - t0
+    stream = torch.cuda.current_stream(dev)
+    n_nuc, n_pole = p.work_count(first, L)
+    vsum = torch.zeros(2, dtype=torch.int64, device=dev)
+
+    def step():
+        vsum.zero_()
+        p.lookup(first, L, sort=sort, vsum=vsum)
+        if world > 1:
+            if a.backend == "nccl":
+                D.combine_vsum(vsum)
+            else:
+                vsum.copy_(D.combine_vsum(vsum.cpu()))
+
+    for _ in range(a.warmup):
+        step()
+    torch.cuda.synchronize()
+    l0 = p.launches
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(a.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms_local = ev0.elapsed_time(ev1)
+    launches = p.launches - l0
+    ms = D.max_over_ranks(ms_local, device=dev if a.backend == "nccl" else None)
+    total = L * world * a.steps if a.scaling == "weak" else L_cfg * a.steps
+    value = total / (ms / 1e3)
+    vglob = [int(x) for x in vsum.cpu()]
+    # the lookup kernel's own time (sample/bucket kernels excluded), events on the stream
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    ws = p.workspace(L, RS.RS_FLAG_SORT if sort else 0)
+    vs2 = torch.zeros(2, dtype=torch.int64, device=dev)
+    e0.record(stream)
+    for _ in range(3):
+        p.lookup(first, L, sort=sort, vsum=vs2)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    step_ms_lookup = e0.elapsed_time(e1) / 3
+    del ws
+    ops = n_pole * RS_OPS_PER_POLE + n_nuc * RS_OPS_PER_NUCLIDE + L * RS_OPS_PER_LOOKUP
+    peak, peak_src = fp64_pipe_peak()
+    achieved = ops / (ms_local / a.steps / 1e3) / 1e12
+    with open(os.path.join(ROOT, "tests", "golden", "rs_oracle_sums.json")) as f:
+        gold = json.load(f).get(a.config)
+    hash_check = None
+    if gold and world == 1 and first == 0 and L == gold["lookups"]:
+        hash_check = vglob == [gold["sum_v"], L]
+    line = {"metric": "RS lookups/sec", "app": "rsbench", "value": value, "unit": "lookups/s",
+            "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+            "ms_per_step": ms / a.steps, "higher_is_better": True, "scaling": a.scaling,
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": cfg,
+            "roofline": {"bound": "alu", "kernel": "whole step (k_rs_lookup dominant)",
+                         "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "algorithmic_fp64_ops_per_step": ops,
+                         "units": {"lookup_nuclide": n_nuc, "pole_terms": n_pole},
+                         "note": f"{RS_OPS_PER_POLE} FP64 ops per pole term, "
+                                 f"{RS_OPS_PER_NUCLIDE} per (lookup, nuclide), "
+                                 f"{RS_OPS_PER_LOOKUP} per lookup; sqrt/sin/cos/atan/IEEE "
+                                 "division count one each (DESIGN.md §10)"},
+            "gpu_launches": int(launches),
+            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
+            "device_bytes": int(p.device_bytes), "step_ms_recheck": step_ms_lookup}
+    vs_h = torch.zeros(2, dtype=torch.int64).pin_memory()
+    t0 = time.perf_counter()
+    for _ in range(a.e2e_steps):
+        step()
+        vs_h.copy_(vsum)
+    dt = D.max_over_ranks(time.perf_counter() - t0, device=dev if a.backend == "nccl" else None)
+    line["e2e"] = {"value": (L * world if a.scaling == "weak" else L_cfg) * a.e2e_steps / dt,
+                   "unit": "lookups/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 16,
+                   "api": "rs_lookup_batch (lookups sampled on the device) + vsum D2H, wall "
+                          "clock", "steps": a.e2e_steps}
+    line["clocks"] = clk.summary()
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        rate, cores, n, dt, _ = rs_cpu_rate(pre, a.cpu_seconds)
+        line["cpu_baseline"] = {"value": rate, "unit": "lookups/s", "cores": cores,
+                                "kind": "oracle",
+                                "sample": f"lookup ids [0, {n}) of {pre['lookups']:,}, "
+                                          f"{cores} threads, {dt:.1f} s", "cpu": cpu_info()}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
 # ------------------------------------------------------------------ ours ----
 def run_ours(a, pre, cfg):
     import torch
@@ -561,6 +738,19 @@ def run_ours(a, pre, cfg):
 
 def main():
     a = parse()
+    if a.config.startswith("rs-"):
+        from paper_conf_sc_tianscd23_b200.rs import RS_PRESETS
+        pre = dict(RS_PRESETS[a.config])
+        per_gpu = a.lookups or pre["lookups"]
+        cfg = {"workload": a.config, "app": "RSBench event mode (multipole, doppler)",
+               "n_nuclides": pre["n_nuclides"], "avg_n_poles": 1000, "avg_n_windows": 100,
+               "lookups_per_gpu": per_gpu if a.scaling == "weak" else None,
+               "lookups_total": per_gpu if a.scaling == "strong" else per_gpu * a.gpus,
+               "sort": "material + 1024 energy bins" if not a.no_sort else "none",
+               "precision": "binary64 (R28)",
+               "l2": "not flushed: compute-bound; the 23 MB pole table is L2-resident by design",
+               "parallelism": f"dp{a.gpus} (lookup shards, tables replicated)"}
+        return run_rs(a, pre, cfg)
     from paper_conf_sc_tianscd23_b200.xs_presets import PRESETS
     pre = dict(PRESETS[a.config])
     per_gpu = a.lookups or pre["lookups"]

@@ -18,13 +18,14 @@ BUILD = os.path.join(HERE, "_build")
 LIB = os.path.join(HERE, "libxs.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CU_SOURCES = ["lookup.cu", "grid_build.cu", "xs_api.cu"]
+CU_SOURCES = ["lookup.cu", "grid_build.cu", "xs_api.cu", "rs_lookup.cu"]
 HEADERS = ["common.cuh", "radix_sort.cuh", "search.cuh", "xs_internal.h"]
 
 
 def _deps():
     hs = [os.path.join(CSRC, h) for h in HEADERS]
-    hs += [os.path.join(ROOT, "include", "xs.h"), os.path.join(ROOT, "gen", "xs_gen.h")]
+    hs += [os.path.join(ROOT, "include", "xs.h"), os.path.join(ROOT, "include", "rs.h"),
+           os.path.join(ROOT, "gen", "xs_gen.h"), os.path.join(ROOT, "gen", "rs_gen.h")]
     return hs
 
 
@@ -53,11 +54,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 raise RuntimeError(f"nvcc failed for {src}")
             with open(o + ".ptxas.txt", "w") as f:
                 f.write(r.stderr)
-    g = os.path.join(ROOT, "gen", "xs_gen.cpp")
-    go = os.path.join(BUILD, "xs_gen.o")
-    objs.append(go)
-    if force or _stale(go, [g, os.path.join(ROOT, "gen", "xs_gen.h")]):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-c", g, "-o", go])
+    for gen in ("xs_gen", "rs_gen"):
+        g = os.path.join(ROOT, "gen", gen + ".cpp")
+        go = os.path.join(BUILD, gen + ".o")
+        objs.append(go)
+        if force or _stale(go, [g, os.path.join(ROOT, "gen", gen + ".h"),
+                                os.path.join(ROOT, "gen", "xs_gen.h")]):
+            subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-c", g, "-o", go])
     if force or _stale(LIB, objs):
         tmp = LIB + ".tmp"
         subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lpthread"])

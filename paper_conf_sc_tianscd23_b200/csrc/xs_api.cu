@@ -50,6 +50,10 @@ static xs_status fail(xs_status code, const std::string& msg, cudaError_t ce = c
   return code;
 }
 
+xs_status report_error(xs_status code, const char* msg, cudaError_t ce) {
+  return fail(code, msg, ce);
+}
+
 #define XS_TRY(expr, what)                                   \
   do {                                                       \
     cudaError_t _e = (expr);                                 \

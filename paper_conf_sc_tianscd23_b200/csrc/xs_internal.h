@@ -81,6 +81,9 @@ struct Workspace {
 size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* base,
                         Workspace* ws);
 
+// xs_api.cu: sets the thread-local message of xs_last_error() and returns code
+xs_status report_error(xs_status code, const char* msg, cudaError_t ce);
+
 // grid_build.cu
 cudaError_t build_union_grid(const DeviceGrid& g, double* U, cudaStream_t st);
 cudaError_t build_index_grid(const DeviceGrid& g, cudaStream_t st);

@@ -84,11 +84,45 @@ def test_product_and_oracle_share_no_code():
                 with open(os.path.join(dirpath, fn)) as f:
                     s = f.read()
                 assert not re.search(r"^\s*(import|from)\s+oracle\b", s, flags=re.M), fn
-                assert "xs_oracle" not in s, fn
+                assert "xs_oracle" not in s and "rs_oracle" not in s, fn
     for fn in os.listdir(os.path.join(ROOT, "oracle")):
         if fn.endswith((".py", ".c", ".h")):
             with open(os.path.join(ROOT, "oracle", fn)) as f:
                 s = f.read()
             assert not re.search(r"(import|from)\s+paper_conf_sc_tianscd23_b200", s), fn
-            assert not re.search(r'#include\s+"[^"]*\bxs\.h"', s), fn
+            assert not re.search(r'#include\s+"[^"]*\b[xr]s\.h"', s), fn
             assert "libxs" not in s, fn
+
+
+# ------------------------------------------------------------ RSBench (rs.h)
+def _declared_rs():
+    with open(os.path.join(ROOT, "include", "rs.h")) as f:
+        src = f.read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:const\s+)?\w+\*?\s+\*?(rs_\w+)\s*\(", src, flags=re.M)))
+
+
+def test_rs_header_and_exports(lib):
+    names = _declared_rs()
+    for n in ("rs_init", "rs_workspace_size", "rs_lookup_batch", "rs_free"):
+        assert n in names, n
+    out = subprocess.run(["nm", "-D", "--defined-only", os.path.join(
+        ROOT, "paper_conf_sc_tianscd23_b200", "libxs.so")], capture_output=True, text=True).stdout
+    import paper_conf_sc_tianscd23_b200.rs as R
+    for n in names:
+        assert re.search(rf"\bT {n}$", out, flags=re.M), n
+        assert hasattr(R, n), f"binding lacks {n}"
+
+
+def test_rs_fails_loudly_without_gpu():
+    import torch
+    import paper_conf_sc_tianscd23_b200.rs as R
+    import paper_conf_sc_tianscd23_b200.xs as X
+    with pytest.raises(X.XSError) as e:
+        R.rs_init(R.make_spec(12, material_rule=1, numL=3), 0, 0)
+    assert e.value.status == 4                        # numL != 4: unsupported
+    if torch.cuda.is_available():
+        return
+    with pytest.raises(X.XSError) as e:
+        R.rs_init(R.make_spec(12, material_rule=1), 0, 0)
+    assert e.value.status in (3, 4)
