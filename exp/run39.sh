@@ -1,0 +1,1 @@
+timeout 600 python exp/rs_variants.py rs-large 0,4,5

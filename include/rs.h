@@ -104,7 +104,7 @@ xs_status rs_work_count(const rs_data* d, uint64_t first_id, uint64_t count, uin
 
 /* Tuning knob: "variant" selects the lookup kernel's launch configuration
  * (0 = 256 threads x 2 blocks/SM, default; 1 = 256 x 3; 2 = 128 x 5;
- * 3 = 128 x 4).  Results do not depend on it.  XS_ERR_INVALID_ARG for an
+ * 3 = 128 x 4; 4 = 256 x 1; 5 = 192 x 2).  Results do not depend on it.  XS_ERR_INVALID_ARG for an
  * unknown name or value. */
 xs_status rs_set_param(rs_data* d, const char* name, int64_t value);
 
