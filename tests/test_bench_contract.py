@@ -18,14 +18,14 @@ def _run(cmd, env=None):
     return lines
 
 
-def _check(line):
+def _check(line, workload="tiny"):
     d = json.loads(line)
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
               "higher_is_better", "scaling", "vs_baseline", "dtype", "data", "config",
               "cpu_baseline", "e2e", "impl"):
         assert k in d, k
     assert d["impl"] == "reference" and d["value"] > 0
-    assert d["config"]["workload"] == "tiny"
+    assert d["config"]["workload"] == workload
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0
     return d
@@ -45,3 +45,12 @@ def test_reference_arm_torchrun_two_ranks():
                   "--steps", "2", "--warmup", "1", "--cpu-seconds", "0.3"])
     assert len(lines) == 1          # rank 0 alone prints
     assert _check(lines[0])["n_gpus"] == 2
+
+
+def test_reference_arm_rsbench():
+    """--config rs-*: the reference arm times the RSBench oracle."""
+    lines = _run([sys.executable, "bench.py", "--impl", "reference", "--config", "rs-tiny",
+                  "--steps", "2", "--warmup", "1", "--cpu-seconds", "0.3"])
+    assert len(lines) == 1
+    d = _check(lines[0], "rs-tiny")
+    assert d["metric"] == "RS lookups/sec"
