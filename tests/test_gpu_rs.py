@@ -171,3 +171,25 @@ def test_rs_workspace_errors(R):
     assert e.value.status == 1
     with pytest.raises(X.XSError):
         R.rs_lookup_batch(p._h, 0, 1000, 0x80, o, None, 0, st)
+
+
+def test_rs_bench_multirank_path_on_one_gpu(R):
+    """bench.py --config rs-tiny on two ranks sharing the GPU over gloo: shards,
+    barrier, max-over-ranks and the vsum all-reduce; the global sum equals
+    the oracle's over both shards (weak scaling: ids [0, 2L))."""
+    import subprocess
+    import sys
+    root = os.path.dirname(HERE)
+    L = GOLDEN["rs-tiny"]["lookups"]
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+                        "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
+                        "29543", "bench.py", "--gpus", "2", "--backend", "gloo", "--config",
+                        "rs-tiny", "--steps", "3", "--warmup", "3", "--no-cpu-baseline"],
+                       cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["lookups_per_step"] == 2 * L
+    S = oracle_for("rs-tiny").run(0, 2 * L, nthreads=NT)
+    assert d["hash"] == S % 999983
