@@ -2412,6 +2412,16 @@ static uint32_t part_tiles(uint64_t count) {
   return static_cast<uint32_t>(t < 1 ? 1 : t);
 }
 
+constexpr int kPartCbits = 7;  // 128 coarse energy bins per material
+
+// Bytes the partitioned A2 keeps in the A2 bin area: H [ntiles][nkeys] plus
+// the key totals and starts (workspace_layout reserves the larger of this and
+// the global-atomic bin array).
+size_t part_bins_bytes(uint64_t count, int32_t n_mats) {
+  const size_t nkeys = static_cast<size_t>(n_mats + 1) << kPartCbits;
+  return (static_cast<size_t>(part_tiles(count)) * nkeys + 2 * nkeys) * 4;
+}
+
 template <int GT>
 static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                                 cudaStream_t st) {
@@ -2465,7 +2475,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
     // positions when per-lookup results are written) in sorted order
     P.need_gidx = 0;
-    P.cbits = 7;  // 128 coarse energy bins per material
+    P.cbits = kPartCbits;
     const int nkeys = (g.n_mats + 1) << P.cbits;
     const uint32_t ntiles = part_tiles(a.count);
     const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;

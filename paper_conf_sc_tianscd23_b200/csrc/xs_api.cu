@@ -90,7 +90,10 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
   size_t o_bins = 0, o_part = 0, o_perm = 0;
   if (flags & XS_FLAG_SORT) {
     o_perm = take(count * 4);
-    o_bins = take(static_cast<size_t>(n_mats + 1) * kEnergyBins * 4);
+    // the bin area serves both A2 forms: the global-atomic bins and the
+    // partitioned A2's tile histograms (whichever is larger for this count)
+    o_bins = take(std::max(static_cast<size_t>(n_mats + 1) * kEnergyBins * 4,
+                           part_bins_bytes(count, n_mats)));
     o_part = take(static_cast<size_t>(n_mats + 1) * (kEnergyBins / 4096) * 4);
   }
   if (ws) {

@@ -95,6 +95,7 @@ cudaError_t build_intervals32(const DeviceGrid& g, cudaStream_t st);
 cudaError_t init_constants();
 
 // lookup.cu
+size_t part_bins_bytes(uint64_t count, int32_t n_mats);  // partitioned A2's bin-area need
 cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                        cudaStream_t st);
 // history mode (R19): `lookups` rounds of explicit lookups over

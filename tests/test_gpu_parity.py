@@ -462,3 +462,22 @@ def test_explicit_lookups_u8_materials(X, host, sort):
     assert np.all(vg[~ok] == 0)
     assert np.array_equal(res["mat"].cpu().numpy(), m.astype(np.int32))
     assert [int(x) for x in vs.cpu()] == [int(v[ok].sum()), int(ok.sum())]
+
+
+def test_explicit_host_io_unchunked_large(X):
+    """Regression: a 17M-lookup sorted batch uploaded in one chunk.  The
+    partitioned A2's tile histograms (2076 tiles x 1664 keys) are larger than
+    the global-atomic bin array; the workspace must reserve the larger of the
+    two (they used to overflow into the staged host inputs)."""
+    g = X.Grid.from_preset("large")
+    L = GOLDEN["large"]["lookups"]
+    vs0, res = g.lookup(0, L, sort=True, want=("energy", "mat"))
+    torch.cuda.synchronize()
+    assert int(vs0[0]) == GOLDEN["large"]["sum_v"]
+    e = res["energy"].cpu().pin_memory()
+    m = res["mat"].cpu().to(torch.uint8).pin_memory()
+    g.set_param("host_chunk", L)
+    vs = torch.zeros(2, dtype=torch.int64).pin_memory()
+    g.lookup_explicit(e, m, sort=True, vsum=vs)
+    assert [int(x) for x in vs] == [GOLDEN["large"]["sum_v"], L]
+    g.close()
