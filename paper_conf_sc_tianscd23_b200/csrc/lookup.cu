@@ -765,16 +765,20 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
 // k_part_fine: one block per coarse key of a valid material: counting sort
 // of its segment by the fine key (the low 18 - cbits bits of the energy
 // bin).  The histogram is scanned once; the output is then produced in
-// windows of consecutive fine bins holding at most kFineCap lookups: each
+// windows of consecutive fine bins holding at most `cap` lookups (as many as
+// the shared memory left after the histograms holds: 24576 energies, or 16384
+// energy + position pairs when per-lookup outputs are written): each
 // window re-reads the segment (L2-resident after the first pass), places its
 // lookups in shared memory and stores the window as one coalesced run.
-constexpr int kFineThreads = 1024, kFineCap = 12288, kFineBinsMax = 4096;
+constexpr int kFineThreads = 1024, kFineBinsMax = 4096;
+constexpr int kFineCapP = 24576, kFineCapPI = 16384;  // energies / energy + position
 __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   extern __shared__ __align__(16) unsigned char smem_fine[];
   uint32_t* s_st = reinterpret_cast<uint32_t*>(smem_fine);            // [nf + 1] bin starts
   uint32_t* s_cu = s_st + kFineBinsMax + 1;                            // [nf] cursors
-  double* s_p = reinterpret_cast<double*>(s_cu + kFineBinsMax + 3);    // [kFineCap]
-  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_p + kFineCap);         // [kFineCap]
+  const uint32_t cap = P.sidx_tmp ? kFineCapPI : kFineCapP;
+  double* s_p = reinterpret_cast<double*>(s_cu + kFineBinsMax + 3);    // [cap]
+  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_p + cap);              // [cap] (positions)
   __shared__ uint32_t s_win[2];
   const int key = blockIdx.x;
   const uint32_t s = P.key_start[key], n = P.key_tot[key];
@@ -806,15 +810,15 @@ __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   uint32_t lo = 0;  // first bin of the window
   while (lo < nf) {
     if (t == 0) {
-      // last bin hi with s_st[hi + 1] - s_st[lo] <= kFineCap (at least lo)
+      // last bin hi with s_st[hi + 1] - s_st[lo] <= cap (at least lo)
       const uint32_t o = s_st[lo];
       uint32_t a = lo, b = nf;  // invariant: bins [lo, a] fit
       while (b - a > 1) {
         const uint32_t m = (a + b) >> 1;
-        if (s_st[m + 1] - o <= static_cast<uint32_t>(kFineCap)) a = m; else b = m;
+        if (s_st[m + 1] - o <= cap) a = m; else b = m;
       }
       s_win[0] = a;
-      s_win[1] = s_st[a + 1] - o <= static_cast<uint32_t>(kFineCap) ? 1u : 0u;
+      s_win[1] = s_st[a + 1] - o <= cap ? 1u : 0u;
     }
     __syncthreads();
     const uint32_t hi = s_win[0];
@@ -2504,7 +2508,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     }
     {
       const size_t fine_smem = (2 * static_cast<size_t>(kFineBinsMax) + 4) * 4 +
-                               static_cast<size_t>(kFineCap) * (per_lookup ? 12 : 8);
+                               (per_lookup ? static_cast<size_t>(kFineCapPI) * 12
+                                           : static_cast<size_t>(kFineCapP) * 8);
       e = cudaFuncSetAttribute(k_part_fine, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                static_cast<int>(fine_smem));
       if (e != cudaSuccess) return e;
