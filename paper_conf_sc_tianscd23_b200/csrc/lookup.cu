@@ -524,7 +524,9 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
 // never depend on it.
 constexpr int kPartItems = kPrepItems;
 constexpr uint32_t kPartChunk = kPrepThreads * kPartItems;  // lookups per block round
-constexpr uint32_t kPartMaxTiles = 4000;  // H [tiles][nkeys] fits the A2 bin area
+// tiles of 8 chunks up to 2^15 tiles (268M lookups; H [tiles][nkeys] is
+// 218 MB there, reserved by workspace_layout), longer tiles beyond
+constexpr uint32_t kPartMaxTiles = 1u << 15;
 
 __host__ __device__ __forceinline__ uint32_t part_tile_chunks(uint64_t count) {
   const uint64_t chunks = (count + kPartChunk - 1) / kPartChunk;

@@ -481,3 +481,17 @@ def test_explicit_host_io_unchunked_large(X):
     g.lookup_explicit(e, m, sort=True, vsum=vs)
     assert [int(x) for x in vs] == [GOLDEN["large"]["sum_v"], L]
     g.close()
+
+
+def test_sorted_batch_above_48m(X):
+    """A sorted batch of more than 48M lookups (partitioned A2 with more than
+    4000 tiles) equals the unsorted batch, per lookup and in the sum."""
+    g = X.Grid.from_preset("small")
+    L = 48_000_000 + 4_321
+    vs_s, rs_ = g.lookup(7, L, sort=True, want=("verification",))
+    vs_u, ru = g.lookup(7, L, sort=False, want=("verification",))
+    torch.cuda.synchronize()
+    assert [int(x) for x in vs_s.cpu()] == [int(x) for x in vs_u.cpu()]
+    assert int(vs_s[1]) == L
+    assert torch.equal(rs_["verification"], ru["verification"])
+    g.close()
