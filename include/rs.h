@@ -24,11 +24,13 @@
  * from xs_last_error(), device pointers owned by the caller and kept alive
  * until the stream work completes, asynchronous on `cuda_stream`, results
  * depend only on (data, global lookup id), no CPU fallback).  Precision:
- * binary64 throughout; the elementary operations keep the oracle's order
- * (no FMA contraction, correctly rounded division), sqrt is IEEE, and
- * sin/cos/atan are CUDA's (a few ulp from the host libm), so macro XS agree
- * with the CPU oracle to ~1e-13 relative rather than bit for bit
- * (R28).
+ * binary64 throughout; the Abrarov series keeps the oracle's operation
+ * order (no FMA contraction, correctly rounded division), sqrt is IEEE,
+ * e^{12iZ} and the phase factors use algebraically equal forms (angle
+ * addition with init-time pole factors, R29; no atan, R30) and
+ * sin/cos are CUDA's, so macro XS agree with the CPU oracle to ~1e-13
+ * relative rather than bit for bit (R28; the tests require <= 1e-11 of
+ * 1 + |M|); energies, materials and the verification sum are exact.
  */
 #ifndef RS_H
 #define RS_H
