@@ -89,6 +89,11 @@ struct Params {
   uint32_t* counts;
   uint32_t* cursor;
   uint32_t* task_next;  // dynamic task counter of the staged gather (zeroed per call)
+  // explicit energies: the gather is launched twice, with and without the
+  // division range checks; each copy runs only if *gate == gate_want
+  // (k_check_energies: 1 = some energy outside the exact fast-division range)
+  const uint32_t* gate;
+  uint32_t gate_want;
   LookupRec* recs;
   uint32_t* bins;   // [(n_mats + 1) * kEnergyBins] histogram -> cursors (A2)
   LookupRec* tmp;   // [count] records in batch order
@@ -128,6 +133,24 @@ __device__ __forceinline__ int32_t grid_index_of(const Params& P, double p) {
   if (GT == XS_GRID_UNIONIZED) return static_cast<int32_t>(union_search(P.U, P.NU, p));
   if (GT == XS_GRID_HASH) return hash_bin(p, P.du, P.B);
   return -1;
+}
+
+// true when this launch of a gated gather pair is the inactive one
+__device__ __forceinline__ bool gated_off(const Params& P) {
+  return P.gate != nullptr && ((*P.gate != 0u) != (P.gate_want != 0u));
+}
+
+// Explicit energies p keep the fast correctly rounded division of A6 exact
+// (no CHECK) when the grid is dyadic63 and every p is 0 or in [2^-440, 2^400]:
+// then an = E[k+1] - p is 0 or a nonzero multiple of ulp >= 2^-492 and at most
+// 2^401, inside div_in_range.  Sets *flag = 1 if any p is outside.
+__global__ void k_check_energies(const double* __restrict__ p, uint32_t n, uint32_t* flag) {
+  bool bad = false;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const double v = p[i];
+    bad |= !(v == 0.0 || (v >= 0x1p-440 && v <= 0x1p400));
+  }
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1u);
 }
 
 __device__ __forceinline__ uint32_t energy_bin(double p) {
@@ -959,6 +982,7 @@ struct RowView {
 // shared memory.
 template <int GT, int U, int MINB, bool CHECK>
 __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
+  if (gated_off(P)) return;
   static_assert(U % kG == 0, "U must be a multiple of the group size");
   constexpr int Q = U / kG;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -1165,6 +1189,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather(Params P) {
 // arithmetic useful.  R = 1 is plain thread-per-lookup.
 template <int GT, int R, int U, int MINB, bool CHECK>
 __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
+  if (gated_off(P)) return;
   constexpr int kTask = 32 * R;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
@@ -1404,6 +1429,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_t(Params P) {
 // than W records (sparse tasks) are read in place from global memory.
 template <int GT, int R, int D, int W, int NW, bool CHECK>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
+  if (gated_off(P)) return;
   constexpr int kTask = 32 * R;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
@@ -1874,6 +1900,7 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
 
 template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false, bool F32 = false>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
+  if (gated_off(P)) return;
   using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
   constexpr int kTask = 32 * R;
   constexpr int S = 2 * D;               // window slots per warp
@@ -2401,15 +2428,43 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
 // column-only grid uses the staged gather); the fp32 variant always runs
 // the staged gather.
 template <int GT>
-static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool sorted, bool f32,
-                                   cudaStream_t st) {
-  const bool check = P.in_energy != nullptr || !g.dyadic63;
+static cudaError_t launch_gather_u1(const DeviceGrid& g, const Params& P, bool sorted, bool f32,
+                                    bool check, cudaStream_t st) {
   if (f32)
     return check ? launch_gather_f32<GT, true>(g, P, st) : launch_gather_f32<GT, false>(g, P, st);
   const bool thread_kernel = sorted || (GT == XS_GRID_UNIONIZED && !g.index);
   if (thread_kernel)
     return check ? launch_gather_tv<GT, true>(g, P, st) : launch_gather_tv<GT, false>(g, P, st);
   return check ? launch_gather_v<GT, true>(g, P, st) : launch_gather_v<GT, false>(g, P, st);
+}
+
+// Generated energies (dyadic grid) never need the division range checks;
+// explicit ones are checked on the device (k_check_energies) and the gather
+// runs as a gated pair, so the unchecked kernel does the work whenever the
+// batch allows it.  Returns the number of kernels launched in *launches.
+template <int GT>
+static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool sorted, bool f32,
+                                   uint32_t* gate, cudaStream_t st, int* launches) {
+  if (!g.dyadic63) {
+    *launches = 1;
+    return launch_gather_u1<GT>(g, P, sorted, f32, true, st);
+  }
+  if (P.in_energy == nullptr || gate == nullptr) {
+    *launches = 1;
+    return launch_gather_u1<GT>(g, P, sorted, f32, false, st);
+  }
+  cudaError_t e = cudaMemsetAsync(gate, 0, sizeof(uint32_t), st);
+  if (e != cudaSuccess) return e;
+  k_check_energies<<<grid_cap(P.count, 256, g.sm_count, 8), 256, 0, st>>>(P.in_energy, P.count,
+                                                                             gate);
+  Params Q = P;
+  Q.gate = gate;
+  Q.gate_want = 0;
+  e = launch_gather_u1<GT>(g, Q, sorted, f32, false, st);
+  if (e != cudaSuccess) return e;
+  Q.gate_want = 1;
+  *launches = 3;
+  return launch_gather_u1<GT>(g, Q, sorted, f32, true, st);
 }
 
 static uint32_t part_tiles(uint64_t count) {
@@ -2540,8 +2595,9 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   }
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   mark(2);
-  e = launch_gather_u<GT>(g, P, binned, (a.flags & XS_FLAG_F32) != 0, st);
-  launched(1);
+  int nl = 0;
+  e = launch_gather_u<GT>(g, P, binned, (a.flags & XS_FLAG_F32) != 0, ws.gate, st, &nl);
+  launched(nl);
   mark(3);
   return e;
 }

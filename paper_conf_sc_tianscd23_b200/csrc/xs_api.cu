@@ -83,7 +83,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
     off += align256(bytes);
     return o;
   };
-  const size_t o_counts = take((2 * (kMaxMats + 1) + 1) * sizeof(uint32_t));
+  const size_t o_counts = take((2 * (kMaxMats + 1) + 2) * sizeof(uint32_t));
   const size_t o_recs = take(count * sizeof(LookupRec));
   const size_t o_tmp = take(count * sizeof(LookupRec));
   const size_t o_mat8 = take(count);
@@ -100,6 +100,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
     char* b = static_cast<char*>(base);
     ws->counts = reinterpret_cast<uint32_t*>(b + o_counts);
     ws->cursor = ws->counts + (kMaxMats + 1);
+    ws->gate = ws->counts + 2 * (kMaxMats + 1) + 1;  // after the task counter
     ws->recs = reinterpret_cast<LookupRec*>(b + o_recs);
     ws->bins = reinterpret_cast<uint32_t*>(b + o_bins);
     ws->partials = reinterpret_cast<uint32_t*>(b + o_part);

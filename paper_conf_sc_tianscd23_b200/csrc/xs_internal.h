@@ -76,6 +76,7 @@ struct Workspace {
   uint8_t* mat8;      // [count]
   uint32_t* partials; // A2 scan: [(n_mats + 1) * kEnergyBins / 4096]
   uint32_t* perm;     // A2: [count]
+  uint32_t* gate;     // [1] k_check_energies flag (explicit energies)
   size_t total;
 };
 size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* base,

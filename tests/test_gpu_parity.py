@@ -495,3 +495,26 @@ def test_sorted_batch_above_48m(X):
     assert int(vs_s[1]) == L
     assert torch.equal(rs_["verification"], ru["verification"])
     g.close()
+
+
+@pytest.mark.parametrize("sort", [False, True])
+def test_explicit_gate_both_kernels_agree(X, sort):
+    """Explicit energies run as a gated pair (k_check_energies): a batch of
+    safe energies takes the unchecked gather, the same batch plus one energy
+    below 2^-440 takes the range-checked one; both equal the oracle."""
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    rng = np.random.default_rng(5)
+    p = rng.random(50_000)
+    m = rng.integers(0, 12, p.size).astype(np.int32)
+    S, M, v = o.run_explicit(p, m, mode=oracle.UNIONIZED, nthreads=NT)
+    for extra in ([], [2.0 ** -450]):
+        pp = np.concatenate([p, extra])
+        mm = np.concatenate([m, np.zeros(len(extra), np.int32)])
+        vs, res = g.lookup_explicit(torch.tensor(pp, device="cuda"), torch.tensor(mm, device="cuda"),
+                                    sort=sort, want=("macro_xs",))
+        torch.cuda.synchronize()
+        assert np.array_equal(res["macro_xs"].cpu().numpy()[:p.size], M)
+        if not extra:
+            assert vs.cpu().tolist() == [S, p.size]
+    g.close()
