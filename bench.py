@@ -535,16 +535,29 @@ def run_rs(a, pre, cfg):
             "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
             "device_bytes": int(p.device_bytes), "step_ms_recheck": step_ms_lookup}
+    # e2e: the shard's (energy, material) pairs from pinned host memory through
+    # rs_lookup_explicit(RS_FLAG_HOST_IO): H2D of 9 B per lookup, the lookups,
+    # vsum back to the host, inside the timed call
+    _, r0 = p.lookup(first, L, sort=sort, want=("energy", "mat"))
+    e_host = r0["energy"].cpu().pin_memory()
+    m_host = r0["mat"].cpu().to(torch.uint8).pin_memory()
+    del r0
     vs_h = torch.zeros(2, dtype=torch.int64).pin_memory()
+    p.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)   # warm-up
+    if world > 1:
+        dist.barrier()
     t0 = time.perf_counter()
     for _ in range(a.e2e_steps):
-        step()
-        vs_h.copy_(vsum)
+        vs_h.zero_()
+        p.lookup_explicit(e_host, m_host, sort=sort, vsum=vs_h)
     dt = D.max_over_ranks(time.perf_counter() - t0, device=dev if a.backend == "nccl" else None)
     line["e2e"] = {"value": (L * world if a.scaling == "weak" else L_cfg) * a.e2e_steps / dt,
-                   "unit": "lookups/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 16,
-                   "api": "rs_lookup_batch (lookups sampled on the device) + vsum D2H, wall "
-                          "clock", "steps": a.e2e_steps}
+                   "unit": "lookups/s", "h2d_bytes_per_step": int(L * 9),
+                   "d2h_bytes_per_step": 16,
+                   "api": "rs_lookup_explicit(RS_FLAG_HOST_IO): pinned host energy (f64) + "
+                          "material (u8) in, vsum out; wall clock per call (the call "
+                          "synchronizes)", "steps": a.e2e_steps,
+                   "vsum_matches_batch": [int(x) for x in vs_h] == [int(x) for x in vsum.cpu()]}
     line["clocks"] = clk.summary()
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         rate, cores, n, dt, _ = rs_cpu_rate(pre, a.cpu_seconds)

@@ -75,6 +75,10 @@ typedef struct {
 } rs_outputs;
 
 #define RS_FLAG_SORT 0x1u     /* R2: bucket by material and energy before R3-R7 */
+#define RS_FLAG_HOST_IO 0x2u  /* rs_lookup_explicit: energy, mat and the outputs
+                                 are HOST pointers (pinned for speed); inputs
+                                 are staged in the workspace and the call
+                                 synchronizes the stream before returning */
 #define RS_FLAG_BASELINE 0x4u /* one thread per lookup in id order, no bucketing
                                  (RSBench's CUDA kernel shape; comparison only) */
 
@@ -96,6 +100,19 @@ xs_status rs_workspace_size(const rs_data* d, uint64_t count, uint32_t flags, si
 xs_status rs_lookup_batch(rs_data* d, uint64_t first_id, uint64_t count, uint32_t flags,
                           const rs_outputs* out, void* workspace, size_t workspace_bytes,
                           void* cuda_stream);
+
+/* R2-R7 for caller-given lookups: energy[count] (binary64) and mat[count]
+ * (material ids as bytes), DEVICE pointers, or HOST pointers with
+ * RS_FLAG_HOST_IO (then `out` holds host pointers too and only vsum and
+ * macro_xs may be requested: XS_ERR_UNSUPPORTED otherwise).  A lookup with
+ * mat >= 12 or an energy outside [0, 1] (R22's window rule is defined there)
+ * is skipped: not counted in vsum, macro_xs = NaN.  Results of valid lookups
+ * equal those of the sampled lookup with the same (energy, material).
+ * flags: RS_FLAG_SORT, RS_FLAG_BASELINE, RS_FLAG_HOST_IO; workspace as
+ * rs_workspace_size(count, flags).  Errors as rs_lookup_batch. */
+xs_status rs_lookup_explicit(rs_data* d, const double* energy, const uint8_t* mat, uint64_t count,
+                             uint32_t flags, const rs_outputs* out, void* workspace,
+                             size_t workspace_bytes, void* cuda_stream);
 
 /* Instrumentation (not part of a lookup): work[0] += the number of
  * (lookup, nuclide) evaluations and work[1] += the number of pole terms R5

@@ -16,7 +16,7 @@ import ctypes as C
 from . import xs as _xs
 
 RS_ABI_VERSION = 1
-RS_FLAG_SORT, RS_FLAG_BASELINE = 0x1, 0x4
+RS_FLAG_SORT, RS_FLAG_HOST_IO, RS_FLAG_BASELINE = 0x1, 0x2, 0x4
 
 # RSBench defaults (R20): 1000 poles and 100 windows per nuclide on
 # average, numL 4, doppler on, seed 42, lookup seed 1070, 10M lookups.
@@ -48,6 +48,8 @@ def _load():
         "rs_workspace_size": (C.c_int, [P, u64, u32, C.POINTER(C.c_size_t)]),
         "rs_lookup_batch": (C.c_int, [P, u64, u64, u32, C.POINTER(rs_outputs), P, C.c_size_t,
                                       P]),
+        "rs_lookup_explicit": (C.c_int, [P, P, P, u64, u32, C.POINTER(rs_outputs), P,
+                                         C.c_size_t, P]),
         "rs_work_count": (C.c_int, [P, u64, u64, P, P]),
         "rs_set_param": (C.c_int, [P, C.c_char_p, C.c_int64]),
         "rs_launch_count": (u64, [P]),
@@ -80,6 +82,11 @@ def rs_workspace_size(d: int, count: int, flags: int) -> int:
 def rs_lookup_batch(d, first_id, count, flags, out: rs_outputs, workspace, ws_bytes, stream):
     _check(lib.rs_lookup_batch(d, first_id, count, flags, C.byref(out), workspace, ws_bytes,
                                C.c_void_p(stream)))
+
+
+def rs_lookup_explicit(d, energy, mat, count, flags, out: rs_outputs, workspace, ws_bytes, stream):
+    _check(lib.rs_lookup_explicit(d, energy, mat, count, flags, C.byref(out), workspace, ws_bytes,
+                                  C.c_void_p(stream)))
 
 
 def rs_work_count(d, first_id, count, work, stream):
@@ -190,4 +197,34 @@ class RSProblem:
         ws = self.workspace(count, flags)
         st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
         rs_lookup_batch(self._h, first_id, count, flags, o, ws.data_ptr(), ws.numel(), st)
+        return vsum, res
+
+    def lookup_explicit(self, energy, mat, sort: bool = True, want=(), vsum=None, stream=None):
+        """R2-R7 for caller-given energies (float64) and materials (uint8).
+        CUDA tensors, or CPU tensors (then RS_FLAG_HOST_IO: staged copies inside
+        the call, which synchronizes; only macro_xs may be requested)."""
+        import torch
+        host = not energy.is_cuda
+        assert mat.dtype == torch.uint8 and energy.dtype == torch.float64
+        count = energy.numel()
+        flags = (RS_FLAG_SORT if sort else 0) | (RS_FLAG_HOST_IO if host else 0)
+        dev = "cpu" if host else self.device
+        if vsum is None:
+            vsum = torch.zeros(2, dtype=torch.int64, device=dev)
+        res = {}
+
+        def mk(name, shape, dt):
+            if name in want:
+                t = torch.empty(shape, dtype=dt, device=dev,
+                                pin_memory=host and torch.cuda.is_available())
+                res[name] = t
+                return t.data_ptr()
+            return None
+        o = rs_outputs(mk("macro_xs", (count, 4), torch.float64),
+                       mk("mat", (count,), torch.int32), mk("energy", (count,), torch.float64),
+                       vsum.data_ptr())
+        ws = self.workspace(count, flags)
+        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
+        rs_lookup_explicit(self._h, energy.data_ptr(), mat.data_ptr(), count, flags, o,
+                           ws.data_ptr(), ws.numel(), st)
         return vsum, res

@@ -193,3 +193,48 @@ def test_rs_bench_multirank_path_on_one_gpu(R):
     assert d["n_gpus"] == 2 and d["lookups_per_step"] == 2 * L
     S = oracle_for("rs-tiny").run(0, 2 * L, nthreads=NT)
     assert d["hash"] == S % 999983
+
+
+@pytest.mark.parametrize("sort", [True, False])
+def test_rs_explicit_equals_sampled(R, sort):
+    """rs_lookup_explicit on the (energy, material) pairs of a sampled batch
+    gives the sampled batch's results bit for bit; device and host buffers."""
+    p = problem_for(R, "rs-tiny")
+    L = 30_000
+    vs0, ref = _run(p, 0, L, sort=True)
+    e = torch.tensor(ref["energy"], device="cuda")
+    m = torch.tensor(ref["mat"].astype(np.uint8), device="cuda")
+    vs, res = p.lookup_explicit(e, m, sort=sort, want=("macro_xs", "mat", "energy"))
+    torch.cuda.synchronize()
+    assert [int(x) for x in vs.cpu()] == vs0
+    assert np.array_equal(res["macro_xs"].cpu().numpy(), ref["macro_xs"])
+    assert np.array_equal(res["mat"].cpu().numpy(), ref["mat"])
+    vh, rh = p.lookup_explicit(e.cpu().pin_memory(), m.cpu().pin_memory(), sort=sort,
+                               want=("macro_xs",))
+    assert [int(x) for x in vh] == vs0
+    assert np.array_equal(rh["macro_xs"].numpy(), ref["macro_xs"])
+
+
+def test_rs_explicit_invalid_and_oracle(R):
+    """Random explicit pairs against the oracle's macro XS; lookups outside the
+    domain (mat >= 12, E outside [0, 1], NaN) are skipped with NaN outputs."""
+    o = oracle_for("rs-tiny")
+    p = problem_for(R, "rs-tiny")
+    rng = np.random.default_rng(3)
+    E = rng.random(5000)
+    E[:4] = [0.0, 1.0, 0.5, np.nextafter(1.0, 0.0)]
+    M = rng.integers(0, 12, E.size).astype(np.uint8)
+    bad = np.zeros(E.size, bool)
+    for i, (e, m) in enumerate([(-0.1, 3), (1.5, 3), (np.nan, 0), (0.3, 12), (0.3, 255)]):
+        E[10 + i], M[10 + i] = e, m
+        bad[10 + i] = True
+    for sort in (True, False):
+        vs, res = p.lookup_explicit(torch.tensor(E, device="cuda"), torch.tensor(M, device="cuda"),
+                                    sort=sort, want=("macro_xs",))
+        torch.cuda.synchronize()
+        X = res["macro_xs"].cpu().numpy()
+        assert np.isnan(X[bad]).all()
+        ref = np.array([o.macro_xs(float(E[i]), int(M[i])) for i in np.flatnonzero(~bad)])
+        _check_close(X[~bad], ref)
+        v = np.argmax(ref, axis=1) + 1
+        assert [int(x) for x in vs.cpu()] == [int(v.sum()), int((~bad).sum())]
