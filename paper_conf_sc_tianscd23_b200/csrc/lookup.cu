@@ -2596,7 +2596,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   mark(2);
   int nl = 0;
-  e = launch_gather_u<GT>(g, P, binned, (a.flags & XS_FLAG_F32) != 0, ws.gate, st, &nl);
+  e = launch_gather_u<GT>(g, P, binned, (a.flags & XS_FLAG_F32) != 0,
+                         a.energy_sampled ? nullptr : ws.gate, st, &nl);
   launched(nl);
   mark(3);
   return e;
@@ -2678,6 +2679,7 @@ cudaError_t run_history(const DeviceGrid& g, const HistoryArgs& h, const Workspa
     a.count = h.n_particles;
     a.flags = h.flags & XS_FLAG_SORT;
     a.in_energy = h.hist_energy;
+    a.energy_sampled = true;  // LCG draws in [0, 1]: the unchecked gather is exact
     a.in_mat = h.hist_mat;
     a.out.macro_xs = h.hist_M;
     a.out.vsum = h.out.vsum;

@@ -59,6 +59,8 @@ struct LookupArgs {
   uint32_t count = 0;
   uint32_t flags = 0;
   const double* in_energy = nullptr;  // explicit mode (device)
+  bool energy_sampled = false;        // in_energy holds the library's own draws
+                                      // (history mode): no range check needed
   const int32_t* in_mat = nullptr;
   const uint8_t* in_mat8 = nullptr;   // XS_FLAG_MAT_U8 (explicit mode, device)
   xs_outputs out{};                    // device pointers
