@@ -298,3 +298,29 @@ def test_run_shards_and_threads(tiny):
     # statistics (R26): E[sigA | mat] grows with the material's concentration sum;
     # every channel is finite
     assert np.isfinite(out["M"]).all()
+
+
+def test_invalid_specs_rejected():
+    for kw in (dict(n_nuclides=0), dict(n_nuclides=100, material_rule=0), dict(numL=3),
+               dict(avg_n_poles=0), dict(avg_n_windows=0)):
+        args = dict(n_nuclides=12, avg_n_poles=1000, avg_n_windows=100, numL=4, material_rule=1)
+        args.update(kw)
+        with pytest.raises(ValueError):
+            oracle.RSOracle(**args)
+
+
+def test_more_windows_than_poles():
+    """n_windows > n_poles: windows of zero poles (space = 0) are background only."""
+    o = oracle.RSOracle(12, 5, 50, material_rule=1)
+    npol, nwin, wr = o.n_poles(), o.n_windows(), o.wrange()
+    assert (nwin > npol).any()
+    for n in range(o.I):
+        sizes = wr[n, :nwin[n], 1] - wr[n, :nwin[n], 0] + 1
+        assert sizes.sum() == npol[n] and sizes.min() >= 0
+    win = o.windows()
+    for n in range(o.I):
+        for E in (0.013, 0.5, 0.99):
+            w = o.window(n, E)
+            if wr[n, w, 1] - wr[n, w, 0] <= 0:      # at most one pole: end-exclusive loop is empty
+                T, A, F = win[n, w]
+                assert list(o.micro_xs(n, E)) == [E * T, E * A, E * F, E * T - E * A]
