@@ -238,3 +238,19 @@ def test_rs_explicit_invalid_and_oracle(R):
         _check_close(X[~bad], ref)
         v = np.argmax(ref, axis=1) + 1
         assert [int(x) for x in vs.cpu()] == [int(v.sum()), int((~bad).sum())]
+
+
+def test_rs_sparse_poles_config(R):
+    """More windows than poles (empty windows, end < start) and a non-default
+    pole count: GPU equals the oracle."""
+    o = oracle.RSOracle(12, 5, 50, 4, 1, 42, 1070, 1)
+    p = R.RSProblem.from_spec(n_nuclides=12, avg_n_poles=5, avg_n_windows=50, material_rule=1)
+    L = 20_000
+    S, ref = o.run(0, L, nthreads=NT, outputs=True)
+    for sort in (True, False):
+        vs, out = _run(p, 0, L, sort=sort)
+        assert vs == [S, L]
+        _check_close(out["macro_xs"], ref["M"])
+    n_nuc, n_pole = p.work_count(0, L)
+    assert n_nuc == int(sum(o.num_nucs()[m] for m in ref["mat"]))
+    p.close()
