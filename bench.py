@@ -385,14 +385,14 @@ def run_history(a, pre, cfg):
 
 
 # ---------------------------------------------------------------- RSBench --
-# Algorithmic FP64 operations of the multipole lookup: each
-# add/sub/mul/compare is one, a correctly rounded quotient by a shared
-# refined reciprocal is 3 (+5 for the reciprocal), and every sqrt, sin, cos,
-# atan and IEEE division counts ONE (so frac is a lower bound on the pipe
-# time the transcendentals really take).
-RS_OPS_PER_POLE = 314
-RS_OPS_PER_NUCLIDE = 46
-RS_OPS_PER_LOOKUP = 5
+# FP64 operations of the multipole lookup as the kernels evaluate it (DESIGN.md
+# §10): each add/sub/mul/fma/compare is one; a complex division by a shared
+# denominator is 3 for the reciprocal's Newton step + 3 per quotient; sqrt,
+# sin, cos and IEEE division count ONE each (so frac is a lower bound on the
+# pipe time the transcendentals really take).
+RS_OPS_PER_POLE = 271
+RS_OPS_PER_NUCLIDE = 75
+RS_OPS_PER_LOOKUP = 11
 
 
 def rs_cpu_rate(pre, target_s, first=0):
