@@ -386,12 +386,14 @@ def run_history(a, pre, cfg):
 
 # ---------------------------------------------------------------- RSBench --
 # FP64 operations of the multipole lookup as the kernels evaluate it (DESIGN.md
-# §10): each add/sub/mul/fma/compare is one; a complex division by a shared
-# denominator is 3 for the reciprocal's Newton step + 3 per quotient; sqrt,
-# sin, cos and IEEE division count ONE each (so frac is a lower bound on the
-# pipe time the transcendentals really take).
-RS_OPS_PER_POLE = 271
-RS_OPS_PER_NUCLIDE = 75
+# §10): each add/sub/mul/fma/compare instruction is one (products and sums
+# contract into FMAs, R28); a complex division by a shared denominator is 3
+# for the reciprocal's Newton step + 3 per quotient; sqrt, sin, cos and IEEE
+# division count ONE each (so frac is a lower bound on the pipe time the
+# transcendentals really take).  Per pole: the FP64 instructions of the
+# compiled pole loop (ncu source view, profiles/r01_ncu_rs_lookup_large_mix.txt).
+RS_OPS_PER_POLE = 206
+RS_OPS_PER_NUCLIDE = 68
 RS_OPS_PER_LOOKUP = 11
 
 
@@ -529,7 +531,7 @@ def run_rs(a, pre, cfg):
                          "units": {"lookup_nuclide": n_nuc, "pole_terms": n_pole},
                          "note": f"{RS_OPS_PER_POLE} FP64 ops per pole term, "
                                  f"{RS_OPS_PER_NUCLIDE} per (lookup, nuclide), "
-                                 f"{RS_OPS_PER_LOOKUP} per lookup; sqrt/sin/cos/atan/IEEE "
+                                 f"{RS_OPS_PER_LOOKUP} per lookup; sqrt/sin/cos/IEEE "
                                  "division count one each (DESIGN.md §10)"},
             "gpu_launches": int(launches),
             "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
