@@ -25,7 +25,8 @@
  * until the stream work completes, asynchronous on `cuda_stream`, results
  * depend only on (data, global lookup id), no CPU fallback).  Precision:
  * binary64 throughout; the Abrarov series keeps the oracle's operation
- * order (no FMA contraction, correctly rounded division), sqrt is IEEE,
+ * order with products and sums contracted into FMAs and divisions within
+ * ~1 ulp, sqrt is IEEE,
  * e^{12iZ} and the phase factors use algebraically equal forms (angle
  * addition with init-time pole factors, R29; no atan, R30) and
  * sin/cos are CUDA's, so macro XS agree with the CPU oracle to ~1e-13

@@ -6,10 +6,11 @@ Bars:
   * energy, material, verification v and the verification sum/hash:
     bit-exact (the argmax is taken on values that agree to ~1e-13);
   * macro XS: |M_gpu - M_oracle| <= RTOL * (1 + |M_oracle|) with
-    RTOL = 1e-11 (R28: the kernels keep the oracle's operation
-    order; only CUDA's sin/cos/atan differ from libm by a few ulp, amplified
-    at most ~1e4-fold near the removable singularities of the Abrarov
-    series).
+    RTOL = 1e-11 (R28-R30: the kernels keep the oracle's
+    operation order up to FMA contraction and ~1-ulp divisions, evaluate
+    e^{12iZ} and the phase factors in algebraically equal forms, and use
+    CUDA's sin/cos — a few ulp, amplified near the removable singularities
+    of the Abrarov series; observed max 1e-13).
 """
 import json
 import os
