@@ -393,7 +393,7 @@ def run_history(a, pre, cfg):
 # transcendentals really take).  Per pole: the FP64 instructions of the
 # compiled pole loop (ncu source view, profiles/r01_ncu_rs_lookup_large_mix.txt).
 RS_OPS_PER_POLE = 206
-RS_OPS_PER_NUCLIDE = 89
+RS_OPS_PER_NUCLIDE = 91
 RS_OPS_PER_LOOKUP = 11
 
 
