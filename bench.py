@@ -388,11 +388,12 @@ def run_history(a, pre, cfg):
 # FP64 operations of the multipole lookup as the kernels evaluate it (DESIGN.md
 # §10): each add/sub/mul/fma/compare instruction is one (products and sums
 # contract into FMAs, R28); a complex division by a shared denominator is 3
-# for the reciprocal's Newton step + 1 per quotient; sqrt, sin, cos and IEEE
+# for the reciprocal's Newton step + 1 per quotient (in the series the a_n
+# weight is folded into the reciprocal: 1 product for both quotients); sqrt, sin, cos and IEEE
 # division count ONE each (so frac is a lower bound on the pipe time the
 # transcendentals really take).  Per pole: the FP64 instructions of the
 # compiled pole loop (ncu source view, profiles/r01_ncu_rs_lookup_large_mix.txt).
-RS_OPS_PER_POLE = 162
+RS_OPS_PER_POLE = 152
 RS_OPS_PER_NUCLIDE = 91
 RS_OPS_PER_LOOKUP = 11
 
