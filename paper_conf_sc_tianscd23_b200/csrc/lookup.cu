@@ -104,6 +104,7 @@ struct Params {
                        // searches only each task's extreme energies)
   // partitioned A2 (k_part_*): H[block][key] lives in bins
   int cbits;            // coarse energy bits per material
+  int fine_direct;      // k_part_fine scatters directly above this many windows
   uint32_t* key_tot;    // [nkeys] lookups per coarse key
   uint32_t* key_start;  // [nkeys] first position of the key
   double* sp_tmp;       // [count] energies in coarse-key order
@@ -663,6 +664,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
   }
 }
 
+constexpr int kColIlp = 8;
 // H[t][key] -> exclusive prefix over tiles t (per key); key totals.  Block =
 // 32 keys x 32 slices of the tiles.
 __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
@@ -672,9 +674,18 @@ __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
   const int sl = threadIdx.y;
   const int per = (nb + 31) / 32;
   const int b0 = sl * per, b1 = min(nb, b0 + per);
+  // both passes keep kColIlp loads in flight (the rows are nkeys * 4 B apart;
+  // a dependent walk is latency-bound at XL's 20k tiles)
   uint32_t sum = 0;
   if (key < nkeys)
-    for (int b = b0; b < b1; ++b) sum += P.bins[static_cast<uint64_t>(b) * nkeys + key];
+    for (int b = b0; b < b1; b += kColIlp) {
+      uint32_t v[kColIlp];
+#pragma unroll
+      for (int u = 0; u < kColIlp; ++u)
+        v[u] = b + u < b1 ? P.bins[static_cast<uint64_t>(b + u) * nkeys + key] : 0u;
+#pragma unroll
+      for (int u = 0; u < kColIlp; ++u) sum += v[u];
+    }
   s_p[sl][threadIdx.x] = sum;
   __syncthreads();
   if (sl == 0) {
@@ -689,11 +700,16 @@ __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
   __syncthreads();
   if (key < nkeys) {
     uint32_t run = s_p[sl][threadIdx.x];
-    for (int b = b0; b < b1; ++b) {
-      uint32_t* h = P.bins + static_cast<uint64_t>(b) * nkeys + key;
-      const uint32_t v = *h;
-      *h = run;
-      run += v;
+    for (int b = b0; b < b1; b += kColIlp) {
+      uint32_t v[kColIlp];
+#pragma unroll
+      for (int u = 0; u < kColIlp; ++u)
+        v[u] = b + u < b1 ? P.bins[static_cast<uint64_t>(b + u) * nkeys + key] : 0u;
+#pragma unroll
+      for (int u = 0; u < kColIlp; ++u) {
+        if (b + u < b1) P.bins[static_cast<uint64_t>(b + u) * nkeys + key] = run;
+        run += v[u];
+      }
     }
   }
 }
@@ -795,7 +811,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
 // energy + position pairs when per-lookup outputs are written): each
 // window re-reads the segment (L2-resident after the first pass), places its
 // lookups in shared memory and stores the window as one coalesced run.
-constexpr int kFineThreads = 1024, kFineBinsMax = 4096;
+constexpr int kFineThreads = 1024, kFineBinsMax = 4096, kFineIlp = 4;
 constexpr int kFineCapP = 24576, kFineCapPI = 16384;  // energies / energy + position
 __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   extern __shared__ __align__(16) unsigned char smem_fine[];
@@ -815,7 +831,19 @@ __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   __syncthreads();
   const double* src = P.sp_tmp + s;
   const uint32_t* isrc = P.sidx_tmp ? P.sidx_tmp + s : nullptr;
-  for (uint32_t i = t; i < n; i += kFineThreads) atomicAdd(&s_cu[energy_bin(src[i]) & fmask], 1u);
+  // kFineIlp independent loads in flight per thread (one block per SM: the
+  // segment streams are bound by memory-level parallelism, not bandwidth)
+  for (uint32_t i0 = t; i0 < n; i0 += kFineIlp * kFineThreads) {
+    double pv[kFineIlp];
+#pragma unroll
+    for (int u = 0; u < kFineIlp; ++u) {
+      const uint32_t i = i0 + u * kFineThreads;
+      pv[u] = i < n ? src[i] : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < kFineIlp; ++u)
+      if (i0 + u * kFineThreads < n) atomicAdd(&s_cu[energy_bin(pv[u]) & fmask], 1u);
+  }
   __syncthreads();
   // exclusive scan -> s_st (nf / kFineThreads bins per thread)
   const uint32_t per = (nf + kFineThreads - 1) / kFineThreads;
@@ -832,6 +860,30 @@ __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   __syncthreads();
   double* dst = P.sp + s;
   uint32_t* idst = P.sidx ? P.sidx + s : nullptr;
+  if (n > static_cast<uint64_t>(P.fine_direct) * cap) {
+    // long segment (XL): one pass that scatters every energy to its bin's
+    // cursor in the output (the segment's output range stays L2-resident)
+    // instead of re-reading the segment once per window
+    for (uint32_t f = t; f < nf; f += kFineThreads) s_cu[f] = s_st[f];
+    __syncthreads();
+    for (uint32_t i0 = t; i0 < n; i0 += kFineIlp * kFineThreads) {
+      double pv[kFineIlp];
+#pragma unroll
+      for (int u = 0; u < kFineIlp; ++u) {
+        const uint32_t i = i0 + u * kFineThreads;
+        pv[u] = i < n ? src[i] : 0.0;
+      }
+#pragma unroll
+      for (int u = 0; u < kFineIlp; ++u) {
+        const uint32_t i = i0 + u * kFineThreads;
+        if (i >= n) continue;
+        const uint32_t q = atomicAdd(&s_cu[energy_bin(pv[u]) & fmask], 1u);
+        dst[q] = pv[u];
+        if (idst) idst[q] = isrc[i];
+      }
+    }
+    return;
+  }
   uint32_t lo = 0;  // first bin of the window
   while (lo < nf) {
     if (t == 0) {
@@ -852,13 +904,22 @@ __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
     if (fits) {
       for (uint32_t f = lo + t; f <= hi; f += kFineThreads) s_cu[f] = s_st[f] - o;
       __syncthreads();
-      for (uint32_t i = t; i < n; i += kFineThreads) {
-        const double p = src[i];
-        const uint32_t f = energy_bin(p) & fmask;
-        if (f >= lo && f <= hi) {
-          const uint32_t q = atomicAdd(&s_cu[f], 1u);
-          s_p[q] = p;
-          if (idst) s_i[q] = isrc[i];
+      for (uint32_t i0 = t; i0 < n; i0 += kFineIlp * kFineThreads) {
+        double pv[kFineIlp];
+#pragma unroll
+        for (int u = 0; u < kFineIlp; ++u) {
+          const uint32_t i = i0 + u * kFineThreads;
+          pv[u] = i < n ? src[i] : 0.0;
+        }
+#pragma unroll
+        for (int u = 0; u < kFineIlp; ++u) {
+          if (i0 + u * kFineThreads >= n) continue;
+          const uint32_t f = energy_bin(pv[u]) & fmask;
+          if (f >= lo && f <= hi) {
+            const uint32_t q = atomicAdd(&s_cu[f], 1u);
+            s_p[q] = pv[u];
+            if (idst) s_i[q] = isrc[i0 + u * kFineThreads];
+          }
         }
       }
       __syncthreads();
@@ -2473,13 +2534,37 @@ static uint32_t part_tiles(uint64_t count) {
   return static_cast<uint32_t>(t < 1 ? 1 : t);
 }
 
-constexpr int kPartCbits = 7;  // 128 coarse energy bins per material
+// Coarse energy bits of the partitioned A2 (2^7 keys per material).
+// A wider key (part_cbits 8, 9) shortens the segments k_part_fine sorts but
+// grows the tile histograms and k_part_place's shared memory, and measured
+// slower at every size (large 2.85 -> 2.98 ms at 8 bits, XL
+// 41.5 -> 42.1 / 42.8 ms at 8 / 9 bits).  Limits: k_part_place holds
+// three key arrays and the tile in shared memory, keys are 16 bit, and the
+// fine histogram has at most kFineBinsMax bins.
+constexpr int kPartCbits = 7, kPartCbitsMax = 9;
+
+static size_t part_place_smem(uint64_t count, int32_t n_mats, int cbits, bool per_lookup) {
+  const size_t nkeys = static_cast<size_t>(n_mats + 1) << cbits;
+  const size_t tlen = static_cast<size_t>(part_tile_chunks(count)) * kPartChunk;
+  return ((3 * nkeys + 1) * 4 + 15) / 16 * 16 + tlen * (per_lookup ? 14 : 10);
+}
+
+bool part_cbits_fit(uint64_t count, int32_t n_mats, int cbits) {
+  return cbits >= 18 - 12 && cbits <= kPartCbitsMax && (static_cast<size_t>(n_mats + 1) << cbits) <= 65536 &&
+         part_place_smem(count, n_mats, cbits, true) <= 227 * 1024;
+}
+
+static int part_cbits(uint64_t count, int32_t n_mats, int requested) {
+  return requested && part_cbits_fit(count, n_mats, requested) ? requested : kPartCbits;
+}
 
 // Bytes the partitioned A2 keeps in the A2 bin area: H [ntiles][nkeys] plus
 // the key totals and starts (workspace_layout reserves the larger of this and
-// the global-atomic bin array).
+// the global-atomic bin array), for the widest coarse key that fits.
 size_t part_bins_bytes(uint64_t count, int32_t n_mats) {
-  const size_t nkeys = static_cast<size_t>(n_mats + 1) << kPartCbits;
+  int c = kPartCbits;
+  while (c < kPartCbitsMax && part_cbits_fit(count, n_mats, c + 1)) ++c;
+  const size_t nkeys = static_cast<size_t>(n_mats + 1) << c;
   return (static_cast<size_t>(part_tiles(count)) * nkeys + 2 * nkeys) * 4;
 }
 
@@ -2536,7 +2621,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
     // positions when per-lookup results are written) in sorted order
     P.need_gidx = 0;
-    P.cbits = kPartCbits;
+    P.cbits = part_cbits(a.count, g.n_mats, g.part_cbits);  // (a request that does not fit: 7)
+    P.fine_direct = g.fine_direct;
     const int nkeys = (g.n_mats + 1) << P.cbits;
     const uint32_t ntiles = part_tiles(a.count);
     const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;
@@ -2555,9 +2641,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     k_part_colscan<<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));
     k_part_keyscan<<<1, 1024, 0, st>>>(P);
     {
-      const size_t tlen = static_cast<size_t>(part_tile_chunks(a.count)) * kPartChunk;
-      const size_t pl_smem = ((3 * static_cast<size_t>(nkeys) + 1) * 4 + 15) / 16 * 16 +
-                             tlen * (per_lookup ? 14 : 10);
+      const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup);
       e = cudaFuncSetAttribute(k_part_place<GT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                static_cast<int>(pl_smem));
       if (e != cudaSuccess) return e;

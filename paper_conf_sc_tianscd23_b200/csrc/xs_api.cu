@@ -680,6 +680,13 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   } else if (!std::strcmp(name, "legacy_sort")) {
     if (value < 0 || value > 1) return fail(XS_ERR_INVALID_ARG, "legacy_sort is 0 or 1");
     G.legacy_sort = static_cast<int>(value);
+  } else if (!std::strcmp(name, "part_cbits")) {
+    if (value != 0 && (value < 6 || value > 9))
+      return fail(XS_ERR_INVALID_ARG, "part_cbits is 0 (default) or 6-9");
+    G.part_cbits = static_cast<int>(value);
+  } else if (!std::strcmp(name, "fine_direct")) {
+    if (value < 0 || value > 1024) return fail(XS_ERR_INVALID_ARG, "fine_direct in [0,1024]");
+    G.fine_direct = static_cast<int>(value);
   } else {
     return fail(XS_ERR_INVALID_ARG, std::string("unknown parameter ") + name);
   }

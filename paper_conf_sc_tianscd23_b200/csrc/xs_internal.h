@@ -49,6 +49,8 @@ struct DeviceGrid {
   int unroll = 0;          // gather variant (0 = default; see launch_gather_u)
   int blocks_per_sm = 0;   // 0 = occupancy calculator
   int legacy_sort = 0;     // 1: A2 through the global-atomic bins + permutation (comparison)
+  int part_cbits = 0;      // partitioned A2 coarse energy bits (0 = default)
+  int fine_direct = 2;     // k_part_fine: direct scatter above this many windows
   // instrumentation (host side)
   uint64_t launches = 0;   // kernels launched by lookup calls
 };
@@ -99,6 +101,7 @@ cudaError_t init_constants();
 
 // lookup.cu
 size_t part_bins_bytes(uint64_t count, int32_t n_mats);  // partitioned A2's bin-area need
+bool part_cbits_fit(uint64_t count, int32_t n_mats, int cbits);  // shared memory / key-width limits
 cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                        cudaStream_t st);
 // history mode (R19): `lookups` rounds of explicit lookups over

@@ -518,3 +518,38 @@ def test_explicit_gate_both_kernels_agree(X, sort):
         if not extra:
             assert vs.cpu().tolist() == [S, p.size]
     g.close()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("fine_direct", [0, 2])
+@pytest.mark.parametrize("cbits", [6, 7, 8, 9])
+def test_part_cbits_tiny_parity(X, cbits, fine_direct):
+    """Every coarse fan-out of the partitioned A2 (part_cbits 6-9), with the
+    fine pass windowed or scattering directly (fine_direct 0: every segment),
+    gives the oracle's per-lookup results; the order inside the sort never
+    matters."""
+    g = X.Grid.from_preset("tiny")
+    g.set_param("part_cbits", cbits)
+    g.set_param("fine_direct", fine_direct)
+    S, ref = oracle_for("tiny").run(3, 100_000, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
+    vs, out = _full_outputs(g, 3, 100_000, sort=True)
+    _compare(out, ref)
+    assert vs == [S, 100_000]
+
+
+@pytest.mark.gpu
+def test_part_cbits_wide_above_2p26(X):
+    """A batch above 2^26 lookups sorted with the widest coarse key
+    (part_cbits 9, 53 MB more tile histograms) agrees, per lookup, with the
+    default (7)."""
+    g = X.Grid.from_preset("small")
+    L = (1 << 26) + 12_345
+    g.set_param("part_cbits", 9)
+    vs_a, ra = g.lookup(11, L, sort=True, want=("verification",))
+    g.set_param("part_cbits", 7)
+    vs_7, r7 = g.lookup(11, L, sort=True, want=("verification",))
+    torch.cuda.synchronize()
+    assert [int(x) for x in vs_a.cpu()] == [int(x) for x in vs_7.cpu()]
+    assert int(vs_a[1]) == L
+    assert torch.equal(ra["verification"], r7["verification"])
+    g.close()
