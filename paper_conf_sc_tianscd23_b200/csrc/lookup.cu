@@ -2440,9 +2440,18 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // blocks); 9-12 TMA-staged record windows (R, stages D, window W records,
   // warps per block); 17-20 TMA-staged interval-table windows (R, group
   // size D, window W entries, warps per block).  Measured best on B200 (large,
-  // large-hash, small): k_gather_s3 (4, 4, 6, 16) = variant 25.
+  // large-hash, small): k_gather_s3 (4, 4, 6, 16) = variant 25, while a
+  // task's windows stay short.  Density d = N * 128 / count (interval entries a
+  // 128-lookup task of one material spans per nuclide, up to the material's
+  // share): with long windows fewer lookups per lane win, variant 20 (2, 2, 8,
+  // 24).  Measured crossover: large/small 8M lookups (d 0.18)
+  // 1.75 vs 1.82 ms, 4M (d 0.36) 1.23 vs 1.16 ms; XL 170M (d 0.18, N 238,847,
+  // cold 9.5 GB interval table) 36.5 vs 33.5 ms gather.
   int v = g.unroll;
-  if (v == 0) v = 25;
+  if (v == 0) {
+    const double d = static_cast<double>(g.N) * 128.0 / static_cast<double>(P.count ? P.count : 1);
+    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : 25;
+  }
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
     case 2: return launch_gather_t<GT, 4, 1, 2, CHECK>(g, P, st);
