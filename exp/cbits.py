@@ -10,10 +10,12 @@ vals = [int(v) for v in sys.argv[2].split(",")]
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 5
 fds = [int(v) for v in sys.argv[4].split(",")] if len(sys.argv) > 4 else [2]
 variants = [int(v) for v in sys.argv[5].split(",")] if len(sys.argv) > 5 else [0]
+caps = [int(v) for v in os.environ.get("FINE_CAPS", "0").split(",")]
 gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")))
 g = X.Grid.from_preset(cfg)
 L = int(sys.argv[6]) if len(sys.argv) > 6 else X.PRESETS[cfg]["lookups"]
-for c, fd, var in [(c, fd, v) for c in vals for fd in fds for v in variants]:
+for c, fd, var, cap in [(c, fd, v, k) for c in vals for fd in fds for v in variants for k in caps]:
+    g.set_param("fine_cap", cap)
     g.set_param("variant", var)
     g.set_param("part_cbits", c)
     g.set_param("fine_direct", fd)
@@ -30,5 +32,5 @@ for c, fd, var in [(c, fd, v) for c in vals for fd in fds for v in variants]:
     en.record(); torch.cuda.synchronize()
     ms = st.elapsed_time(en) / reps
     t = g.timing_read(); g.timing(False); n = t["calls"] or 1
-    print(f"{cfg} cbits={c} fd={fd} v={var} {ms:8.3f} ms/step {L/ms/1e6:8.3f} G/s count {t['ms_count']/n:.3f} "
+    print(f"{cfg} cbits={c} fd={fd} v={var} cap={cap} {ms:8.3f} ms/step {L/ms/1e6:8.3f} G/s count {t['ms_count']/n:.3f} "
           f"bucket {t['ms_bucket']/n:.3f} gather {t['ms_gather']/n:.3f} hash_ok={ok}", flush=True)

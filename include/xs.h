@@ -248,7 +248,8 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
  * sort, 6-9; 0 = the default, 7; a value whose tables do not fit the batch
  * falls back to 7), "fine_direct" (the sort's fine pass scatters a coarse
  * key's segment in one pass when it exceeds this many shared-memory windows,
- * else sorts it window by window; default 2) and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in
+ * else sorts it window by window; default 2), "fine_cap" (that window in
+ * energies, 2048-24576; 0 = the default 24576) and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in
  * chunks of this many lookups, overlapped with the lookups of the previous
  * chunk; default 10^7, split evenly).  INVALID_ARG for an
  * unknown name or value.  Never changes results. */

@@ -105,6 +105,7 @@ struct Params {
   // partitioned A2 (k_part_*): H[block][key] lives in bins
   int cbits;            // coarse energy bits per material
   int fine_direct;      // k_part_fine scatters directly above this many windows
+  int fine_cap;         // k_part_fine window (lookups)
   uint32_t* key_tot;    // [nkeys] lookups per coarse key
   uint32_t* key_start;  // [nkeys] first position of the key
   double* sp_tmp;       // [count] energies in coarse-key order
@@ -813,19 +814,20 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
 // lookups in shared memory and stores the window as one coalesced run.
 constexpr int kFineThreads = 1024, kFineBinsMax = 4096, kFineIlp = 4;
 constexpr int kFineCapP = 24576, kFineCapPI = 16384;  // energies / energy + position
+__host__ __device__ constexpr size_t fine_hist_bytes(uint32_t nf) { return ((2 * nf + 1) * 4 + 15) / 16 * 16; }
 __global__ void __launch_bounds__(kFineThreads) k_part_fine(Params P) {
   extern __shared__ __align__(16) unsigned char smem_fine[];
+  const int fb = 18 - P.cbits;
+  const uint32_t nf = 1u << fb, fmask = nf - 1u;
   uint32_t* s_st = reinterpret_cast<uint32_t*>(smem_fine);            // [nf + 1] bin starts
-  uint32_t* s_cu = s_st + kFineBinsMax + 1;                            // [nf] cursors
-  const uint32_t cap = P.sidx_tmp ? kFineCapPI : kFineCapP;
-  double* s_p = reinterpret_cast<double*>(s_cu + kFineBinsMax + 3);    // [cap]
+  uint32_t* s_cu = s_st + nf + 1;                                      // [nf] cursors
+  const uint32_t cap = static_cast<uint32_t>(P.fine_cap);
+  double* s_p = reinterpret_cast<double*>(smem_fine + fine_hist_bytes(nf));  // [cap]
   uint32_t* s_i = reinterpret_cast<uint32_t*>(s_p + cap);              // [cap] (positions)
   __shared__ uint32_t s_win[2];
   const int key = blockIdx.x;
   const uint32_t s = P.key_start[key], n = P.key_tot[key];
   if (n == 0) return;
-  const int fb = 18 - P.cbits;
-  const uint32_t nf = 1u << fb, fmask = nf - 1u;
   const int t = threadIdx.x;
   for (uint32_t f = t; f < nf; f += kFineThreads) s_cu[f] = 0;
   __syncthreads();
@@ -2657,9 +2659,12 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       k_part_place<GT><<<nb, kPrepThreads, pl_smem, st>>>(P);
     }
     {
-      const size_t fine_smem = (2 * static_cast<size_t>(kFineBinsMax) + 4) * 4 +
-                               (per_lookup ? static_cast<size_t>(kFineCapPI) * 12
-                                           : static_cast<size_t>(kFineCapP) * 8);
+      // window: fine_cap energies (2/3 of it with batch positions), default
+      // the most that fits one 1024-thread block per SM
+      const uint32_t cap_p = g.fine_cap ? static_cast<uint32_t>(g.fine_cap) : kFineCapP;
+      P.fine_cap = static_cast<int>(per_lookup ? (g.fine_cap ? cap_p * 2 / 3 : kFineCapPI) : cap_p);
+      const size_t fine_smem = fine_hist_bytes(1u << (18 - P.cbits)) +
+                               static_cast<size_t>(P.fine_cap) * (per_lookup ? 12 : 8);
       e = cudaFuncSetAttribute(k_part_fine, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                static_cast<int>(fine_smem));
       if (e != cudaSuccess) return e;

@@ -687,6 +687,10 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   } else if (!std::strcmp(name, "fine_direct")) {
     if (value < 0 || value > 1024) return fail(XS_ERR_INVALID_ARG, "fine_direct in [0,1024]");
     G.fine_direct = static_cast<int>(value);
+  } else if (!std::strcmp(name, "fine_cap")) {
+    if (value != 0 && (value < 2048 || value > 24576))
+      return fail(XS_ERR_INVALID_ARG, "fine_cap is 0 (default) or 2048-24576");
+    G.fine_cap = static_cast<int>(value);
   } else {
     return fail(XS_ERR_INVALID_ARG, std::string("unknown parameter ") + name);
   }

@@ -521,9 +521,10 @@ def test_explicit_gate_both_kernels_agree(X, sort):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("fine_direct", [0, 2])
+@pytest.mark.parametrize("fine_cap", [0, 2048])
+@pytest.mark.parametrize("fine_direct", [0, 2, 1024])
 @pytest.mark.parametrize("cbits", [6, 7, 8, 9])
-def test_part_cbits_tiny_parity(X, cbits, fine_direct):
+def test_part_cbits_tiny_parity(X, cbits, fine_direct, fine_cap):
     """Every coarse fan-out of the partitioned A2 (part_cbits 6-9), with the
     fine pass windowed or scattering directly (fine_direct 0: every segment),
     gives the oracle's per-lookup results; the order inside the sort never
@@ -531,6 +532,7 @@ def test_part_cbits_tiny_parity(X, cbits, fine_direct):
     g = X.Grid.from_preset("tiny")
     g.set_param("part_cbits", cbits)
     g.set_param("fine_direct", fine_direct)
+    g.set_param("fine_cap", fine_cap)  # 2048: many windows per segment
     S, ref = oracle_for("tiny").run(3, 100_000, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
     vs, out = _full_outputs(g, 3, 100_000, sort=True)
     _compare(out, ref)
