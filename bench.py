@@ -340,7 +340,7 @@ def run_history(a, pre, cfg):
                          "note": f"algorithmic bytes per chained lookup = {balg:.0f} "
                                  "(E[n] x (4 + 96) B + unionized search probes)"},
             "gpu_launches": int(tm["kernel_launches"]),
-            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash": D.global_hash(vglob), "lookups_per_step": vglob[1],
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
             "clocks": clk.summary()}
     # e2e: the public call from a host program (nothing to upload: particles
@@ -535,7 +535,7 @@ def run_rs(a, pre, cfg):
                                  f"{RS_OPS_PER_LOOKUP} per lookup; sqrt/sin/cos/IEEE "
                                  "division count one each (DESIGN.md §10)"},
             "gpu_launches": int(launches),
-            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash": D.global_hash(vglob), "lookups_per_step": vglob[1],
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
             "device_bytes": int(p.device_bytes), "step_ms_recheck": step_ms_lookup}
     # e2e: the shard's (energy, material) pairs from pinned host memory through
@@ -710,7 +710,7 @@ def run_ours(a, pre, cfg):
             "phase_ms_per_step": {k: tm[k] / max(1, tm["calls"])
                                   for k in ("ms_count", "ms_bucket", "ms_gather")},
             "gpu_launches": int(tm["kernel_launches"]),
-            "hash": vglob[0] % 999983, "lookups_per_step": vglob[1],
+            "hash": D.global_hash(vglob), "lookups_per_step": vglob[1],
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
             "grid_device_bytes": int(g.info.device_bytes)}
     # ------------------------------------------------------------- e2e leg

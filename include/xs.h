@@ -167,6 +167,11 @@ typedef struct {
 #define XS_TABLE_MATS 4         /* [int32]  n_mats*max_num_nucs                 */
 #define XS_TABLE_CONCS 5        /* [double] n_mats*max_num_nucs                 */
 #define XS_TABLE_INDEX_GRID_T 6 /* [int32]  IGT (I*NU), nuclide-major            */
+#define XS_TABLE_INTERVALS 7    /* [double] I*N*14: interval table (DESIGN.md §4 K0d):
+                                   entry (n, k) = {E[k+1], E[k+1] - E[k], ~1/gap, 0,
+                                   (hi.c, hi.c - lo.c) x 5}; entry N-1 is zero     */
+#define XS_TABLE_INTERVALS32 8  /* [double] I*N*10: fp32-variant table (K0e): {E[k+1],
+                                   gap, ~1/gap, 0} then 12 floats (h_c, d_c) x 5, 0, 0 */
 
 uint32_t xs_abi_version(void);
 
@@ -193,6 +198,25 @@ xs_status xs_workspace_size(const xs_grid* g, uint64_t count, uint32_t flags, si
 xs_status xs_lookup_batch(xs_grid* g, uint64_t first_id, uint64_t count, uint32_t flags,
                           const xs_outputs* out, void* workspace, size_t workspace_bytes,
                           void* cuda_stream);
+
+/* Energy-range shard of a sampled batch (multi-GPU strong scaling; DESIGN.md
+ * §6): A1 for lookup ids [first_id, first_id + count), then A2-A8 only for the
+ * lookups whose energy p lies in shard `shard` of `n_shards`:
+ *   b_s <= p < b_{s+1},  b_s = RN(s / n_shards) (binary64 quotient) for
+ *   0 < s < n_shards, b_0 = -inf, b_{n_shards} = +inf,
+ * so the shards of one batch partition it (every lookup is looked up by
+ * exactly one shard) and the vsum of all shards equals xs_lookup_batch's.
+ * Each shard keeps the full batch's density in energy (a rank's lookups are
+ * as close together as in one big batch, unlike a contiguous id range).
+ * vsum += {sum v, #lookups in the shard}; per-lookup outputs (device
+ * pointers indexed by batch position) are written only for the shard's
+ * lookups, the other positions are left untouched.  Requires XS_FLAG_SORT
+ * (the partitioned A2), optionally XS_FLAG_F32; XS_FLAG_BASELINE and
+ * XS_FLAG_HOST_IO are INVALID_ARG; a batch or variant the partitioned A2
+ * cannot serve is UNSUPPORTED.  Workspace as xs_workspace_size(count, flags). */
+xs_status xs_lookup_batch_shard(xs_grid* g, uint64_t first_id, uint64_t count, int32_t shard,
+                                int32_t n_shards, uint32_t flags, const xs_outputs* out,
+                                void* workspace, size_t workspace_bytes, void* cuda_stream);
 
 /* A2-A8 for caller-given lookups: energy[i] (any double; outside the grid the
  * XS are extrapolated) and mat[i] (0 <= mat < n_mats; an out-of-range mat

@@ -29,6 +29,10 @@ _SOURCES = [os.path.join(_HERE, "xs_oracle.c"), os.path.join(_HERE, "xs_oracle.h
 
 UNIONIZED, NUCLIDE, HASH = 0, 1, 2
 F32 = 0x10   # OR into a mode: the fp32 variant (R18)
+# run() modes whose M output is an error scale of the binary64 result instead
+# of M: SCALE_A = sum_j |x_c conc_j|, SCALE_S = sum_j conc_j
+# (|hi.c| + |f| (|hi.c| + |lo.c|)) (R18's a-priori scale)
+SCALE_A, SCALE_S = 0x20, 0x40
 _lock = threading.Lock()
 _lib = None
 
@@ -99,6 +103,9 @@ def lib() -> C.CDLL:
                 "oracle_run_explicit": (u64, [P, P, P, u64, C.c_int, C.c_int, P, P]),
                 "oracle_run_history": (u64, [P, u64, u64, i32, C.c_int, C.c_int, P, P, P, P]),
                 "oracle_hash_finalize": (u64, [u64]),
+                "oracle_macro_scales": (None, [P, d, i32, P, P]),
+                "oracle_index_grid_rows": (None, [P, i64, i64, P]),
+                "oracle_hash_grid": (None, [P, P]),
                 "xsgen_num_nucs": (C.c_int, [i32, i32, P]),
                 "xsgen_max_num_nucs": (i32, [i32, i32]),
                 "xsgen_mats": (C.c_int, [i32, i32, i32, P]),
@@ -290,6 +297,25 @@ class Oracle:
             raise MemoryError
         return out
 
+    def index_grid_rows(self, e0: int, e1: int) -> np.ndarray:
+        """IG rows [e0, e1) by the definition (R6)."""
+        out = np.empty((e1 - e0, self.I), np.int32)
+        lib().oracle_index_grid_rows(self._h, e0, e1, _ptr(out))
+        return out
+
+    def hash_grid(self, B: int) -> np.ndarray:
+        """The whole hash grid HG [B][I] (R7); B = the context's hash_bins."""
+        out = np.empty((B, self.I), np.int32)
+        lib().oracle_hash_grid(self._h, _ptr(out))
+        return out
+
+    def macro_scales(self, p: float, mat: int):
+        """(A, S): Q12's sum_j |x_c conc_j| and R18's a-priori scale."""
+        A = np.zeros(5, np.float64)
+        S = np.zeros(5, np.float64)
+        lib().oracle_macro_scales(self._h, p, mat, _ptr(A), _ptr(S))
+        return A, S
+
     def hash_bin(self, p: float) -> int:
         return lib().oracle_hash_bin(self._h, p)
 
@@ -358,9 +384,13 @@ class Oracle:
         return S, dict(p=p, mat=mat, M=M, v=v)
 
     def run_explicit(self, p: np.ndarray, mat: np.ndarray, mode: int = UNIONIZED,
-                     nthreads: int = 1):
+                     nthreads: int = 1, outputs: bool = True):
+        """Caller-given lookups.  Returns (S, M, v), or S alone (outputs=False)."""
         p = np.ascontiguousarray(p, np.float64)
         mat = np.ascontiguousarray(mat, np.int32)
+        if not outputs:
+            return lib().oracle_run_explicit(self._h, _ptr(p), _ptr(mat), len(p), mode, nthreads,
+                                             None, None)
         M = np.empty((len(p), 5), np.float64)
         v = np.empty(len(p), np.int32)
         S = lib().oracle_run_explicit(self._h, _ptr(p), _ptr(mat), len(p), mode, nthreads,

@@ -29,6 +29,8 @@ extern "C" {
 enum { ORACLE_UNIONIZED = 0, ORACLE_NUCLIDE = 1, ORACLE_HASH = 2 };
 /* OR'ed into `mode` of oracle_lookup / oracle_run*: the fp32 variant (R18) */
 enum { ORACLE_F32 = 0x10 };
+/* run modes that return an error scale in M instead of M (oracle_macro_scales) */
+enum { ORACLE_SCALE_A = 0x20, ORACLE_SCALE_S = 0x40 };
 
 typedef struct oracle_ctx oracle_ctx;
 
@@ -118,6 +120,12 @@ uint64_t oracle_run_history(const oracle_ctx* c, uint64_t first_particle, uint64
 
 /* hash = S mod 999983, once, after the global sum (R13). */
 uint64_t oracle_hash_finalize(uint64_t S);
+/* error scales of the binary64 result (Q12's A_c, R18's S_c) */
+void oracle_macro_scales(const oracle_ctx* c, double p, int32_t mat, double A[5], double S[5]);
+/* IG rows [e0, e1) by definition (R6), [e1 - e0][I] */
+void oracle_index_grid_rows(const oracle_ctx* c, int64_t e0, int64_t e1, int32_t* out);
+/* the hash grid HG[b][n] (R7), [B][I] */
+void oracle_hash_grid(const oracle_ctx* c, int32_t* out);
 
 #ifdef __cplusplus
 }

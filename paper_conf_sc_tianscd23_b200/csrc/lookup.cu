@@ -104,6 +104,11 @@ struct Params {
                        // searches only each task's extreme energies)
   // partitioned A2 (k_part_*): H[block][key] lives in bins
   int cbits;            // coarse energy bits per material
+  int nkr;              // coarse keys per material: (energy_bin >> (18 - cbits)) in
+                        // [kc_lo, kc_lo + nkr) (all 2^cbits of them unless sharded)
+  int kc_lo;
+  int shard;            // 1: only lookups with e_lo <= p < e_hi are looked up
+  double e_lo, e_hi;    //    (energy-range shard, xs_lookup_batch_shard)
   int fine_direct;      // k_part_fine scatters directly above this many windows
   int fine_cap;         // k_part_fine window (lookups)
   uint32_t* key_tot;    // [nkeys] lookups per coarse key
@@ -155,7 +160,7 @@ __global__ void k_check_energies(const double* __restrict__ p, uint32_t n, uint3
   if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1u);
 }
 
-__device__ __forceinline__ uint32_t energy_bin(double p) {
+__host__ __device__ __forceinline__ uint32_t energy_bin(double p) {
   const double q = p * static_cast<double>(kEnergyBins);
   if (!(q > 0.0)) return 0u;
   return q < static_cast<double>(kEnergyBins - 1) ? static_cast<uint32_t>(q) : kEnergyBins - 1u;
@@ -575,7 +580,13 @@ __device__ __forceinline__ void affine_pow(uint64_t n, uint64_t& A, uint64_t& C)
 }
 
 __device__ __forceinline__ uint32_t part_key(const Params& P, const Sample& s) {
-  return (static_cast<uint32_t>(s.mat) << P.cbits) | (energy_bin(s.p) >> (18 - P.cbits));
+  return static_cast<uint32_t>(s.mat) * static_cast<uint32_t>(P.nkr) +
+         ((energy_bin(s.p) >> (18 - P.cbits)) - static_cast<uint32_t>(P.kc_lo));
+}
+
+// energy-range shard filter (always true outside shard mode)
+__device__ __forceinline__ bool in_shard(const Params& P, double p) {
+  return !P.shard || (p >= P.e_lo && p < P.e_hi);
 }
 
 // The kPartItems lookups of thread t in the chunk starting at c0 (the same
@@ -596,6 +607,7 @@ __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint6
       const double pe = lcg_double(st);
       st = lcg_next(st);
       smp[it] = Sample{pe, pick_material(lcg_double(st))};
+      ok[it] = ok[it] && in_shard(P, pe);
     }
   }
 }
@@ -621,7 +633,7 @@ struct PartStream {
 template <int GT>
 __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
   extern __shared__ uint32_t s_h[];  // [nkeys]
-  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int nkeys = (P.n_mats + 1) * P.nkr;
   const uint32_t tchunks = part_tile_chunks(P.count);
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
@@ -670,7 +682,7 @@ constexpr int kColIlp = 8;
 // 32 keys x 32 slices of the tiles.
 __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
   __shared__ uint32_t s_p[32][33];
-  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int nkeys = (P.n_mats + 1) * P.nkr;
   const int key = blockIdx.x * 32 + threadIdx.x;
   const int sl = threadIdx.y;
   const int per = (nb + 31) / 32;
@@ -717,7 +729,7 @@ __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
 
 // key_start = exclusive scan of key_tot (one block); counts[m] per material
 __global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
-  const int nkeys = (P.n_mats + 1) << P.cbits;
+  const int nkeys = (P.n_mats + 1) * P.nkr;
   const int per = (nkeys + 1023) / 1024;
   const int k0 = threadIdx.x * per, k1 = min(nkeys, k0 + per);
   uint32_t sum = 0;
@@ -730,8 +742,8 @@ __global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
   }
   __syncthreads();
   for (int m = threadIdx.x; m <= P.n_mats; m += blockDim.x) {
-    const uint32_t s = P.key_start[m << P.cbits];
-    const uint32_t e = m < P.n_mats ? P.key_start[(m + 1) << P.cbits] : total;
+    const uint32_t s = P.key_start[m * P.nkr];
+    const uint32_t e = m < P.n_mats ? P.key_start[(m + 1) * P.nkr] : total;
     P.counts[m] = e - s;
   }
 }
@@ -743,8 +755,8 @@ __global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
 template <int GT>
 __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
   extern __shared__ __align__(16) unsigned char smem_pl[];
-  const int nkeys = (P.n_mats + 1) << P.cbits;
-  const int nvalid = P.n_mats << P.cbits;
+  const int nkeys = (P.n_mats + 1) * P.nkr;
+  const int nvalid = P.n_mats * P.nkr;
   const uint32_t tchunks = part_tile_chunks(P.count);
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
@@ -1835,6 +1847,7 @@ struct AccF64 {  // binary64 (R10, R11): entry = K0d, 7 x 16 B
       for (int c = 0; c < 5; ++c) M[r][c] = 0.0;
   }
   __device__ __forceinline__ double get(int r, int c) const { return M[r][c]; }
+  __device__ __forceinline__ void flush() {}  // one accumulation level (R11)
   template <bool SHARED>
   __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
                                          int r1) {
@@ -1842,19 +1855,34 @@ struct AccF64 {  // binary64 (R10, R11): entry = K0d, 7 x 16 B
   }
 };
 
+// R18's accumulation block: nuclides are summed in blocks of kF32Block (list
+// order); flush() after nuclides 15, 31, ... and after the last one
+constexpr int kF32Block = 16;
+
 template <int R, bool CHECK>
 struct AccF32 {  // binary32 variant (R18): entry = K0e, 5 x 16 B
   static_assert(R % 2 == 0, "fp32 accumulators pair lookups");
   static constexpr int kE = kIv32Doubles / 2;
-  float2 M[R / 2][5];  // {lookup 2q, lookup 2q+1}
+  float2 M[R / 2][5];  // block sums {lookup 2q, lookup 2q+1}
+  float2 T[R / 2][5];  // totals
   __device__ __forceinline__ void zero() {
 #pragma unroll
     for (int q = 0; q < R / 2; ++q)
 #pragma unroll
-      for (int c = 0; c < 5; ++c) M[q][c] = make_float2(0.0f, 0.0f);
+      for (int c = 0; c < 5; ++c) M[q][c] = T[q][c] = make_float2(0.0f, 0.0f);
+  }
+  // T += B, B = 0 (fma(B, 1, T) is the correctly rounded sum)
+  __device__ __forceinline__ void flush() {
+#pragma unroll
+    for (int q = 0; q < R / 2; ++q)
+#pragma unroll
+      for (int c = 0; c < 5; ++c) {
+        T[q][c] = ffma2(M[q][c], make_float2(1.0f, 1.0f), T[q][c]);
+        M[q][c] = make_float2(0.0f, 0.0f);
+      }
   }
   __device__ __forceinline__ double get(int r, int c) const {
-    return static_cast<double>((r & 1) ? M[r >> 1][c].y : M[r >> 1][c].x);
+    return static_cast<double>((r & 1) ? T[r >> 1][c].y : T[r >> 1][c].x);
   }
   template <bool SHARED>
   __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
@@ -2152,7 +2180,9 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
         const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
         stage_nuclide_iv<R, false>(g2, n_int, conc, p, acc);
       }
+      if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
     }
+    if (nn & (kF32Block - 1)) acc.flush();
     __syncwarp();
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -2552,7 +2582,7 @@ static uint32_t part_tiles(uint64_t count) {
 // 41.5 -> 42.1 / 42.8 ms at 8 / 9 bits).  Limits: k_part_place holds
 // three key arrays and the tile in shared memory, keys are 16 bit, and the
 // fine histogram has at most kFineBinsMax bins.
-constexpr int kPartCbits = 7, kPartCbitsMax = 9;
+constexpr int kPartCbits = 7, kPartCbitsMin = 6, kPartCbitsMax = 9;
 
 static size_t part_place_smem(uint64_t count, int32_t n_mats, int cbits, bool per_lookup) {
   const size_t nkeys = static_cast<size_t>(n_mats + 1) << cbits;
@@ -2561,7 +2591,7 @@ static size_t part_place_smem(uint64_t count, int32_t n_mats, int cbits, bool pe
 }
 
 bool part_cbits_fit(uint64_t count, int32_t n_mats, int cbits) {
-  return cbits >= 18 - 12 && cbits <= kPartCbitsMax && (static_cast<size_t>(n_mats + 1) << cbits) <= 65536 &&
+  return cbits >= kPartCbitsMin && cbits <= kPartCbitsMax && (static_cast<size_t>(n_mats + 1) << cbits) <= 65536 &&
          part_place_smem(count, n_mats, cbits, true) <= 227 * 1024;
 }
 
@@ -2572,11 +2602,33 @@ static int part_cbits(uint64_t count, int32_t n_mats, int requested) {
 // Bytes the partitioned A2 keeps in the A2 bin area: H [ntiles][nkeys] plus
 // the key totals and starts (workspace_layout reserves the larger of this and
 // the global-atomic bin array), for the widest coarse key that fits.
+static size_t part_bins_need(uint64_t count, size_t nkeys) {
+  return (static_cast<size_t>(part_tiles(count)) * nkeys + 2 * nkeys) * 4;
+}
 size_t part_bins_bytes(uint64_t count, int32_t n_mats) {
   int c = kPartCbits;
   while (c < kPartCbitsMax && part_cbits_fit(count, n_mats, c + 1)) ++c;
-  const size_t nkeys = static_cast<size_t>(n_mats + 1) << c;
-  return (static_cast<size_t>(part_tiles(count)) * nkeys + 2 * nkeys) * 4;
+  return part_bins_need(count, static_cast<size_t>(n_mats + 1) << c);
+}
+
+uint32_t energy_bin_host(double p) { return energy_bin(p); }
+
+// Coarse-key range of the partitioned A2 for a batch: all 2^cbits coarse
+// keys per material, or (energy-range shard) only those of [e_lo, e_hi).
+struct PartKeys {
+  int cbits, kc_lo, nkr;
+  size_t nkeys(int32_t n_mats) const { return static_cast<size_t>(n_mats + 1) * nkr; }
+};
+static PartKeys part_keys(const LookupArgs& a, int cbits) {
+  PartKeys k{cbits, 0, 1 << cbits};
+  if (a.shard) {
+    const int fb = 18 - cbits;
+    const uint32_t lo = a.e_lo > 0.0 ? energy_bin(a.e_lo) : 0u;
+    const uint32_t hi = a.e_hi < 1.0 ? energy_bin(a.e_hi) : kEnergyBins - 1u;
+    k.kc_lo = static_cast<int>(lo >> fb);
+    k.nkr = static_cast<int>(hi >> fb) - k.kc_lo + 1;
+  }
+  return k;
 }
 
 template <int GT>
@@ -2627,14 +2679,30 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28);
-  if (binned && staged && !g.legacy_sort &&
-      part_tile_chunks(a.count) <= 12) {  // k_part_place stages a tile in shared memory
+  // partitioned A2: the widest coarse key at or below the request whose tile
+  // histograms fit the workspace's bin area (a chunk of a host-input batch
+  // may allow a wider key than the batch the workspace was sized for)
+  PartKeys pk = part_keys(a, part_cbits(a.count, g.n_mats, g.part_cbits));
+  while (pk.cbits > kPartCbitsMin &&
+         part_bins_need(a.count, pk.nkeys(g.n_mats)) > ws.bins_bytes)
+    pk = part_keys(a, pk.cbits - 1);
+  const bool part_ok = part_tile_chunks(a.count) <= 12 &&  // k_part_place stages a tile in smem
+                       part_cbits_fit(a.count, g.n_mats, pk.cbits) &&
+                       part_bins_need(a.count, pk.nkeys(g.n_mats)) <= ws.bins_bytes;
+  if (a.shard && !(binned && staged && !g.legacy_sort && part_ok))
+    return cudaErrorNotSupported;  // energy-range shards need the partitioned A2
+  if (binned && staged && !g.legacy_sort && part_ok) {
     // partitioned A2 (k_part_*) feeding the staged gather: energies (+ batch
     // positions when per-lookup results are written) in sorted order
     P.need_gidx = 0;
-    P.cbits = part_cbits(a.count, g.n_mats, g.part_cbits);  // (a request that does not fit: 7)
+    P.cbits = pk.cbits;
+    P.kc_lo = pk.kc_lo;
+    P.nkr = pk.nkr;
+    P.shard = a.shard ? 1 : 0;
+    P.e_lo = a.e_lo;
+    P.e_hi = a.e_hi;
     P.fine_direct = g.fine_direct;
-    const int nkeys = (g.n_mats + 1) << P.cbits;
+    const int nkeys = static_cast<int>(pk.nkeys(g.n_mats));
     const uint32_t ntiles = part_tiles(a.count);
     const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;
     P.bins = ws.bins;  // H [ntiles][nkeys]
@@ -2668,7 +2736,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       e = cudaFuncSetAttribute(k_part_fine, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                static_cast<int>(fine_smem));
       if (e != cudaSuccess) return e;
-      k_part_fine<<<g.n_mats << P.cbits, kFineThreads, fine_smem, st>>>(P);
+      k_part_fine<<<g.n_mats * P.nkr, kFineThreads, fine_smem, st>>>(P);
     }
     launched(5);
   } else if (binned) {

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <array>
 #include <cstdio>
 #include <cstring>
@@ -87,13 +88,14 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
   const size_t o_recs = take(count * sizeof(LookupRec));
   const size_t o_tmp = take(count * sizeof(LookupRec));
   const size_t o_mat8 = take(count);
-  size_t o_bins = 0, o_part = 0, o_perm = 0;
+  size_t o_bins = 0, o_part = 0, o_perm = 0, bins_bytes = 0;
   if (flags & XS_FLAG_SORT) {
     o_perm = take(count * 4);
     // the bin area serves both A2 forms: the global-atomic bins and the
     // partitioned A2's tile histograms (whichever is larger for this count)
-    o_bins = take(std::max(static_cast<size_t>(n_mats + 1) * kEnergyBins * 4,
-                           part_bins_bytes(count, n_mats)));
+    bins_bytes = std::max(static_cast<size_t>(n_mats + 1) * kEnergyBins * 4,
+                          part_bins_bytes(count, n_mats));
+    o_bins = take(bins_bytes);
     o_part = take(static_cast<size_t>(n_mats + 1) * (kEnergyBins / 4096) * 4);
   }
   if (ws) {
@@ -107,6 +109,7 @@ size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* ba
     ws->perm = reinterpret_cast<uint32_t*>(b + o_perm);
     ws->tmp = reinterpret_cast<LookupRec*>(b + o_tmp);
     ws->mat8 = reinterpret_cast<uint8_t*>(b + o_mat8);
+    ws->bins_bytes = bins_bytes;
     ws->total = off;
   }
   return off;
@@ -399,10 +402,15 @@ xs_status xs_workspace_size(const xs_grid* g, uint64_t count, uint32_t flags, si
   return XS_OK;
 }
 
+struct ShardSel {
+  bool on = false;
+  double e_lo = 0.0, e_hi = 0.0;
+};
+
 static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* energy,
                                const int32_t* mat, uint64_t count, uint32_t flags,
                                const xs_outputs* out, void* workspace, size_t ws_bytes,
-                               void* cuda_stream) {
+                               void* cuda_stream, ShardSel shard = ShardSel()) {
   if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
   if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
   if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
@@ -434,6 +442,9 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   a.in_mat8 = mat8 ? reinterpret_cast<const uint8_t*>(mat) : nullptr;
   a.out = *out;
   a.launches = &g->d.launches;
+  a.shard = shard.on;
+  a.e_lo = shard.e_lo;
+  a.e_hi = shard.e_hi;
   if (g->timing) {
     if (g->ev_used == g->ev.size()) {
       std::array<cudaEvent_t, 4> evs{};
@@ -513,6 +524,9 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
       e = run_lookup(g->d, c, ws, st);
     }
   }
+  if (e == cudaErrorNotSupported && shard.on)
+    return fail(XS_ERR_UNSUPPORTED, "energy-range shards need the partitioned A2 (XS_FLAG_SORT, "
+                                    "staged gather variant, batch <= 268M lookups)");
   if (e != cudaSuccess) return fail(XS_ERR_CUDA, "lookup launch", e);
   if (host_io) {
     struct {
@@ -536,6 +550,25 @@ xs_status xs_lookup_batch(xs_grid* g, uint64_t first_id, uint64_t count, uint32_
     return fail(XS_ERR_UNSUPPORTED, "sampled batches need the 12 XSBench materials");
   return lookup_common(g, first_id, nullptr, nullptr, count, flags, out, workspace,
                        workspace_bytes, cuda_stream);
+}
+
+xs_status xs_lookup_batch_shard(xs_grid* g, uint64_t first_id, uint64_t count, int32_t shard,
+                                int32_t n_shards, uint32_t flags, const xs_outputs* out,
+                                void* workspace, size_t workspace_bytes, void* cuda_stream) {
+  if (g && g->d.n_mats != XSGEN_N_MATS)
+    return fail(XS_ERR_UNSUPPORTED, "sampled batches need the 12 XSBench materials");
+  if (n_shards < 1 || shard < 0 || shard >= n_shards)
+    return fail(XS_ERR_INVALID_ARG, "need 0 <= shard < n_shards");
+  if (!(flags & XS_FLAG_SORT) || (flags & (XS_FLAG_BASELINE | XS_FLAG_HOST_IO)))
+    return fail(XS_ERR_INVALID_ARG, "energy-range shards need XS_FLAG_SORT and device outputs "
+                                    "(no XS_FLAG_BASELINE / XS_FLAG_HOST_IO)");
+  ShardSel s;
+  s.on = true;
+  s.e_lo = shard == 0 ? -HUGE_VAL : static_cast<double>(shard) / static_cast<double>(n_shards);
+  s.e_hi = shard == n_shards - 1 ? HUGE_VAL
+                                 : static_cast<double>(shard + 1) / static_cast<double>(n_shards);
+  return lookup_common(g, first_id, nullptr, nullptr, count, flags, out, workspace,
+                       workspace_bytes, cuda_stream, s);
 }
 
 xs_status xs_lookup_explicit(xs_grid* g, const double* energy, const int32_t* mat, uint64_t count,
@@ -649,6 +682,9 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
     case XS_TABLE_INDEX_GRID_T:
       if (!G.index_t) return fail(XS_ERR_UNSUPPORTED, "grid has no column-layout index grid");
       src = G.index_t; len = G.index_len; es = 4; break;
+    case XS_TABLE_INTERVALS: src = G.iv; len = static_cast<uint64_t>(G.I) * G.N * kIvDoubles; break;
+    case XS_TABLE_INTERVALS32:
+      src = G.iv32; len = static_cast<uint64_t>(G.I) * G.N * kIv32Doubles; break;
     case XS_TABLE_NUM_NUCS: src = G.num_nucs; len = G.n_mats; es = 4; break;
     case XS_TABLE_MATS: src = G.mats; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; es = 4; break;
     case XS_TABLE_CONCS: src = G.concs; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; break;

@@ -69,6 +69,10 @@ struct LookupArgs {
   xs_outputs out{};                    // device pointers
   cudaEvent_t* ev = nullptr;           // [4] phase events (optional)
   uint64_t* launches = nullptr;        // incremented per kernel launch
+  // energy-range shard (xs_lookup_batch_shard): only lookups with
+  // e_lo <= p < e_hi are looked up (partitioned A2 only)
+  bool shard = false;
+  double e_lo = 0.0, e_hi = 0.0;
 };
 
 // workspace layout for a batch
@@ -82,6 +86,8 @@ struct Workspace {
   uint32_t* partials; // A2 scan: [(n_mats + 1) * kEnergyBins / 4096]
   uint32_t* perm;     // A2: [count]
   uint32_t* gate;     // [1] k_check_energies flag (explicit energies)
+  size_t bins_bytes;  // capacity of the bin area (the partitioned A2's tile
+                      // histograms must fit it: coarse keys are narrowed if not)
   size_t total;
 };
 size_t workspace_layout(uint64_t count, uint32_t flags, int32_t n_mats, void* base,
@@ -102,6 +108,7 @@ cudaError_t init_constants();
 
 // lookup.cu
 size_t part_bins_bytes(uint64_t count, int32_t n_mats);  // partitioned A2's bin-area need
+uint32_t energy_bin_host(double p);  // A2's energy bin of p (same arithmetic as the device)
 bool part_cbits_fit(uint64_t count, int32_t n_mats, int cbits);  // shared memory / key-width limits
 cudaError_t run_lookup(const DeviceGrid& g, const LookupArgs& a, const Workspace& ws,
                        cudaStream_t st);

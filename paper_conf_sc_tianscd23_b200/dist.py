@@ -57,5 +57,6 @@ def max_over_ranks(value: float, device=None, group=None) -> float:
 
 def global_hash(vsum_global) -> int:
     """hash = (sum over all ranks of v) mod 999983, applied once after the
-    global reduction (R13)."""
-    return int(vsum_global[0]) % 999983
+    global reduction (R13) — the library's xs_hash_finalize."""
+    from .xs import xs_hash_finalize
+    return int(xs_hash_finalize(int(vsum_global[0]) & 0xFFFFFFFFFFFFFFFF))

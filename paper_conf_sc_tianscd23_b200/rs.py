@@ -175,7 +175,7 @@ class RSProblem:
         return self._ws
 
     def lookup(self, first_id: int, count: int, sort: bool = True, baseline: bool = False,
-               want=(), vsum=None, stream=None):
+               want=(), vsum=None):
         """R1-R7 for lookup ids [first_id, first_id+count) on the current stream.
         Returns (vsum tensor [2] on device, dict of the outputs in `want`:
         macro_xs [count][4], mat, energy)."""
@@ -195,11 +195,11 @@ class RSProblem:
                        mk("mat", (count,), torch.int32), mk("energy", (count,), torch.float64),
                        vsum.data_ptr())
         ws = self.workspace(count, flags)
-        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
+        st = torch.cuda.current_stream(self.device).cuda_stream  # torch's allocator orders reuse here
         rs_lookup_batch(self._h, first_id, count, flags, o, ws.data_ptr(), ws.numel(), st)
         return vsum, res
 
-    def lookup_explicit(self, energy, mat, sort: bool = True, want=(), vsum=None, stream=None):
+    def lookup_explicit(self, energy, mat, sort: bool = True, want=(), vsum=None):
         """R2-R7 for caller-given energies (float64) and materials (uint8).
         CUDA tensors, or CPU tensors (then RS_FLAG_HOST_IO: staged copies inside
         the call, which synchronizes; only macro_xs may be requested)."""
@@ -224,7 +224,7 @@ class RSProblem:
                        mk("mat", (count,), torch.int32), mk("energy", (count,), torch.float64),
                        vsum.data_ptr())
         ws = self.workspace(count, flags)
-        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
+        st = torch.cuda.current_stream(self.device).cuda_stream  # torch's allocator orders reuse here
         rs_lookup_explicit(self._h, energy.data_ptr(), mat.data_ptr(), count, flags, o,
                            ws.data_ptr(), ws.numel(), st)
         return vsum, res

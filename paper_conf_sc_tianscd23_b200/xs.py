@@ -23,7 +23,8 @@ XS_GRID_UNIONIZED, XS_GRID_NUCLIDE, XS_GRID_HASH = 0, 1, 2
 XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE, XS_FLAG_F32 = 0x1, 0x2, 0x4, 0x8
 XS_FLAG_MAT_U8 = 0x10
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
- XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T) = range(7)
+ XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T, XS_TABLE_INTERVALS,
+ XS_TABLE_INTERVALS32) = range(9)
 XS_INDEX_AUTO, XS_INDEX_ROW, XS_INDEX_COL, XS_INDEX_BOTH = 0, 1, 2, 3
 INDEX_LAYOUTS = {"auto": 0, "row": 1, "col": 2, "both": 3}
 STATUS = {0: "XS_OK", 1: "XS_ERR_INVALID_ARG", 2: "XS_ERR_OUT_OF_MEMORY", 3: "XS_ERR_CUDA",
@@ -77,7 +78,7 @@ EXPORTS = ["xs_abi_version", "xs_init_grid", "xs_init_grid_data", "xs_grid_get_i
            "xs_workspace_size", "xs_lookup_batch", "xs_lookup_explicit", "xs_verify",
            "xs_nuclide_index", "xs_get_table", "xs_set_param", "xs_hash_finalize",
            "xs_free_grid", "xs_last_error", "xs_timing_enable", "xs_timing_read",
-           "xs_history_workspace_size", "xs_lookup_history"]
+           "xs_history_workspace_size", "xs_lookup_history", "xs_lookup_batch_shard"]
 
 
 def _load() -> C.CDLL:
@@ -96,6 +97,8 @@ def _load() -> C.CDLL:
         "xs_workspace_size": (st, [P, u64, u32, C.POINTER(C.c_size_t)]),
         "xs_lookup_batch": (st, [P, u64, u64, u32, C.POINTER(xs_outputs), P, C.c_size_t, P]),
         "xs_lookup_explicit": (st, [P, P, P, u64, u32, C.POINTER(xs_outputs), P, C.c_size_t, P]),
+        "xs_lookup_batch_shard": (st, [P, u64, u64, i32, i32, u32, C.POINTER(xs_outputs), P,
+                                       C.c_size_t, P]),
         "xs_verify": (st, [P, P, u64, P, P]),
         "xs_nuclide_index": (st, [P, P, P, u64, P, P]),
         "xs_get_table": (st, [P, i32, u64, u64, P]),
@@ -158,6 +161,12 @@ def xs_workspace_size(g: int, count: int, flags: int) -> int:
 def xs_lookup_batch(g, first_id, count, flags, out: xs_outputs, workspace, ws_bytes, stream):
     _check(lib.xs_lookup_batch(g, first_id, count, flags, C.byref(out), workspace, ws_bytes,
                                stream))
+
+
+def xs_lookup_batch_shard(g, first_id, count, shard, n_shards, flags, out: xs_outputs, workspace,
+                          ws_bytes, stream):
+    _check(lib.xs_lookup_batch_shard(g, first_id, count, shard, n_shards, flags, C.byref(out),
+                                     workspace, ws_bytes, stream))
 
 
 def xs_lookup_explicit(g, energy, mat, count, flags, out: xs_outputs, workspace, ws_bytes,
@@ -320,8 +329,15 @@ class Grid:
                        mk("verification", (count,), torch.int32), vsum.data_ptr())
         return o, res
 
+    def _stream(self) -> int:
+        """torch's current stream of the grid's device: workspace and outputs
+        are allocated by torch's caching allocator, which orders their reuse
+        on this stream, so every call is enqueued on it."""
+        import torch
+        return torch.cuda.current_stream(self.device).cuda_stream
+
     def lookup(self, first_id: int, count: int, sort: bool = False, baseline: bool = False,
-               want=(), vsum=None, stream=None, f32: bool = False):
+               want=(), vsum=None, f32: bool = False):
         """A1-A8 for lookup ids [first_id, first_id+count) on the current stream
         (f32: the fp32 variant, XS_FLAG_F32).
         Returns (vsum tensor [2] uint64-as-int64 on device, dict of outputs)."""
@@ -332,12 +348,34 @@ class Grid:
             vsum = torch.zeros(2, dtype=torch.int64, device=self.device)
         o, res = self._outputs(count, want, vsum)
         ws = self.workspace(count, flags)
-        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
-        xs_lookup_batch(self._h, first_id, count, flags, o, ws.data_ptr(), ws.numel(), st)
+        xs_lookup_batch(self._h, first_id, count, flags, o, ws.data_ptr(), ws.numel(),
+                        self._stream())
         return vsum, res
 
-    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, stream=None,
-                        f32: bool = False):
+    def lookup_shard(self, first_id: int, count: int, shard: int, n_shards: int, want=(),
+                     vsum=None, f32: bool = False, outputs=None):
+        """Energy-range shard `shard` of `n_shards` of the sampled batch
+        [first_id, first_id+count) (xs_lookup_batch_shard; A2 always on).
+        Per-lookup outputs are batch-position indexed and written only for
+        the shard's lookups; pass `outputs` (a dict from an earlier call) to
+        let several shards fill the same tensors."""
+        import torch
+        flags = XS_FLAG_SORT | (XS_FLAG_F32 if f32 else 0)
+        if vsum is None:
+            vsum = torch.zeros(2, dtype=torch.int64, device=self.device)
+        if outputs is None:
+            o, res = self._outputs(count, want, vsum)
+        else:
+            res = outputs
+            g = lambda k: res[k].data_ptr() if k in res else None  # noqa: E731
+            o = xs_outputs(g("macro_xs"), g("energy"), g("mat"), g("grid_index"),
+                           g("verification"), vsum.data_ptr())
+        ws = self.workspace(count, flags)
+        xs_lookup_batch_shard(self._h, first_id, count, shard, n_shards, flags, o,
+                              ws.data_ptr(), ws.numel(), self._stream())
+        return vsum, res
+
+    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, f32: bool = False):
         """A2-A8 for caller-given (energy, material).  energy/mat are CUDA
         tensors (float64 / int32 or uint8 -> XS_FLAG_MAT_U8), or CPU tensors
         (then XS_FLAG_HOST_IO: staged copies inside the call, outputs returned
@@ -352,13 +390,12 @@ class Grid:
             vsum = torch.zeros(2, dtype=torch.int64, device="cpu" if host else self.device)
         o, res = self._outputs(count, want, vsum, host=host)
         ws = self.workspace(count, flags)
-        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
         xs_lookup_explicit(self._h, energy.data_ptr(), mat.data_ptr(), count, flags, o,
-                           ws.data_ptr(), ws.numel(), st)
+                           ws.data_ptr(), ws.numel(), self._stream())
         return vsum, res
 
     def lookup_history(self, first_particle: int, n_particles: int, lookups: int = 34,
-                       sort: bool = False, want=(), vsum=None, stream=None):
+                       sort: bool = False, want=(), vsum=None):
         """History mode (R19): n_particles x lookups chained lookups.
         Per-lookup outputs in `want` (macro_xs, energy, mat, verification) are
         [n_particles * lookups] (lookup i of particle q at q * lookups + i)."""
@@ -370,9 +407,8 @@ class Grid:
         n = xs_history_workspace_size(self._h, n_particles, flags)
         if self._ws is None or self._ws.numel() < n:
             self._ws = torch.empty(max(n, 256), dtype=torch.uint8, device=self.device)
-        st = stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
         xs_lookup_history(self._h, first_particle, n_particles, lookups, flags, o,
-                          self._ws.data_ptr(), self._ws.numel(), st)
+                          self._ws.data_ptr(), self._ws.numel(), self._stream())
         return vsum, res
 
     def verify(self, macro_xs, vsum=None):
@@ -397,7 +433,9 @@ class Grid:
                 XS_TABLE_UNION_ENERGY: i.n_union, XS_TABLE_INDEX_GRID: i.index_grid_len,
                 XS_TABLE_NUM_NUCS: i.n_mats, XS_TABLE_MATS: i.n_mats * i.max_num_nucs,
                 XS_TABLE_CONCS: i.n_mats * i.max_num_nucs,
-                XS_TABLE_INDEX_GRID_T: i.index_grid_len if i.index_layout & 2 else 0}
+                XS_TABLE_INDEX_GRID_T: i.index_grid_len if i.index_layout & 2 else 0,
+                XS_TABLE_INTERVALS: i.n_isotopes * i.n_gridpoints * 14,
+                XS_TABLE_INTERVALS32: i.n_isotopes * i.n_gridpoints * 10}
         dt = np.int32 if which in (XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS, XS_TABLE_MATS,
                                    XS_TABLE_INDEX_GRID_T) \
             else np.float64

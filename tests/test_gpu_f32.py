@@ -3,10 +3,12 @@ oracle's fp32 variant, element by element, and against the binary64 oracle
 within the north_star's fp32 tolerance.
 
 Bars: energy, material, grid index and verification bit-exact; macro XS
-bit-exact against the oracle's R18 arithmetic (same binary32 fused
-multiply-adds in the same order); the verification sum equals the oracle's
-fp32 golden sum at full size; |M32 - M64| within 1e-5 relative for
-99.9% of channel values (north_star "1e-5 if an fp32 variant is offered").
+bit-exact against the oracle's R18 arithmetic (binary32, one rounding per
+operation, blocked accumulation, same order); the verification sum equals
+the oracle's fp32 golden sum at full size; against binary64, for EVERY
+channel value (north_star "1e-5 if an fp32 variant is offered", in SURVEY
+Q12's condition-aware form): |M32 - M64| <= 1e-5 sum_j |x_c conc_j|, and
+R18's a-priori bound |M32 - M64| <= (16 + ceil(n/16) + 4) 2^-24 S_c.
 """
 import json
 import os
@@ -60,10 +62,22 @@ def test_tiny_f32_parity(X, grid_type, bins, sort):
     assert np.array_equal(out["verification"], ref["v"])
     assert [int(x) for x in vs.cpu()] == [S, 100_000]
     assert S == GOLDEN["tiny"]["sum_v_f32"]
-    # the north_star tolerance against binary64
-    _, r64 = o.run(0, 100_000, mode=mode, nthreads=NT, outputs=True)
-    rel = np.abs(out["macro_xs"] - r64["M"]) / np.maximum(np.abs(r64["M"]), 1e-300)
-    assert np.quantile(rel, 0.999) < 1e-5
+    # the north_star tolerance against binary64, element-wise
+    _check_vs_binary64(o, 0, 100_000, mode, out["macro_xs"], ref["mat"])
+
+
+def _check_vs_binary64(o, first, count, mode, M32, mat):
+    """Element-wise: Q12's 1e-5 and R18's a-priori bound against binary64."""
+    _, r64 = o.run(first, count, mode=mode, nthreads=NT, outputs=True)
+    _, ra = o.run(first, count, mode=oracle.SCALE_A, nthreads=NT, outputs=True)
+    _, rs = o.run(first, count, mode=oracle.SCALE_S, nthreads=NT, outputs=True)
+    d = np.abs(M32 - r64["M"])
+    q12 = d / ra["M"]
+    assert q12.max() <= 1e-5, (q12.max(), np.unravel_index(q12.argmax(), q12.shape))
+    n = o.num_nucs()[mat].astype(np.float64)
+    factor = (16 + np.ceil(n / 16) + 4) * 2.0 ** -24
+    assert np.all(d <= factor[:, None] * rs["M"])
+    return q12.max()
 
 
 @pytest.mark.parametrize("variant", [0, 31, 32, 33, 34, 36])
@@ -115,6 +129,30 @@ def test_full_config_f32_hash(X, name):
     mode = oracle.HASH if X.PRESETS[name]["grid_type"] == "hash" else oracle.UNIONIZED
     _, M, _ = o.run_explicit(E, mt, mode=mode | oracle.F32, nthreads=NT)
     assert np.array_equal(Mx, M)
+
+
+@pytest.mark.parametrize("name", ["large"])
+def test_full_config_f32_every_lookup(X, name):
+    """All 17M lookups of the sorted fp32 batch (bench --f32's launch):
+    bit-exact against the oracle's R18 and within the north_star's 1e-5
+    (Q12, element-wise) of binary64 — fuel has 321 nuclides here."""
+    gold = GOLDEN[name]
+    L = gold["lookups"]
+    g = X.Grid.from_preset(name)
+    vs, res = g.lookup(0, L, sort=True, want=("macro_xs", "verification"), f32=True)
+    torch.cuda.synchronize()
+    M32 = res["macro_xs"].cpu().numpy()
+    v32 = res["verification"].cpu().numpy()
+    del res
+    g.close()
+    assert [int(x) for x in vs.cpu()] == [gold["sum_v_f32"], L]
+    o = _oracle(name, hash_bins=8192)
+    S, ref = o.run(0, L, mode=oracle.HASH | oracle.F32, nthreads=NT, outputs=True)
+    bad = np.nonzero(~np.all(M32 == ref["M"], axis=1))[0]
+    assert bad.size == 0, (bad[:5], M32[bad[:3]], ref["M"][bad[:3]])
+    assert np.array_equal(v32, ref["v"])
+    worst = _check_vs_binary64(o, 0, L, oracle.HASH, M32, ref["mat"])
+    assert worst < 1e-5
 
 
 def test_f32_rejects_baseline(X):
