@@ -43,7 +43,15 @@ def parse():
                     choices=["tiny", "small", "large", "large-hash", "xl", "rs-tiny", "rs-small",
                              "rs-large"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
+                    help="strong (default): L lookups in total over N GPUs; weak: L per GPU")
+    ap.add_argument("--shard", default="energy", choices=["energy", "ids"],
+                    help="strong scaling of sorted batches: energy-range shards of all L "
+                         "lookups (default) or contiguous id ranges")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="skip the N=1 context legs (strong-scaling projection, unsorted "
+                         "batch, the paper's kernel shape)")
+    ap.add_argument("--extra-steps", type=int, default=10)
     ap.add_argument("--no-sort", action="store_true", help="skip A2 (material/energy binning)")
     ap.add_argument("--f32", action="store_true",
                     help="the fp32 variant (XS_FLAG_F32, DESIGN.md R18; hash vs the oracle's "
@@ -184,11 +192,13 @@ def cpu_info():
     return name
 
 
-def oracle_sample_rate(pre, target_s: float, first: int = 0, f32: bool = False):
+def oracle_sample_rate(pre, target_s: float, first: int = 0, f32: bool = False,
+                       cores: int | None = None):
     """Time the CPU oracle (as it stands) on a bounded sample of the workload
-    on all host cores.  Returns (lookups/s, cores, description, sum_v)."""
+    on all host cores (or `cores` threads).  Returns (lookups/s, cores,
+    description, sum_v, n)."""
     import oracle
-    cores = os.cpu_count() or 1
+    cores = cores or os.cpu_count() or 1
     mode = ORACLE_MODE[pre["grid_type"]] | (oracle.F32 if f32 else 0)
     o = oracle.Oracle.from_spec(pre["n_isotopes"], pre["n_gridpoints"], conc_seed=1070 * 1070,
                                 material_rule=pre["material_rule"],
@@ -577,6 +587,62 @@ def run_rs(a, pre, cfg):
 
 
 # ------------------------------------------------------------------ ours ----
+def _timed_steps(step, stream, k, world, dist):
+    """k steps bracketed by barrier + synchronize, one CUDA event per step
+    boundary on the launching stream.  Returns (total ms, per-step ms list)."""
+    import torch
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(k + 1)]
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs[0].record(stream)
+    for q in range(k):
+        step()
+        evs[q + 1].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    per = [evs[q].elapsed_time(evs[q + 1]) for q in range(k)]
+    return evs[0].elapsed_time(evs[k]), per
+
+
+def _time_fn(fn, stream, k, warm=2):
+    import torch
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(k):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / k
+
+
+def strong_projection(g, L, f32, stream, value1, ms1, steps=5):
+    """One-GPU projection of strong scaling (L fixed): every rank's shard is
+    timed alone on this GPU; the R-GPU step is the slowest shard (the A9
+    all-reduce of 16 bytes, ~20 us over NVLink, is not included).  Two
+    partitions: energy-range shards (the bench's multi-GPU default,
+    xs_lookup_batch_shard) and contiguous id ranges."""
+    out = {}
+    for R in (2, 4, 8):
+        per_e, per_i = [], []
+        for r in range(R):
+            per_e.append(_time_fn(lambda: g.lookup_shard(0, L, r, R, f32=f32), stream, steps))
+            a, b = r * L // R, (r + 1) * L // R
+            per_i.append(_time_fn(lambda: g.lookup(a, b - a, sort=True, f32=f32), stream, steps))
+        me, mi = max(per_e), max(per_i)
+        out[str(R)] = {"energy_shards": {"ms_per_step": me, "value": L / (me / 1e3),
+                                         "speedup": ms1 / me, "efficiency": ms1 / me / R,
+                                         "rank_ms": [round(x, 4) for x in per_e]},
+                       "id_shards": {"ms_per_step": mi, "value": L / (mi / 1e3),
+                                     "speedup": ms1 / mi, "efficiency": ms1 / mi / R}}
+    return out
+
+
 def run_ours(a, pre, cfg):
     import torch
     import torch.distributed as dist
@@ -596,8 +662,13 @@ def run_ours(a, pre, cfg):
         else:
             dist.init_process_group("gloo")
     sort = not a.no_sort
+    f32 = a.f32
     L_cfg = a.lookups or pre["lookups"]
-    first, L = D.shard_range(rank, world, L_cfg, a.scaling)
+    # strong scaling of a sorted batch: energy-range shards of all L lookups
+    # (each rank keeps the full batch's energy density); otherwise
+    # contiguous id ranges (weak: L per rank; strong unsorted: L / R)
+    energy_shards = a.scaling == "strong" and sort and world > 1 and a.shard == "energy"
+    first, L = (0, L_cfg) if energy_shards else D.shard_range(rank, world, L_cfg, a.scaling)
 
     t0 = time.time()
     g = X.Grid.from_preset(a.config, device=local)
@@ -605,62 +676,73 @@ def run_ours(a, pre, cfg):
     init_s = time.time() - t0
     stream = torch.cuda.current_stream(dev)
 
-    # untimed: per-material counts of this shard (exact algorithmic bytes)
-    # and the inputs of the end-to-end leg
-    f32 = a.f32
-    vs0, res0 = g.lookup(first, L, sort=sort, want=("mat", "energy"), f32=f32)
+    def lookup(vsum=None, want=()):
+        if energy_shards:
+            return g.lookup_shard(0, L_cfg, rank, world, want=want, vsum=vsum, f32=f32)
+        return g.lookup(first, L, sort=sort, want=want, vsum=vsum, f32=f32)
+
+    # untimed: this rank's lookups (per-material counts for the exact
+    # algorithmic work; the inputs of the end-to-end leg)
+    vs0, res0 = lookup(want=("mat", "energy"))
     torch.cuda.synchronize()
+    if energy_shards:   # positions of other shards are not written: recompute the batch
+        _, full = g.lookup(0, L_cfg, want=("mat", "energy"))
+        e = full["energy"]
+        lo, hi = D.energy_shard_bounds(rank, world)
+        sel = (e >= lo) & (e < hi)
+        res0 = {"energy": e[sel].contiguous(), "mat": full["mat"][sel].contiguous()}
+        del full, e, sel
+    n_local = int(vs0[1])
     mats = torch.bincount(res0["mat"].long(), minlength=g.info.n_mats).cpu().tolist()
     num_nucs = g.table(X.XS_TABLE_NUM_NUCS).tolist()
     nuc_lookups = sum(c * n for c, n in zip(mats, num_nucs))
     idx_bytes = 4 if pre["grid_type"] == "unionized" else 8
     gather_bytes = nuc_lookups * (idx_bytes + 96)            # A4 + A5 per launch
-    search_bytes = L * 8 * math.ceil(math.log2(max(2, g.info.n_union - 1))) \
+    search_probes = math.ceil(math.log2(max(2, g.info.n_union - 1))) \
         if pre["grid_type"] == "unionized" else 0
-    balg_per_lookup = (gather_bytes + search_bytes) / L      # SURVEY §8(d) B_alg
+    search_bytes = n_local * 8 * search_probes
+    balg_per_lookup = (gather_bytes + search_bytes) / max(1, n_local)  # SURVEY §8(d) B_alg
     gold = golden().get(a.config)
-    hash_check = None
-    if gold and first == 0 and L == gold["lookups"]:
-        hash_check = (int(vs0[0]) == gold["sum_v_f32" if f32 else "sum_v"] and
-                      int(vs0[1]) == L)
 
     vsum = torch.zeros(2, dtype=torch.int64, device=dev)
+    a9 = [torch.cuda.Event(enable_timing=True) for _ in range(2 * (a.steps + a.warmup))]
+    a9_used = [0]
 
     def step():
         vsum.zero_()
-        g.lookup(first, L, sort=sort, vsum=vsum, f32=f32)
+        lookup(vsum=vsum)
         if world > 1:
+            q = a9_used[0]
+            if q + 1 < len(a9):
+                a9[q].record(stream)
             if a.backend == "nccl":
                 D.combine_vsum(vsum)      # A9 over NCCL (NVLink / NVSwitch)
             else:
                 vsum.copy_(D.combine_vsum(vsum.cpu()))
+            if q + 1 < len(a9):
+                a9[q + 1].record(stream)
+                a9_used[0] = q + 2
 
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
+    a9_used[0] = 0
     g.timing(True)
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        ev0.record(stream)
-        for _ in range(a.steps):
-            step()
-        ev1.record(stream)
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-    ms_local = ev0.elapsed_time(ev1)
+        ms_local, per_step = _timed_steps(step, stream, a.steps, world, dist)
     tm = g.timing_read()
     g.timing(False)
+    a9_ms = (sum(a9[q].elapsed_time(a9[q + 1]) for q in range(0, a9_used[0], 2)) /
+             max(1, a9_used[0] // 2)) if world > 1 else 0.0
     ms = D.max_over_ranks(ms_local, device=dev if a.backend == "nccl" else None)
+    med = statistics.median(per_step)
+    med_max = D.max_over_ranks(med, device=dev if a.backend == "nccl" else None)
     total_lookups = L * world * a.steps if a.scaling == "weak" else L_cfg * a.steps
     value = total_lookups / (ms / 1e3)
     vglob = [int(x) for x in vsum.cpu()]
+    hash_check = None
+    if gold and vglob[1] == gold["lookups"] and (a.scaling == "strong" or world == 1):
+        hash_check = vglob == [gold["sum_v_f32" if f32 else "sum_v"], gold["lookups"]]
 
     peak, peak_src = measured_peaks()
     gather_ms = tm["ms_gather"] / max(1, tm["calls"])
@@ -668,14 +750,15 @@ def run_ours(a, pre, cfg):
     traffic_per_lookup, traffic_src = ncu_traffic(a.config, sort)
     roofline_hbm = {"bound": "hbm", "kernel": GATHER_KERNEL[sort], "achieved": achieved,
                     "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                    "traffic": traffic_per_lookup * L if traffic_per_lookup else None,
+                    "traffic": traffic_per_lookup * n_local if traffic_per_lookup else None,
                     "peak_source": peak_src,
                     "algorithmic_bytes_per_launch": gather_bytes,
                     "gather_ms_per_launch": gather_ms,
                     "traffic_source": traffic_src,
                     "note": "algorithmic bytes = sum over lookups of n_nuclides(mat) x "
-                            f"({idx_bytes} B index + 96 B record pair); L2/L1/shared-memory "
-                            "reuse lets frac exceed 1"}
+                            f"({idx_bytes} B index + 96 B record pair); on sorted batches the "
+                            "pairs are re-read from shared memory and L2, so frac > 1 measures "
+                            "reuse, not HBM bandwidth (traffic = DRAM bytes per launch, ncu)"}
     if sort:
         # energy-sorted batches re-read each record pair from shared memory for
         # ~40 lookups: the staged gather is bound by the FP64 pipe
@@ -701,14 +784,19 @@ def run_ours(a, pre, cfg):
 
     line = {"metric": "XS lookups/sec", "value": value, "unit": "lookups/s", "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps,
+            "ms_per_step_median": med_max,
             "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None,
-            "dtype": "f32" if f32 else "f64", "data": "synthetic", "config": cfg,
+            "dtype": "f32" if f32 else "f64", "data": "synthetic",
+            "config": dict(cfg, shard=("energy ranges [r/R, (r+1)/R) of all L lookups "
+                                       "(xs_lookup_batch_shard)" if energy_shards else
+                                       "contiguous lookup-id ranges")),
             "roofline": roofline,
             "roofline_hbm": roofline_hbm,
             "hbm_gather_roofline_frac_8TBs": step_frac,
             "balg_bytes_per_lookup": balg_per_lookup,
             "phase_ms_per_step": {k: tm[k] / max(1, tm["calls"])
                                   for k in ("ms_count", "ms_bucket", "ms_gather")},
+            "a9_allreduce_ms_per_step": a9_ms,
             "gpu_launches": int(tm["kernel_launches"]),
             "hash": D.global_hash(vglob), "lookups_per_step": vglob[1],
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
@@ -729,18 +817,51 @@ def run_ours(a, pre, cfg):
         dt = D.max_over_ranks(dt, device=dev if a.backend == "nccl" else None)
         e2e_total = L * world * a.e2e_steps if a.scaling == "weak" else L_cfg * a.e2e_steps
         line["e2e"] = {"value": e2e_total / dt, "unit": "lookups/s",
-                       "h2d_bytes_per_step": int(L * 9), "d2h_bytes_per_step": 16,
+                       "h2d_bytes_per_step": int(e_host.numel() * 9), "d2h_bytes_per_step": 16,
                        "api": "xs_lookup_explicit(XS_FLAG_HOST_IO | XS_FLAG_MAT_U8): pinned host "
                               "energy (f64) + material (u8) in, vsum out; wall clock per call "
                               "(the call synchronizes)",
                        "steps": a.e2e_steps,
                        "vsum_matches_batch": [int(x) for x in vs_h] == [int(x) for x in vs0]}
+        del e_host, m_host
     line["clocks"] = clk.summary()
+    # ------------------------------------------- single-GPU context legs
+    if world == 1 and not a.no_extras:
+        if sort and pre["lookups"] >= 1_000_000:
+            line["projection_strong"] = {
+                "note": "one-GPU projection of strong scaling (L fixed): each rank's shard "
+                        "timed alone on this GPU, R-GPU step = slowest shard; A9 (16-byte "
+                        "all-reduce) not included; weak scaling (L per rank, no exchange "
+                        "but A9) projects to R x value",
+                **strong_projection(g, L, f32, stream, value, ms / a.steps)}
+        # config 3 unsorted and the paper's kernel shape, as context
+        if sort and not f32:
+            g.timing(True)
+            ms_u = _time_fn(lambda: g.lookup(first, L, sort=False), stream, a.extra_steps)
+            tmu = g.timing_read()
+            g.timing(False)
+            gms = tmu["ms_gather"] / max(1, tmu["calls"])
+            tr, trs = ncu_traffic(a.config, False)
+            ach = gather_bytes / (gms / 1e3) / 1e9
+            line["unsorted"] = {
+                "value": L / (ms_u / 1e3), "ms_per_step": ms_u, "unit": "lookups/s",
+                "roofline": {"bound": "hbm", "kernel": GATHER_KERNEL[False], "achieved": ach,
+                             "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                             "gather_ms_per_launch": gms,
+                             "dram_bytes_per_lookup": tr, "traffic_source": trs,
+                             "dram_frac": (tr * L / (gms / 1e3) / 1e9 / peak) if tr else None}}
+            ms_b = _time_fn(lambda: g.lookup(first, L, baseline=True), stream, 3, warm=1)
+            line["paper_kernel_shape"] = {
+                "value": L / (ms_b / 1e3), "ms_per_step": ms_b, "unit": "lookups/s",
+                "what": "XS_FLAG_BASELINE: XSBench-CUDA shape (thread per lookup, id order, "
+                        "no bucketing), same exact arithmetic, on this B200"}
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         try:
             rate, cores, desc, S, n = oracle_sample_rate(pre, a.cpu_seconds, f32=f32)
+            rate1, _, desc1, _, _ = oracle_sample_rate(pre, a.cpu_seconds / 4, f32=f32, cores=1)
             line["cpu_baseline"] = {"value": rate, "unit": "lookups/s", "cores": cores,
-                                    "kind": "oracle", "sample": desc, "cpu": cpu_info()}
+                                    "kind": "oracle", "sample": desc, "cpu": cpu_info(),
+                                    "t1_value": rate1, "t1_sample": desc1}
         except Exception as e:  # the oracle is test infrastructure; report, don't fail
             line["cpu_baseline"] = {"value": None, "unit": "lookups/s", "cores": None,
                                     "kind": "oracle", "sample": f"failed: {e}"}
@@ -752,8 +873,30 @@ def run_ours(a, pre, cfg):
     return 0
 
 
+def _free_port() -> int:
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def self_launch(a) -> int | None:
+    """`bench.py --gpus N` outside torchrun: start N ranks (one per GPU) with
+    torch.distributed.run on 127.0.0.1 and relay rank 0's line."""
+    if a.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    import subprocess
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={a.gpus}", "--master-addr", "127.0.0.1",
+           "--master-port", str(_free_port()), os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     a = parse()
+    rc = self_launch(a)
+    if rc is not None:
+        return rc
     if a.config.startswith("rs-"):
         from paper_conf_sc_tianscd23_b200.rs import RS_PRESETS
         pre = dict(RS_PRESETS[a.config])

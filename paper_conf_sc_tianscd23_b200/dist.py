@@ -9,7 +9,10 @@ measurement, not part of the method.
 
 Scaling modes:
   weak   - every rank owns `per_rank` lookups: ids [r*per_rank, (r+1)*per_rank)
-  strong - a fixed total L split as [floor(r L / R), floor((r+1) L / R))
+  strong - a fixed total L split as [floor(r L / R), floor((r+1) L / R)), or
+           (sorted batches, bench.py's default) energy-range shards: every rank
+           samples all L lookups and looks up those with b_r <= p < b_{r+1}
+           (xs_lookup_batch_shard), so each keeps the full batch's density
 """
 from __future__ import annotations
 
@@ -27,6 +30,16 @@ def shard_range(rank: int, world: int, lookups: int, scaling: str = "weak") -> t
         b = (rank + 1) * lookups // world
         return a, b - a
     raise ValueError(f"unknown scaling {scaling!r}")
+
+
+def energy_shard_bounds(rank: int, world: int) -> tuple[float, float]:
+    """[lo, hi) of energy shard `rank` of `world` as xs_lookup_batch_shard
+    defines it: b_s = s / world in binary64, b_0 = -inf, b_world = +inf."""
+    if world < 1 or not 0 <= rank < world:
+        raise ValueError("bad rank/world")
+    lo = rank / world if rank > 0 else float("-inf")
+    hi = (rank + 1) / world if rank < world - 1 else float("inf")
+    return lo, hi
 
 
 def env_rank() -> tuple[int, int, int]:

@@ -386,6 +386,7 @@ def test_bench_multirank_path_on_one_gpu(X):
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
                         "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
                         "29541", "bench.py", "--gpus", "2", "--backend", "gloo", "--config", "small",
+                        "--scaling", "weak",
                         "--steps", "3", "--warmup", "3", "--no-cpu-baseline", "--no-e2e"],
                        cwd=root, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-2000:]
@@ -396,6 +397,29 @@ def test_bench_multirank_path_on_one_gpu(X):
     # ids [0, 34M): rank 0's shard is the golden small batch; the global sum
     # must equal the oracle's over both shards
     assert d["hash"] == (GOLDEN["small"]["sum_v"] + _small_second_shard_sum()) % 999983
+
+
+def test_bench_strong_energy_shards_on_one_gpu(X):
+    """bench.py's default multi-GPU mode (strong scaling, energy-range
+    shards) with two gloo ranks sharing the GPU, self-launched by
+    `bench.py --gpus 2` (no torchrun on the command line): the global
+    verification sum is the one-batch golden sum."""
+    import subprocess
+    import sys
+    root = os.path.dirname(HERE)
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--backend", "gloo",
+                        "--config", "small", "--steps", "3", "--warmup", "3",
+                        "--no-cpu-baseline", "--e2e-steps", "1"],
+                       cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong"
+    assert d["lookups_per_step"] == 17_000_000
+    assert d["hash"] == GOLDEN["small"]["hash"] and d["hash_matches_oracle"] is True
+    assert d["e2e"]["vsum_matches_batch"] is True
+    assert d["a9_allreduce_ms_per_step"] > 0
 
 
 def _small_second_shard_sum():
