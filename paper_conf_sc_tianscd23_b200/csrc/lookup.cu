@@ -27,6 +27,16 @@ namespace xs {
 
 __constant__ JumpTable c_jump;
 
+// pick_material(RN(s) * 2^-63) from the raw state (integer thresholds in
+// constant memory, common.cuh fill_pick_thresholds): 1 + #{k : s >= c_k},
+// 12 -> 0 (fuel)
+__device__ __forceinline__ int pick_material_state(uint64_t s) {
+  int c = 0;
+#pragma unroll
+  for (int k = 0; k < 11; ++k) c += s >= c_jump.pick[k] ? 1 : 0;
+  return c == 11 ? 0 : c + 1;
+}
+
 cudaError_t init_constants() {
   JumpTable t = make_jump_table();
   return cudaMemcpyToSymbol(c_jump, &t, sizeof(t));
@@ -57,7 +67,7 @@ __device__ __forceinline__ Sample sample_lookup(uint64_t seed, uint64_t id) {
   s = lcg_next(s);
   const double p = lcg_double(s);
   s = lcg_next(s);
-  return Sample{p, pick_material(lcg_double(s))};
+  return Sample{p, pick_material_state(s)};
 }
 
 struct Params {
@@ -261,7 +271,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_sample(Params P) {
         st = lcg_next(st);
         const double pe = lcg_double(st);
         st = lcg_next(st);
-        smp[it] = Sample{pe, pick_material(lcg_double(st))};
+        smp[it] = Sample{pe, pick_material_state(st)};
       }
       lo[it] = 0;
       hi[it] = P.NU - 1;
@@ -606,7 +616,7 @@ __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint6
       st = lcg_next(st);
       const double pe = lcg_double(st);
       st = lcg_next(st);
-      smp[it] = Sample{pe, pick_material(lcg_double(st))};
+      smp[it] = Sample{pe, pick_material_state(st)};
       ok[it] = ok[it] && in_shard(P, pe);
     }
   }
@@ -679,13 +689,17 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
 
 constexpr int kColIlp = 8;
 // H[t][key] -> exclusive prefix over tiles t (per key); key totals.  Block =
-// 32 keys x 32 slices of the tiles.
+// KX keys x SY slices of the tiles (KX * SY = 1024): few keys (energy-range
+// shards) take more slices per key so that the latency-bound column walks
+// spread over more SMs.
+template <int KX, int SY>
 __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
-  __shared__ uint32_t s_p[32][33];
+  static_assert(KX * SY == 1024, "block");
+  __shared__ uint32_t s_p[SY][KX + 1];
   const int nkeys = (P.n_mats + 1) * P.nkr;
-  const int key = blockIdx.x * 32 + threadIdx.x;
+  const int key = blockIdx.x * KX + threadIdx.x;
   const int sl = threadIdx.y;
-  const int per = (nb + 31) / 32;
+  const int per = (nb + SY - 1) / SY;
   const int b0 = sl * per, b1 = min(nb, b0 + per);
   // both passes keep kColIlp loads in flight (the rows are nkeys * 4 B apart;
   // a dependent walk is latency-bound at XL's 20k tiles)
@@ -703,7 +717,7 @@ __global__ void __launch_bounds__(1024) k_part_colscan(Params P, int nb) {
   __syncthreads();
   if (sl == 0) {
     uint32_t run = 0;
-    for (int q = 0; q < 32; ++q) {
+    for (int q = 0; q < SY; ++q) {
       const uint32_t v = s_p[q][threadIdx.x];
       s_p[q][threadIdx.x] = run;
       run += v;
@@ -2235,6 +2249,293 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   }
 }
 
+// ------------------------------------------- k_gather_s4 (staged, LDGSTS) --
+// The staged gather of k_gather_s3 with a cheaper producer: the windows of a
+// group of D nuclides are packed back to back into one of two per-warp
+// buffers of C interval entries, copied by all 32 lanes at once with 16-B
+// cp.async (32/D lanes per nuclide, no per-copy elected issue), completing
+// on the buffer's mbarrier (one cp.async arrive per lane).  Each nuclide's
+// place in its group buffer is a segmented warp scan of the window sizes,
+// done in the A4 prologue.  A window that does not fit its group's buffer is
+// read in place from global memory (rare: C is ~1.5x a group's mean size).
+// The material table is staged packed (CSR) instead of [n_mats][max_nucs].
+// Arithmetic, operation order and results are those of k_gather_s3 (R10/R11,
+// R18 for F32).
+struct alignas(16) NucWin {
+  int32_t klo, khi;   // bracket range of the task's extreme energies (A4)
+  uint32_t noff;      // n * N
+  uint32_t off;       // entry offset in the group buffer, kNoBuf = read in place
+};
+constexpr uint32_t kNoBuf = 0xffffffffu;
+
+struct alignas(16) GatherSmem4 {
+  int32_t num[kMaxMats];
+  uint32_t off[kMaxMats + 1];   // bucket start of material m
+  uint32_t cnt[kMaxMats];
+  uint32_t toff[kMaxMats + 1];  // first task of material m
+  uint32_t roff[kMaxMats + 1];  // first table entry of material m (CSR)
+};
+
+template <int C, int NW, bool F32>
+__host__ __device__ constexpr size_t s4_warp_bytes(int max_nucs) {
+  return 2 * static_cast<size_t>(C) * (F32 ? kIv32Doubles : kIvDoubles) * 8 +  // buffers
+         static_cast<size_t>(max_nucs) * sizeof(NucWin) + 16;                   // windows + bars
+}
+
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
+  if (gated_off(P)) return;
+  using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
+  constexpr int kTask = 32 * R;
+  constexpr int kE = Acc::kE;            // 16-B units per interval entry
+  constexpr int LPN = 32 / D;            // copying lanes per nuclide
+  static_assert(D >= 1 && D <= 32 && (32 % D) == 0, "group size divides the warp");
+  static_assert(C <= 255, "buffer offsets");
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem4& G = *reinterpret_cast<GatherSmem4*>(smem_raw);
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem4));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0, roff = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      G.num[m] = P.num_nucs[m];
+      G.off[m] = run;
+      G.cnt[m] = c;
+      G.toff[m] = trun;
+      G.roff[m] = roff;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+      roff += static_cast<uint32_t>(P.num_nucs[m]);
+    }
+    G.off[P.n_mats] = run;
+    G.toff[P.n_mats] = trun;
+    G.roff[P.n_mats] = roff;
+  }
+  __syncthreads();
+  const int tab = static_cast<int>(G.roff[P.n_mats]);
+  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
+    int m = 0;
+    while (static_cast<uint32_t>(i) >= G.roff[m + 1]) ++m;
+    const int src = m * P.max_nucs + (i - static_cast<int>(G.roff[m]));
+    const int32_t n = P.mats[src];
+    MatEntry me;
+    me.conc = P.concs[src];
+    me.noff = static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N);
+    me.n = n;
+    s_tab[i] = me;
+  }
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab) + ((tab * sizeof(MatEntry) + 15) / 16) * 16;
+  unsigned char* mine = wbase + s4_warp_bytes<C, NW, F32>(P.max_nucs) * warp;
+  double2* s_buf = reinterpret_cast<double2*>(mine);                            // [2][C * kE]
+  NucWin* s_k = reinterpret_cast<NucWin*>(mine + 2 * static_cast<size_t>(C) * kE * 16);
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(s_k + P.max_nucs);              // [2]
+  if (lane == 0) {
+    mbar_init(&s_bar[0], 32);
+    mbar_init(&s_bar[1], 32);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = G.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(F32 ? P.iv32 : P.iv);
+  uint32_t phase = 0;  // parity bit per buffer
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+    while (task >= G.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
+    double p[R];
+    int32_t gidx[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < G.cnt[m];
+      LookupRec rec{0.5, 0u, 0};
+      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
+      p[r] = rec.p;
+      gidx[r] = rec.gidx;
+      idx[r] = rec.idx;
+    }
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const int32_t tg = gidx[r]; gidx[r] = gidx[r + 1]; gidx[r + 1] = tg;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    double plo = valid[0] ? p[0] : 2.0, phi = -1.0;
+    int32_t ulo = valid[0] ? gidx[0] : 0x7fffffff, uhi = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid[r]) {
+        phi = p[r];
+        uhi = gidx[r];
+      }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double a = __shfl_xor_sync(0xffffffffu, plo, o);
+      const double b = __shfl_xor_sync(0xffffffffu, phi, o);
+      plo = a < plo ? a : plo;
+      phi = b > phi ? b : phi;
+    }
+    if (GT == XS_GRID_UNIONIZED && !P.need_gidx) {
+      ulo = union_lower_tab(P, plo);
+      uhi = union_upper_tab(P, phi);
+    } else {
+      ulo = __reduce_min_sync(0xffffffffu, ulo);
+      uhi = __reduce_max_sync(0xffffffffu, uhi);
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
+    const int nn = G.num[m];
+    const MatEntry* row = s_tab + G.roff[m];
+    // A4 for the two extremes of every nuclide, and each window's place in
+    // its group buffer (segmented scan of the sizes over groups of D lanes;
+    // 32 nuclides per round, so groups never straddle rounds)
+    for (int j0 = 0; j0 < nn; j0 += 32) {
+      const int j = j0 + lane;
+      int32_t klo = 0, khi = 0;
+      uint32_t noff = 0;
+      if (j < nn) {
+        const MatEntry me = row[j];
+        noff = me.noff;
+        if (GT == XS_GRID_UNIONIZED) {
+          if (P.index_t) {
+            klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
+            khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
+          } else {
+            klo = __ldg(P.index + static_cast<int64_t>(ulo) * P.I + me.n);
+            khi = __ldg(P.index + static_cast<int64_t>(uhi) * P.I + me.n);
+          }
+        } else {
+          const RowView<GT> rlo(P, GT == XS_GRID_HASH ? hash_bin(plo, P.du, P.B) : 0);
+          const RowView<GT> rhi(P, GT == XS_GRID_HASH ? hash_bin(phi, P.du, P.B) : 0);
+          klo = rlo.bracket(P, me.n, me.noff, plo);
+          khi = rhi.bracket(P, me.n, me.noff, phi);
+        }
+      }
+      const int32_t n_int = khi - klo;
+      const int size = (j < nn && n_int < C) ? n_int + 1 : 0;
+      int incl = size;
+#pragma unroll
+      for (int o = 1; o < D; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if ((lane & (D - 1)) >= o) incl += v;
+      }
+      if (j < nn) {
+        NucWin w;
+        w.klo = klo;
+        w.khi = khi;
+        w.noff = noff;
+        w.off = (size > 0 && incl <= C) ? static_cast<uint32_t>(incl - size) : kNoBuf;
+        s_k[j] = w;
+      }
+    }
+    __syncwarp();
+    // A5 producer: all lanes copy group g's windows (LPN lanes per nuclide,
+    // 16 B per cp.async) into buffer g & 1, then arrive on its mbarrier
+    auto issue_group = [&](int g) {
+      if (g * D >= nn) return;  // warp-uniform
+      const int j = g * D + lane / LPN;
+      if (j < nn) {
+        const NucWin w = s_k[j];
+        if (w.off != kNoBuf) {
+          const double2* src = iv2 + static_cast<uint64_t>(w.noff + static_cast<uint32_t>(w.klo)) * kE;
+          double2* dst = s_buf + (g & 1) * (C * kE) + w.off * kE;
+          const int nch = (w.khi - w.klo + 1) * kE;
+          for (int c = lane % LPN; c < nch; c += LPN) cp_async16(dst + c, src + c);
+        }
+      }
+      cp_async_mbar_arrive(&s_bar[g & 1]);
+    };
+    issue_group(0);
+    issue_group(1);
+
+    Acc acc;
+    acc.zero();
+    for (int j = 0; j < nn; ++j) {
+      if (j % D == 0) {
+        const int g = j / D;
+        if (g >= 1) {
+          __syncwarp();  // every lane is done with buffer (g + 1) & 1 (group g - 1)
+          issue_group(g + 1);
+        }
+        mbar_wait(&s_bar[g & 1], (phase >> (g & 1)) & 1u);
+        phase ^= 1u << (g & 1);
+      }
+      const NucWin w = s_k[j];
+      const double conc = row[j].conc;
+      const int n_int = w.khi - w.klo;
+      if (w.off != kNoBuf) {
+        stage_nuclide_iv<R, true>(s_buf + ((j / D) & 1) * (C * kE) + w.off * kE, n_int, conc, p, acc);
+      } else {
+        const double2* g2 = iv2 + static_cast<uint64_t>(w.noff + static_cast<uint32_t>(w.klo)) * kE;
+        stage_nuclide_iv<R, false>(g2, n_int, conc, p, acc);
+      }
+      if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
+    }
+    if (nn & (kF32Block - 1)) acc.flush();
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (acc.get(r, c) > mx) {
+          mx = acc.get(r, c);
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = acc.get(r, c);
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -2466,6 +2767,31 @@ static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false>
+static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  int tab = 0;
+  {
+    // packed material table size: launch-time upper bound n_mats * max_nucs
+    // would waste shared memory; the kernel packs sum(num_nucs) entries
+    tab = g.tab_total;
+  }
+  const size_t smem = sizeof(GatherSmem4) + ((static_cast<size_t>(tab) * sizeof(MatEntry) + 15) / 16) * 16 +
+                      NW * s4_warp_bytes<C, NW, F32>(g.max_nucs);
+  auto kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32>;
+  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
@@ -2482,7 +2808,7 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   int v = g.unroll;
   if (v == 0) {
     const double d = static_cast<double>(g.N) * 128.0 / static_cast<double>(P.count ? P.count : 1);
-    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : 25;
+    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : 40;
   }
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
@@ -2505,6 +2831,13 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 26: return launch_gather_s3<GT, 4, 4, 6, 20, CHECK>(g, P, st);
     case 27: return launch_gather_s3<GT, 4, 2, 6, 24, CHECK>(g, P, st);
     case 28: return launch_gather_s3<GT, 4, 4, 4, 16, CHECK>(g, P, st);
+    // k_gather_s4 (R, D, C, NW): LDGSTS-staged group buffers
+    case 40: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK>(g, P, st);
+    case 41: return launch_gather_s4<GT, 4, 8, 20, 20, CHECK>(g, P, st);
+    case 42: return launch_gather_s4<GT, 4, 4, 12, 16, CHECK>(g, P, st);
+    case 43: return launch_gather_s4<GT, 4, 4, 12, 20, CHECK>(g, P, st);
+    case 44: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK>(g, P, st);
+    case 45: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
@@ -2520,7 +2853,10 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
     case 31: return launch_gather_s3<GT, 4, 2, 8, 16, CHECK, false, true>(g, P, st);
     case 34: return launch_gather_s3<GT, 4, 2, 8, 20, CHECK, false, true>(g, P, st);
     case 36: return launch_gather_s3<GT, 4, 4, 6, 24, CHECK, false, true>(g, P, st);
-    default: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
+    case 35: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
+    case 47: return launch_gather_s4<GT, 4, 8, 20, 20, CHECK, true>(g, P, st);
+    case 48: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK, true>(g, P, st);
+    default: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true>(g, P, st);  // = 46
   }
 }
 
@@ -2678,7 +3014,8 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.tmp = ws.tmp;
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
-  const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28);
+  const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
+                      (variant >= 40 && variant <= 48);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)
@@ -2717,7 +3054,12 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     const size_t hs = static_cast<size_t>(nkeys) * 4;
     k_part_count<GT><<<nb, kPrepThreads, hs, st>>>(P);
     mark(1);
-    k_part_colscan<<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));
+    if (nkeys >= 32 * 148)
+      k_part_colscan<32, 32><<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));
+    else if (nkeys >= 8 * 148)
+      k_part_colscan<8, 128><<<(nkeys + 7) / 8, dim3(8, 128), 0, st>>>(P, static_cast<int>(ntiles));
+    else
+      k_part_colscan<2, 512><<<(nkeys + 1) / 2, dim3(2, 512), 0, st>>>(P, static_cast<int>(ntiles));
     k_part_keyscan<<<1, 1024, 0, st>>>(P);
     {
       const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup);
@@ -2794,7 +3136,7 @@ __global__ void k_hist_init(uint64_t seed, uint64_t first, uint32_t n, int32_t L
     s = lcg_next(s);
     E[q] = lcg_double(s);
     s = lcg_next(s);
-    mat[q] = pick_material(lcg_double(s));
+    mat[q] = pick_material_state(s);
     st[q] = s;
   }
 }
@@ -2828,7 +3170,7 @@ __global__ void k_hist_advance(HistoryArgs h, int32_t i) {
     s = lcg_next(s);
     h.hist_energy[q] = lcg_double(s);
     s = lcg_next(s);
-    h.hist_mat[q] = pick_material(lcg_double(s));
+    h.hist_mat[q] = pick_material_state(s);
     h.hist_state[q] = s;
   }
 }

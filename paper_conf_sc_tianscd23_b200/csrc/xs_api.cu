@@ -228,6 +228,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   G.N = N;
   G.n_mats = d->n_mats;
   G.max_nucs = d->max_num_nucs;
+  for (int32_t m = 0; m < d->n_mats; ++m) G.tab_total += d->num_nucs[m];
   G.grid_type = d->grid_type;
   G.B = d->grid_type == XS_GRID_HASH ? d->hash_bins : 0;
   G.du = G.B ? 1.0 / static_cast<double>(G.B) : 0.0;
@@ -704,8 +705,9 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   DeviceGrid& G = g->d;
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
-          (value >= 17 && value <= 28) || (value >= 31 && value <= 36)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28 or 31-36");
+          (value >= 17 && value <= 28) || (value >= 31 && value <= 36) ||
+          (value >= 40 && value <= 48)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-48");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");

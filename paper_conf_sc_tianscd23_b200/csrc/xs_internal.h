@@ -27,6 +27,7 @@ struct DeviceGrid {
   int32_t I = 0;
   int64_t N = 0;
   int32_t n_mats = 0, max_nucs = 0;
+  int32_t tab_total = 0;     // sum of num_nucs (packed material table entries)
   int32_t grid_type = 0, B = 0;
   double du = 0.0;
   uint64_t lookup_seed = 0;
