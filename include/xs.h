@@ -158,6 +158,19 @@ typedef struct {
 #define XS_FLAG_MAT_U8 0x10u  /* xs_lookup_explicit: `mat` points to uint8_t[count]
                                  (a material id per byte) instead of int32_t —
                                  a quarter of the material bytes to upload    */
+#define XS_FLAG_HOST_ASYNC 0x20u /* like XS_FLAG_HOST_IO (host pointers in and out),
+                                 but the call does not wait: the inputs are
+                                 uploaded on the library's copy stream and the
+                                 outputs (vsum included) are copied back on
+                                 `cuda_stream`; the caller keeps the host
+                                 buffers and the workspace alive and
+                                 unmodified, and synchronizes `cuda_stream`
+                                 before reading outputs.  The upload of one
+                                 call overlaps the lookups of the previous
+                                 call when the two use different workspaces
+                                 (a workspace's staging area is reused only
+                                 after the call that last used it is done).
+                                 Not combinable with XS_FLAG_HOST_IO.        */
 
 /* tables for xs_get_table (element type in brackets) */
 #define XS_TABLE_NUCLIDE_GRID 0 /* [double] I*N*6                               */

@@ -26,6 +26,7 @@
 namespace xs {
 
 __constant__ JumpTable c_jump;
+__device__ uint4 g_pick_tab[256];  // pick_material per 2^51-state bucket (below), 4096 B
 
 // pick_material(RN(s) * 2^-63) from the raw state (integer thresholds in
 // constant memory, common.cuh fill_pick_thresholds): 1 + #{k : s >= c_k},
@@ -37,9 +38,43 @@ __device__ __forceinline__ int pick_material_state(uint64_t s) {
   return c == 11 ? 0 : c + 1;
 }
 
+// The same through a 4096-bucket table of the top 12 state bits (built at
+// init by make_pick_table, staged in shared memory per block): a bucket
+// whose first and last state pick the same material picks it everywhere
+// (the count above is monotone in s); the 11 buckets holding a threshold
+// say kPickExact and take the compares.
+constexpr int kPickBuckets = 4096;
+constexpr uint8_t kPickExact = 0xff;
+__device__ __forceinline__ void pick_table_fill(uint8_t* t) {
+  for (int b = threadIdx.x; b < kPickBuckets / 16; b += blockDim.x)
+    reinterpret_cast<uint4*>(t)[b] = g_pick_tab[b];
+}
+__device__ __forceinline__ int pick_material_tab(const uint8_t* t, uint64_t s) {
+  const int m = t[s >> 51];
+  return m != kPickExact ? m : pick_material_state(s);
+}
+
+// host: the bucket table of pick_material_tab (same integer decision)
+static void make_pick_table(const JumpTable& t, uint8_t* out) {
+  auto pick = [&](uint64_t s) {
+    int c = 0;
+    for (int k = 0; k < 11; ++k) c += s >= t.pick[k] ? 1 : 0;
+    return c == 11 ? 0 : c + 1;
+  };
+  for (int b = 0; b < 4096; ++b) {
+    const uint64_t lo = static_cast<uint64_t>(b) << 51, hi = lo + ((1ull << 51) - 1);
+    const int a = pick(lo), z = pick(hi);
+    out[b] = a == z ? static_cast<uint8_t>(a) : 0xff;
+  }
+}
+
 cudaError_t init_constants() {
   JumpTable t = make_jump_table();
-  return cudaMemcpyToSymbol(c_jump, &t, sizeof(t));
+  cudaError_t e = cudaMemcpyToSymbol(c_jump, &t, sizeof(t));
+  if (e != cudaSuccess) return e;
+  alignas(16) uint8_t tab[4096];
+  make_pick_table(t, tab);
+  return cudaMemcpyToSymbol(g_pick_tab, tab, sizeof(tab));
 }
 
 // ------------------------------------------------------------------ A1 ----
@@ -119,6 +154,8 @@ struct Params {
   int kc_lo;
   int shard;            // 1: only lookups with e_lo <= p < e_hi are looked up
   double e_lo, e_hi;    //    (energy-range shard, xs_lookup_batch_shard)
+  double* slab_p;       // shard mode: k_part_count keeps the tile's lookups of the
+  uint64_t* slab_k;     // shard (energy; position << 16 | key) for k_part_place
   int fine_direct;      // k_part_fine scatters directly above this many windows
   int fine_cap;         // k_part_fine window (lookups)
   uint32_t* key_tot;    // [nkeys] lookups per coarse key
@@ -603,8 +640,8 @@ __device__ __forceinline__ bool in_shard(const Params& P, double p) {
 // assignment in k_part_count and k_part_place).  sc = stream state at the
 // chunk's first lookup, tA, tC = LCG^(2 kPartItems t).
 __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint64_t sc, uint64_t tA,
-                                             uint64_t tC, Sample (&smp)[kPartItems],
-                                             bool (&ok)[kPartItems]) {
+                                             uint64_t tC, const uint8_t* s_pick,
+                                             Sample (&smp)[kPartItems], bool (&ok)[kPartItems]) {
   uint64_t st = (tA * sc + tC) & kMask63;
 #pragma unroll
   for (int it = 0; it < kPartItems; ++it) {
@@ -616,7 +653,7 @@ __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint6
       st = lcg_next(st);
       const double pe = lcg_double(st);
       st = lcg_next(st);
-      smp[it] = Sample{pe, pick_material_state(st)};
+      smp[it] = Sample{pe, pick_material_tab(s_pick, st)};
       ok[it] = ok[it] && in_shard(P, pe);
     }
   }
@@ -650,8 +687,12 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
   const bool outputs = P.out_E || P.out_mat || P.out_gidx || P.out_M || P.out_v;
   PartStream ps;
   ps.init(P);
+  __shared__ uint32_t s_kept;
+  __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
+  pick_table_fill(s_pick);  // (first use after the tile loop's barrier)
   for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
     for (int t = threadIdx.x; t < nkeys; t += blockDim.x) s_h[t] = 0;
+    if (threadIdx.x == 0) s_kept = 0;
     __syncthreads();
     uint64_t sc = ps.at(P, tl * tlen);
     for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
@@ -659,11 +700,18 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
       if (c0 >= P.count) break;
       Sample smp[kPartItems];
       bool ok[kPartItems];
-      part_samples(P, c0, sc, ps.tA, ps.tC, smp, ok);
+      part_samples(P, c0, sc, ps.tA, ps.tC, s_pick, smp, ok);
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
         if (!ok[it]) continue;
-        atomicAdd(&s_h[part_key(P, smp[it])], 1u);
+        const uint32_t key = part_key(P, smp[it]);
+        atomicAdd(&s_h[key], 1u);
+        if (P.slab_p && smp[it].mat < P.n_mats) {  // shard: keep it for k_part_place
+          const uint32_t q = atomicAdd(&s_kept, 1u);
+          const uint64_t at = static_cast<uint64_t>(tl) * tlen + q;
+          P.slab_p[at] = smp[it].p;
+          P.slab_k[at] = ((c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it) << 16) | key;
+        }
         if (!outputs) continue;
         const uint32_t i = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
         const bool valid = smp[it].mat < P.n_mats;
@@ -780,6 +828,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
   double* s_p = reinterpret_cast<double*>(smem_pl + ((3 * static_cast<size_t>(nkeys) + 1) * 4 + 15) / 16 * 16);
   uint16_t* s_k = reinterpret_cast<uint16_t*>(s_p + tlen);
   uint32_t* s_i = reinterpret_cast<uint32_t*>(s_k + tlen);
+  __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
+  pick_table_fill(s_pick);  // (first use after the tile loop's barrier)
   PartStream ps;
   ps.init(P);
   for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
@@ -801,13 +851,24 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
     }
     __syncthreads();
     const uint32_t nloc = s_ls[nvalid];  // valid lookups of the tile
+    if (P.slab_p) {  // shard: the tile's lookups of the shard, kept by k_part_count
+      for (uint32_t i = threadIdx.x; i < nloc; i += kPrepThreads) {
+        const uint64_t at = static_cast<uint64_t>(tl) * tlen + i;
+        const uint64_t kk = P.slab_k[at];
+        const uint32_t key = static_cast<uint32_t>(kk & 0xffffu);
+        const uint32_t q = atomicAdd(&s_lc[key], 1u);
+        s_p[q] = P.slab_p[at];
+        s_k[q] = static_cast<uint16_t>(key);
+        if (P.sidx_tmp) s_i[q] = static_cast<uint32_t>(kk >> 16);
+      }
+    }
     uint64_t sc = ps.at(P, tl * tlen);
-    for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
+    for (uint32_t c = 0; c < tchunks && !P.slab_p; ++c, sc = ps.next(sc)) {
       const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
       if (c0 >= P.count) break;
       Sample smp[kPartItems];
       bool ok[kPartItems];
-      part_samples(P, c0, sc, ps.tA, ps.tC, smp, ok);
+      part_samples(P, c0, sc, ps.tA, ps.tC, s_pick, smp, ok);
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
         if (!ok[it] || smp[it].mat >= P.n_mats) continue;  // invalid lookups are not gathered
@@ -2928,7 +2989,7 @@ static size_t part_place_smem(uint64_t count, int32_t n_mats, int cbits, bool pe
 
 bool part_cbits_fit(uint64_t count, int32_t n_mats, int cbits) {
   return cbits >= kPartCbitsMin && cbits <= kPartCbitsMax && (static_cast<size_t>(n_mats + 1) << cbits) <= 65536 &&
-         part_place_smem(count, n_mats, cbits, true) <= 227 * 1024;
+         part_place_smem(count, n_mats, cbits, true) + kPickBuckets + 64 <= 227 * 1024;
 }
 
 static int part_cbits(uint64_t count, int32_t n_mats, int requested) {
@@ -3051,6 +3112,14 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     double* sp = reinterpret_cast<double*>(ws.recs);
     P.sp = sp;
     P.sidx = per_lookup ? reinterpret_cast<uint32_t*>(sp + a.count) : nullptr;
+    // shard mode: k_part_count keeps the shard's lookups of tile t at slots
+    // t * tlen + q, q < the tile's lookups (so every slot is < count): energy
+    // and (position << 16 | key) in the record area (16 B per lookup), which
+    // k_part_fine writes only after k_part_place has read them
+    if (a.shard) {
+      P.slab_p = sp;
+      P.slab_k = reinterpret_cast<uint64_t*>(sp + a.count);
+    }
     const size_t hs = static_cast<size_t>(nkeys) * 4;
     k_part_count<GT><<<nb, kPrepThreads, hs, st>>>(P);
     mark(1);

@@ -25,6 +25,8 @@ struct xs_grid {
   uint64_t host_chunk = 10000000;  // host-input chunk (lookups), measured on B200 (large)
   cudaStream_t copy_stream = nullptr;
   std::vector<cudaEvent_t> chunk_ev;
+  // XS_FLAG_HOST_ASYNC: per workspace, the event after the last call that used it
+  std::vector<std::pair<const void*, cudaEvent_t>> ws_done;
   // per-phase event timing (xs_timing_enable / xs_timing_read)
   bool timing = false;
   std::vector<std::array<cudaEvent_t, 4>> ev;
@@ -153,7 +155,7 @@ static size_t staging_layout(uint64_t count, void* base, Staging* s) {
 
 static size_t total_workspace(uint64_t count, uint32_t flags, int32_t n_mats) {
   size_t w = workspace_layout(count, flags, n_mats, nullptr, nullptr);
-  if (flags & XS_FLAG_HOST_IO) w += staging_layout(count, nullptr, nullptr);
+  if (flags & (XS_FLAG_HOST_IO | XS_FLAG_HOST_ASYNC)) w += staging_layout(count, nullptr, nullptr);
   return w;
 }
 
@@ -415,8 +417,13 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   if (!g || !out) return fail(XS_ERR_INVALID_ARG, "NULL grid/outputs");
   if (!out->vsum) return fail(XS_ERR_INVALID_ARG, "outputs.vsum is required");
   if (count >= (1ULL << 32)) return fail(XS_ERR_INVALID_ARG, "count must be < 2^32");
-  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE | XS_FLAG_F32 | XS_FLAG_MAT_U8))
+  if (flags & ~(XS_FLAG_SORT | XS_FLAG_HOST_IO | XS_FLAG_BASELINE | XS_FLAG_F32 | XS_FLAG_MAT_U8 |
+                XS_FLAG_HOST_ASYNC))
     return fail(XS_ERR_INVALID_ARG, "unknown flag bits");
+  if ((flags & XS_FLAG_HOST_ASYNC) && (flags & XS_FLAG_HOST_IO))
+    return fail(XS_ERR_INVALID_ARG, "XS_FLAG_HOST_ASYNC and XS_FLAG_HOST_IO are exclusive");
+  const bool async_io = (flags & XS_FLAG_HOST_ASYNC) != 0;
+  if (async_io) flags = (flags & ~XS_FLAG_HOST_ASYNC) | XS_FLAG_HOST_IO;  // same staging
   if ((flags & XS_FLAG_MAT_U8) && !energy)
     return fail(XS_ERR_INVALID_ARG, "XS_FLAG_MAT_U8 applies to explicit lookups only");
   const bool mat8 = (flags & XS_FLAG_MAT_U8) != 0;
@@ -463,10 +470,37 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
   // equal chunks of at most host_chunk lookups
   const uint64_t nch = (count + g->host_chunk - 1) / g->host_chunk;
   const uint64_t chunk = (count + nch - 1) / nch;
-  const bool chunked = host_io && energy && nch > 1;
+  const bool chunked = host_io && energy && nch > 1 && !async_io;
+  cudaEvent_t ws_ev = nullptr;  // async: completion of the last call on this workspace
+  if (async_io) {
+    for (auto& pr : g->ws_done)
+      if (pr.first == workspace) ws_ev = pr.second;
+    if (!ws_ev) {
+      XS_TRY(cudaEventCreateWithFlags(&ws_ev, cudaEventDisableTiming), "cudaEventCreate");
+      g->ws_done.emplace_back(workspace, ws_ev);
+      XS_TRY(cudaEventRecord(ws_ev, st), "event");
+    }
+    if (!g->copy_stream)
+      XS_TRY(cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking), "copy stream");
+    if (g->chunk_ev.empty()) {
+      cudaEvent_t ev;
+      XS_TRY(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming), "cudaEventCreate");
+      g->chunk_ev.push_back(ev);
+    }
+  }
   if (host_io) {
     staging_layout(count, static_cast<char*>(workspace) + wbytes, &sg);
-    if (energy && !chunked) {
+    if (energy && async_io) {
+      // upload on the copy stream once the workspace's previous call is done,
+      // overlapping whatever the caller's stream is still running
+      XS_TRY(cudaStreamWaitEvent(g->copy_stream, ws_ev, 0), "wait");
+      XS_TRY(cudaMemcpyAsync(sg.energy, energy, count * 8, cudaMemcpyHostToDevice, g->copy_stream),
+             "H2D energy");
+      XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * mat_es, cudaMemcpyHostToDevice, g->copy_stream),
+             "H2D mat");
+      XS_TRY(cudaEventRecord(g->chunk_ev[0], g->copy_stream), "event");
+      XS_TRY(cudaStreamWaitEvent(st, g->chunk_ev[0], 0), "wait");
+    } else if (energy && !chunked) {
       XS_TRY(cudaMemcpyAsync(sg.energy, energy, count * 8, cudaMemcpyHostToDevice, st), "H2D energy");
       XS_TRY(cudaMemcpyAsync(sg.mat, mat, count * mat_es, cudaMemcpyHostToDevice, st), "H2D mat");
     }
@@ -539,7 +573,10 @@ static xs_status lookup_common(xs_grid* g, uint64_t first_id, const double* ener
               {out->verification, sg.v, count * 4}, {out->vsum, sg.vsum, 16}};
     for (auto& c : cp)
       if (c.dst) XS_TRY(cudaMemcpyAsync(c.dst, c.src, c.n, cudaMemcpyDeviceToHost, st), "D2H output");
-    XS_TRY(cudaStreamSynchronize(st), "lookup (host io) completion");
+    if (async_io)
+      XS_TRY(cudaEventRecord(ws_ev, st), "event");
+    else
+      XS_TRY(cudaStreamSynchronize(st), "lookup (host io) completion");
   }
   return XS_OK;
 }
@@ -774,6 +811,7 @@ void xs_free_grid(xs_grid* g) {
   for (auto& e : g->ev)
     for (auto x : e) cudaEventDestroy(x);
   for (auto x : g->chunk_ev) cudaEventDestroy(x);
+  for (auto& pr : g->ws_done) cudaEventDestroy(pr.second);
   if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
   cudaFree(g->d.grid);
   cudaFree(g->d.iv);

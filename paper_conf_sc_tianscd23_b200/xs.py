@@ -22,6 +22,7 @@ XS_ABI_VERSION = 1
 XS_GRID_UNIONIZED, XS_GRID_NUCLIDE, XS_GRID_HASH = 0, 1, 2
 XS_FLAG_SORT, XS_FLAG_HOST_IO, XS_FLAG_BASELINE, XS_FLAG_F32 = 0x1, 0x2, 0x4, 0x8
 XS_FLAG_MAT_U8 = 0x10
+XS_FLAG_HOST_ASYNC = 0x20
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
  XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T, XS_TABLE_INTERVALS,
  XS_TABLE_INTERVALS32) = range(9)
@@ -304,6 +305,9 @@ class Grid:
         t = xs_timing_read(self._h)
         return {k: getattr(t, k) for k, _ in xs_timing._fields_}
 
+    def workspace_size(self, count: int, flags: int = 0) -> int:
+        return xs_workspace_size(self._h, count, flags)
+
     def workspace(self, count: int, flags: int = 0):
         import torch
         n = xs_workspace_size(self._h, count, flags)
@@ -375,21 +379,28 @@ class Grid:
                               ws.data_ptr(), ws.numel(), self._stream())
         return vsum, res
 
-    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, f32: bool = False):
+    def lookup_explicit(self, energy, mat, sort=False, want=(), vsum=None, f32: bool = False,
+                        asynchronous: bool = False, workspace=None):
         """A2-A8 for caller-given (energy, material).  energy/mat are CUDA
         tensors (float64 / int32 or uint8 -> XS_FLAG_MAT_U8), or CPU tensors
         (then XS_FLAG_HOST_IO: staged copies inside the call, outputs returned
-        on the host)."""
+        on the host).  asynchronous=True (host tensors, pinned): XS_FLAG_HOST_ASYNC
+        — the call returns before the work is done; synchronize the current
+        stream before reading the outputs, and pass a different `workspace`
+        (uint8 CUDA tensor of xs_workspace_size bytes) to consecutive calls
+        so that the upload of one overlaps the lookups of the other."""
         import torch
         host = not energy.is_cuda
-        flags = ((XS_FLAG_SORT if sort else 0) | (XS_FLAG_HOST_IO if host else 0) |
-                 (XS_FLAG_F32 if f32 else 0) |
+        if asynchronous and not host:
+            raise ValueError("asynchronous=True takes host (pinned) tensors")
+        io = (XS_FLAG_HOST_ASYNC if asynchronous else XS_FLAG_HOST_IO) if host else 0
+        flags = ((XS_FLAG_SORT if sort else 0) | io | (XS_FLAG_F32 if f32 else 0) |
                  (XS_FLAG_MAT_U8 if mat.dtype == torch.uint8 else 0))
         count = energy.numel()
         if vsum is None:
             vsum = torch.zeros(2, dtype=torch.int64, device="cpu" if host else self.device)
         o, res = self._outputs(count, want, vsum, host=host)
-        ws = self.workspace(count, flags)
+        ws = workspace if workspace is not None else self.workspace(count, flags)
         xs_lookup_explicit(self._h, energy.data_ptr(), mat.data_ptr(), count, flags, o,
                            ws.data_ptr(), ws.numel(), self._stream())
         return vsum, res

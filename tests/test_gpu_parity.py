@@ -581,3 +581,38 @@ def test_part_cbits_wide_above_2p26(X):
     assert int(vs_a[1]) == L
     assert torch.equal(ra["verification"], r7["verification"])
     g.close()
+
+
+@pytest.mark.parametrize("sort", [False, True])
+def test_explicit_host_async_pipelined(X, sort):
+    """XS_FLAG_HOST_ASYNC: consecutive calls on two alternating workspaces
+    (upload of one overlapping the lookups of the other) give each call's
+    own results; nothing is read before the stream is synchronized."""
+    g = X.Grid.from_preset("tiny")
+    o = oracle_for("tiny")
+    rng = np.random.default_rng(33)
+    batches = []
+    for k in range(5):
+        p = rng.random(40_000 + 1_000 * k)
+        m = rng.integers(0, 12, p.size).astype(np.uint8)
+        S, M, v = o.run_explicit(p, m.astype(np.int32), mode=oracle.UNIONIZED, nthreads=NT)
+        batches.append((torch.tensor(p).pin_memory(), torch.tensor(m).pin_memory(), S, M, v))
+    fl = (X.XS_FLAG_SORT if sort else 0) | X.XS_FLAG_HOST_ASYNC | X.XS_FLAG_MAT_U8
+    n = g.workspace_size(45_000, fl)
+    wss = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    outs = []
+    for k, (pt, mt, *_rest) in enumerate(batches):
+        vs = torch.zeros(2, dtype=torch.int64).pin_memory()
+        _, res = g.lookup_explicit(pt, mt, sort=sort, vsum=vs, want=("macro_xs", "verification"),
+                                   asynchronous=True, workspace=wss[k % 2])
+        outs.append((vs, res))
+    torch.cuda.synchronize()
+    for (pt, mt, S, M, v), (vs, res) in zip(batches, outs):
+        assert vs.tolist() == [S, pt.numel()]
+        assert np.array_equal(res["macro_xs"].numpy(), M)
+        assert np.array_equal(res["verification"].numpy(), v)
+    with pytest.raises(X.XSError):   # exclusive with XS_FLAG_HOST_IO
+        X.xs_lookup_explicit(g._h, batches[0][0].data_ptr(), batches[0][1].data_ptr(), 10,
+                             X.XS_FLAG_HOST_IO | X.XS_FLAG_HOST_ASYNC | X.XS_FLAG_MAT_U8,
+                             X.xs_outputs(None, None, None, None, None, outs[0][0].data_ptr()),
+                             wss[0].data_ptr(), wss[0].numel(), torch.cuda.current_stream().cuda_stream)

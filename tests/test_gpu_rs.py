@@ -185,7 +185,8 @@ def test_rs_bench_multirank_path_on_one_gpu(R):
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
                         "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
                         "29543", "bench.py", "--gpus", "2", "--backend", "gloo", "--config",
-                        "rs-tiny", "--steps", "3", "--warmup", "3", "--no-cpu-baseline"],
+                        "rs-tiny", "--scaling", "weak", "--steps", "3", "--warmup", "3",
+                            "--no-cpu-baseline"],
                        cwd=root, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-2000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
