@@ -2899,6 +2899,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 43: return launch_gather_s4<GT, 4, 4, 12, 20, CHECK>(g, P, st);
     case 44: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK>(g, P, st);
     case 45: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK>(g, P, st);
+    case 49: return launch_gather_s4<GT, 3, 4, 8, 24, CHECK>(g, P, st);
+    case 50: return launch_gather_s4<GT, 3, 8, 16, 20, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
@@ -3076,7 +3078,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
-                      (variant >= 40 && variant <= 48);
+                      (variant >= 40 && variant <= 50);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)
