@@ -110,6 +110,7 @@ struct Params {
   const double* grid;
   const double* iv;         // interval table [I][N][kIvDoubles] (K0d)
   const double* iv32;       // fp32-variant interval table [I][N][kIv32Doubles] (K0e)
+  const double* ivu;        // 128-B line-aligned interval table [I][N][16] (K0u), or null
   int32_t I;
   int64_t N;
   const double* U;
@@ -727,6 +728,73 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
         }
         if (!valid) write_invalid(P, i);
       }
+    }
+    __syncthreads();
+    uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
+    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) row[t] = s_h[t];
+    __syncthreads();
+  }
+}
+
+// k_part_count for an energy-range shard (xs_lookup_batch_shard): A1 for
+// every lookup of the batch, but only ~1/n_shards of them are this shard's.
+// Each thread draws its four energies (two LCG steps each), the warp
+// compacts the lookups inside [e_lo, e_hi) through shared memory (ballot +
+// prefix), and the material pick, coarse key, histogram and the slab entry
+// for k_part_place are computed once per kept lookup with all lanes busy.
+constexpr int kShardWarps = kPrepThreads / 32;
+__global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
+  extern __shared__ uint32_t s_h[];  // [nkeys]
+  __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
+  __shared__ double s_cp[kShardWarps][32 * kPartItems];
+  __shared__ uint64_t s_cs[kShardWarps][32 * kPartItems];
+  __shared__ uint32_t s_ci[kShardWarps][32 * kPartItems];
+  __shared__ uint32_t s_kept;
+  const int nkeys = (P.n_mats + 1) * P.nkr;
+  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
+  const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  pick_table_fill(s_pick);
+  PartStream ps;
+  ps.init(P);
+  for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
+    for (int t = threadIdx.x; t < nkeys; t += blockDim.x) s_h[t] = 0;
+    if (threadIdx.x == 0) s_kept = 0;
+    __syncthreads();
+    uint64_t sc = ps.at(P, tl * tlen);
+    for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
+      const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
+      if (c0 >= P.count) break;
+      uint64_t st = (ps.tA * sc + ps.tC) & kMask63;
+      uint32_t run = 0;
+#pragma unroll
+      for (int it = 0; it < kPartItems; ++it) {
+        const uint64_t i = c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it;
+        st = lcg_next(st);
+        const double pe = lcg_double(st);
+        st = lcg_next(st);
+        const bool keep = i < P.count && pe >= P.e_lo && pe < P.e_hi;
+        const uint32_t ball = __ballot_sync(0xffffffffu, keep);
+        if (keep) {
+          const uint32_t q = run + __popc(ball & ((1u << lane) - 1u));
+          s_cp[warp][q] = pe;
+          s_cs[warp][q] = st;
+          s_ci[warp][q] = static_cast<uint32_t>(i);
+        }
+        run += __popc(ball);
+      }
+      __syncwarp();
+      for (uint32_t q = lane; q < run; q += 32) {
+        const Sample smp{s_cp[warp][q], pick_material_tab(s_pick, s_cs[warp][q])};
+        const uint32_t key = part_key(P, smp);
+        atomicAdd(&s_h[key], 1u);
+        const uint32_t at_q = atomicAdd(&s_kept, 1u);
+        const uint64_t at = static_cast<uint64_t>(tl) * tlen + at_q;
+        P.slab_p[at] = smp.p;
+        P.slab_k[at] = (static_cast<uint64_t>(s_ci[warp][q]) << 16) | key;
+      }
+      __syncwarp();
     }
     __syncthreads();
     uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
@@ -2310,6 +2378,205 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
   }
 }
 
+// ------------------------------------------------ k_gather_u (unsorted) --
+// Unsorted (material-bucketed) batches: every (lookup, nuclide) reads one
+// entry of the 128-B line-aligned interval table K0u, {E[k+1], gap,
+// recip(gap), 0 | h0, d0, h1, d1 | h2, d2, h3, d3 | h4, d4, 0, 0}, as four
+// 32-byte loads (LDG.256) by the lookup's four lanes: one L1 wavefront and
+// one 128-B line per (lookup, nuclide), where the record-pair gather
+// (k_gather) touches 96 B across 1-2 lines with two loads per lane.  Lane 0
+// computes f (R10, division by the stored reciprocal, correctly rounded),
+// lanes 1-3 the channels of their quarter.  Same arithmetic as every other
+// path (bit-identical M).
+constexpr int kGU = 4;                  // lanes per lookup
+constexpr int kLPTU = 32 / kGU;         // lookups per warp task (8)
+constexpr int kIvuDoubles = 16;         // K0u entry (128 B)
+
+__device__ __forceinline__ double4 ld_nc_256(const double* p) {
+  double4 v;
+  asm volatile("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+               : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w)
+               : "l"(p));
+  return v;
+}
+
+template <int GT, int U, int MINB, bool CHECK>
+__global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
+  if (gated_off(P)) return;
+  static_assert(U % kGU == 0, "U must be a multiple of the group size");
+  constexpr int Q = U / kGU;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem& S = *reinterpret_cast<GatherSmem*>(smem_raw);
+  const int tab = P.n_mats * P.max_nucs;
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem));
+  for (int t = threadIdx.x; t < tab; t += blockDim.x) {
+    const int32_t n = P.mats[t];
+    MatEntry me;
+    me.conc = P.concs[t];
+    me.noff = n >= 0 ? static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N) : 0u;
+    me.n = n;
+    s_tab[t] = me;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      S.num[m] = P.num_nucs[m];
+      S.off[m] = run;
+      S.cnt[m] = c;
+      S.toff[m] = trun;
+      run += c;
+      trun += (c + kLPTU - 1) / kLPTU;
+    }
+    S.off[P.n_mats] = run;
+    S.toff[P.n_mats] = trun;
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const int g = lane / kGU;
+  const int r = lane - g * kGU;
+  const int base = g * kGU;
+  const uint32_t total_tasks = S.toff[P.n_mats];
+  const uint32_t warps_per_block = blockDim.x >> 5;
+  const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
+  const uint32_t nw = gridDim.x * warps_per_block;
+  const double* __restrict__ ivu = P.ivu + r * 4;   // this lane's quarter of an entry
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  for (uint32_t task = gw; task < total_tasks; task += nw) {
+    while (task >= S.toff[m + 1]) ++m;
+    const uint32_t slot = (task - S.toff[m]) * kLPTU + g;
+    const bool valid = slot < S.cnt[m];
+    LookupRec rec{0.5, 0u, 0};
+    if (valid) rec = load_rec(P, S.off[m] + slot);
+    const double p = rec.p;
+    const int nn = valid ? S.num[m] : 0;
+    const int nw_loop = S.num[m];
+    const MatEntry* row = s_tab + m * P.max_nucs;
+    const RowView<GT> rv(P, valid ? rec.gidx : 0);
+
+    double acc_a = 0.0, acc_b = 0.0;
+    int32_t knext[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const int j = r + q * kGU;
+      int32_t kq = 0;
+      if (j < nn) {
+        const MatEntry me = row[j];
+        kq = rv.bracket(P, me.n, me.noff, p);
+      }
+      knext[q] = kq;
+    }
+    auto round = [&](const int j0, auto tail_tag) {
+      constexpr bool TAIL = decltype(tail_tag)::value;
+      int32_t kcur[Q];
+#pragma unroll
+      for (int q = 0; q < Q; ++q) kcur[q] = knext[q];
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {  // A4 for the next round
+        const int j = j0 + U + r + q * kGU;
+        int32_t kq = 0;
+        if (j < nn) {
+          const MatEntry me = row[j];
+          kq = rv.bracket(P, me.n, me.noff, p);
+        }
+        knext[q] = kq;
+      }
+      double4 v[U];
+      double cc[U];
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + t;
+        const int32_t kt = __shfl_sync(0xffffffffu, kcur[t / kGU], base + (t % kGU));
+        const MatEntry me = row[TAIL ? (j < nw_loop ? j : 0) : j];
+        cc[t] = me.conc;
+        uint32_t off = me.noff + static_cast<uint32_t>(kt);
+        if (TAIL) off = j < nw_loop ? off : 0u;
+        v[t] = ld_nc_256(ivu + static_cast<uint64_t>(off) * kIvuDoubles);
+      }
+      // A6: f from lane 0's quarter {E[k+1], gap, recip}; every lane computes
+      // it from its own quarter (branch-free), lane 0's value is broadcast
+      double fl[U];
+      bool fast = true;
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const double an = dsub(v[t].x, p);
+        fl[t] = div_by_recip(an, v[t].y, v[t].z);
+        if (CHECK) fast &= (r != 0) || div_in_range(an, v[t].y);
+      }
+      if (CHECK && !__all_sync(0xffffffffu, fast)) {
+#pragma unroll
+        for (int t = 0; t < U; ++t)
+          if (r == 0) fl[t] = ddiv(dsub(v[t].x, p), v[t].y);
+      }
+#pragma unroll
+      for (int t = 0; t < U; ++t) {
+        const int j = j0 + t;
+        const double f = __shfl_sync(0xffffffffu, fl[t], base);
+        const double xa = dsub(v[t].x, dmul(f, v[t].y));
+        const double xb = dsub(v[t].z, dmul(f, v[t].w));
+        if (!TAIL || j < nw_loop) {  // warp-uniform
+          const double c = cc[t];
+          acc_a = dadd(acc_a, dmul(xa, c));
+          acc_b = dadd(acc_b, dmul(xb, c));
+        }
+      }
+    };
+    int j0 = 0;
+    for (; j0 + U <= nw_loop; j0 += U) round(j0, std::false_type{});
+    if (j0 < nw_loop) round(j0, std::true_type{});
+    // A8: channels (t, s, a, f, nf) = (a@r1, b@r1, a@r2, b@r2, a@r3)
+    double M[5];
+    M[0] = __shfl_sync(0xffffffffu, acc_a, base + 1);
+    M[1] = __shfl_sync(0xffffffffu, acc_b, base + 1);
+    M[2] = __shfl_sync(0xffffffffu, acc_a, base + 2);
+    M[3] = __shfl_sync(0xffffffffu, acc_b, base + 2);
+    M[4] = __shfl_sync(0xffffffffu, acc_a, base + 3);
+    if (valid && r == 0) {
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (M[c] > mx) {
+          mx = M[c];
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[rec.idx] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(rec.idx) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = M[c];
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][kGatherThreads / 32];
+  if (lane == 0) {
+    s_red[0][threadIdx.x >> 5] = acc_v;
+    s_red[1][threadIdx.x >> 5] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (uint32_t w = 0; w < warps_per_block; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // ------------------------------------------- k_gather_s4 (staged, LDGSTS) --
 // The staged gather of k_gather_s3 with a cheaper producer: the windows of a
 // group of D nuclides are packed back to back into one of two per-warp
@@ -2711,6 +2978,7 @@ static Params make_params(const DeviceGrid& g) {
   P.grid = g.grid;
   P.iv = g.iv;
   P.iv32 = g.iv32;
+  P.ivu = g.ivu;
   P.I = g.I;
   P.N = g.N;
   P.U = g.U;
@@ -2759,8 +3027,33 @@ static cudaError_t launch_gather(const DeviceGrid& g, const Params& P, cudaStrea
 // energy (grid and lookups) is a multiple of 2^-63 in [0, 1] (DESIGN.md §4:
 // then |hi.E - p| and |hi.E - lo.E| are 0 or >= 2^-63), which holds for
 // generated grids with sampled lookups; otherwise the checked kernel runs.
+template <int GT, int U, int MINB, bool CHECK>
+static cudaError_t launch_gather_un(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  const size_t smem = sizeof(GatherSmem) + static_cast<size_t>(g.n_mats) * g.max_nucs * sizeof(MatEntry);
+  auto kern = k_gather_u<GT, U, MINB, CHECK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGatherThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, kGatherThreads, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  if (g.ivu && (g.unroll == 0 || (g.unroll >= 51 && g.unroll <= 54))) {
+    switch (g.unroll) {  // k_gather_u (nuclides per round U, min blocks of 256)
+      case 52: return launch_gather_un<GT, 8, 2, CHECK>(g, P, st);
+      case 53: return launch_gather_un<GT, 4, 4, CHECK>(g, P, st);
+      case 54: return launch_gather_un<GT, 8, 3, CHECK>(g, P, st);
+      default: return launch_gather_un<GT, 4, 3, CHECK>(g, P, st);  // 51
+    }
+  }
   switch (g.unroll) {
     case 1: return launch_gather<GT, 3, 3, CHECK>(g, P, st);
     case 2: return launch_gather<GT, 3, 4, CHECK>(g, P, st);
@@ -3123,7 +3416,12 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       P.slab_k = reinterpret_cast<uint64_t*>(sp + a.count);
     }
     const size_t hs = static_cast<size_t>(nkeys) * 4;
-    k_part_count<GT><<<nb, kPrepThreads, hs, st>>>(P);
+    // energy-range shards without per-lookup outputs: the compacting count
+    const bool outputs = a.out.energy || a.out.mat || a.out.grid_index;
+    if (a.shard && !outputs)
+      k_part_count_shard<<<nb, kPrepThreads, hs, st>>>(P);
+    else
+      k_part_count<GT><<<nb, kPrepThreads, hs, st>>>(P);
     mark(1);
     if (nkeys >= 32 * 148)
       k_part_colscan<32, 32><<<(nkeys + 31) / 32, dim3(32, 32), 0, st>>>(P, static_cast<int>(ntiles));

@@ -262,6 +262,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cudaFree(G.grid);
     cudaFree(G.iv);
     cudaFree(G.iv32);
+    cudaFree(G.ivu);
     cudaFree(G.U);
     cudaFree(G.UB);
     cudaFree(G.index);
@@ -293,7 +294,18 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     cleanup();
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
-  G.device_bytes = grid_bytes + iv_bytes + iv32_bytes + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
+  // K0u (unsorted gather): optional, only where it leaves ample memory free
+  // (large: 514 MB; XL: 10.9 GB); without it unsorted batches use k_gather
+  const size_t ivu_bytes = static_cast<size_t>(I) * N * 16 * sizeof(double);
+  {
+    size_t free_b = 0, total_b = 0;
+    cudaMemGetInfo(&free_b, &total_b);
+    if (free_b > ivu_bytes + (static_cast<size_t>(24) << 30) && cudaMalloc(&G.ivu, ivu_bytes) != cudaSuccess) {
+      G.ivu = nullptr;
+      cudaGetLastError();
+    }
+  }
+  G.device_bytes = grid_bytes + iv_bytes + iv32_bytes + (G.ivu ? ivu_bytes : 0) + G.NU * 8 + (G.NU ? (G.UBn + 1) * 4 : 0) + G.index_len * 4 * (G.index_layout == XS_INDEX_BOTH ? 2 : 1) + d->n_mats * 4 + tab * 12;
   e = cudaMemcpyAsync(G.grid, d->nuclide_grid, grid_bytes, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(G.num_nucs, d->num_nucs, d->n_mats * 4, cudaMemcpyHostToDevice, st);
@@ -301,6 +313,7 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
   if (e == cudaSuccess) e = cudaMemcpyAsync(G.concs, d->concs, tab * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = build_intervals(G, st);
   if (e == cudaSuccess) e = build_intervals32(G, st);
+  if (e == cudaSuccess && G.ivu) e = build_intervals_u(G, st);
   if (e == cudaSuccess && G.grid_type == XS_GRID_UNIONIZED) {
     e = build_union_grid(G, G.U, st);
     if (e == cudaSuccess) e = build_union_table(G, st);
@@ -723,6 +736,9 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
     case XS_TABLE_INTERVALS: src = G.iv; len = static_cast<uint64_t>(G.I) * G.N * kIvDoubles; break;
     case XS_TABLE_INTERVALS32:
       src = G.iv32; len = static_cast<uint64_t>(G.I) * G.N * kIv32Doubles; break;
+    case XS_TABLE_INTERVALS_U:
+      if (!G.ivu) return fail(XS_ERR_UNSUPPORTED, "grid has no K0u table");
+      src = G.ivu; len = static_cast<uint64_t>(G.I) * G.N * 16; break;
     case XS_TABLE_NUM_NUCS: src = G.num_nucs; len = G.n_mats; es = 4; break;
     case XS_TABLE_MATS: src = G.mats; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; es = 4; break;
     case XS_TABLE_CONCS: src = G.concs; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; break;
@@ -743,8 +759,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
           (value >= 17 && value <= 28) || (value >= 31 && value <= 36) ||
-          (value >= 40 && value <= 50)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-50");
+          (value >= 40 && value <= 54)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-54");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
@@ -816,6 +832,7 @@ void xs_free_grid(xs_grid* g) {
   cudaFree(g->d.grid);
   cudaFree(g->d.iv);
   cudaFree(g->d.iv32);
+  cudaFree(g->d.ivu);
   cudaFree(g->d.U);
   cudaFree(g->d.UB);
   cudaFree(g->d.index);

@@ -35,6 +35,7 @@ struct DeviceGrid {
   double* grid = nullptr;    // [I][N][6]
   double* iv = nullptr;      // [I][N][kIvDoubles] interval table (K0d), or null
   double* iv32 = nullptr;    // [I][N][kIv32Doubles] fp32-variant interval table (K0e)
+  double* ivu = nullptr;     // [I][N][16] 128-B line-aligned interval table (K0u), or null
   double* U = nullptr;       // [NU]
   int32_t* UB = nullptr;     // [UBn + 1]: UB[b] = ub(U, b / UBn)  (A3 search table)
   int32_t UBn = 0;           // power of two
@@ -105,6 +106,7 @@ cudaError_t build_hash_grid(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_union_table(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_intervals(const DeviceGrid& g, cudaStream_t st);
 cudaError_t build_intervals32(const DeviceGrid& g, cudaStream_t st);
+cudaError_t build_intervals_u(const DeviceGrid& g, cudaStream_t st);
 cudaError_t init_constants();
 
 // lookup.cu

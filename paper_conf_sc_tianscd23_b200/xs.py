@@ -25,7 +25,7 @@ XS_FLAG_MAT_U8 = 0x10
 XS_FLAG_HOST_ASYNC = 0x20
 (XS_TABLE_NUCLIDE_GRID, XS_TABLE_UNION_ENERGY, XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS,
  XS_TABLE_MATS, XS_TABLE_CONCS, XS_TABLE_INDEX_GRID_T, XS_TABLE_INTERVALS,
- XS_TABLE_INTERVALS32) = range(9)
+ XS_TABLE_INTERVALS32, XS_TABLE_INTERVALS_U) = range(10)
 XS_INDEX_AUTO, XS_INDEX_ROW, XS_INDEX_COL, XS_INDEX_BOTH = 0, 1, 2, 3
 INDEX_LAYOUTS = {"auto": 0, "row": 1, "col": 2, "both": 3}
 STATUS = {0: "XS_OK", 1: "XS_ERR_INVALID_ARG", 2: "XS_ERR_OUT_OF_MEMORY", 3: "XS_ERR_CUDA",
@@ -446,7 +446,8 @@ class Grid:
                 XS_TABLE_CONCS: i.n_mats * i.max_num_nucs,
                 XS_TABLE_INDEX_GRID_T: i.index_grid_len if i.index_layout & 2 else 0,
                 XS_TABLE_INTERVALS: i.n_isotopes * i.n_gridpoints * 14,
-                XS_TABLE_INTERVALS32: i.n_isotopes * i.n_gridpoints * 10}
+                XS_TABLE_INTERVALS32: i.n_isotopes * i.n_gridpoints * 10,
+                XS_TABLE_INTERVALS_U: i.n_isotopes * i.n_gridpoints * 16}
         dt = np.int32 if which in (XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS, XS_TABLE_MATS,
                                    XS_TABLE_INDEX_GRID_T) \
             else np.float64

@@ -69,12 +69,13 @@ def _compare(out, ref, mode_index=True):
 
 # ------------------------------------------------------------------- tiny --
 @pytest.mark.parametrize("variant", ["default", "sort", "baseline", "v1", "v2", "v3", "v4",
+                                     "v51", "v52", "v53", "v54",
                                      "sort-v1", "sort-v3", "sort-v4", "sort-v9", "sort-v10",
                                      "sort-v11", "sort-v12", "sort-v17", "sort-v18", "sort-v19",
                                      "sort-v20", "sort-v21", "sort-v22", "sort-v23",
                                      "sort-v24", "sort-v25", "sort-v26", "sort-v27", "sort-v28",
                                      "sort-v40", "sort-v41", "sort-v42", "sort-v43", "sort-v44",
-                                     "sort-v45"])
+                                     "sort-v45", "sort-v49", "sort-v50"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -449,7 +450,8 @@ def test_explicit_host_io_chunked(X, sort):
         assert np.array_equal(res["verification"].numpy(), v)
 
 
-@pytest.mark.parametrize("variant", [0, 9, 17, 19, 20, 21, 25, 28, 40, 41, 42, 43, 44, 45])
+@pytest.mark.parametrize("variant", [0, 9, 17, 19, 20, 21, 25, 28, 40, 41, 42, 43, 44, 45, 49,
+                                     50])
 @pytest.mark.parametrize("grid_type,bins", [("unionized", 0), ("hash", 97)])
 def test_vsum_only_sorted(X, variant, grid_type, bins):
     """Sorted batches with only vsum requested (no per-lookup outputs: the
