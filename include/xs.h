@@ -185,9 +185,9 @@ typedef struct {
                                    (hi.c, hi.c - lo.c) x 5}; entry N-1 is zero     */
 #define XS_TABLE_INTERVALS32 8  /* [double] I*N*10: fp32-variant table (K0e): {E[k+1],
                                    gap, ~1/gap, 0} then 12 floats (h_c, d_c) x 5, 0, 0 */
-#define XS_TABLE_INTERVALS_U 9  /* [double] I*N*16: K0d's entry in a 128-B line-aligned
-                                   layout for unsorted batches (K0u): {E[k+1], gap,
-                                   ~1/gap, 0, (hi.c, hi.c - lo.c) x 5, 0, 0};
+#define XS_TABLE_INTERVALS_U 9  /* [double] I*N*12: the unsorted gather's 96-B,
+                                   32-B aligned entries (K0u): {E[k+1], gap,
+                                   (hi.c, hi.c - lo.c) x 5}; entry N-1 is zero;
                                    UNSUPPORTED when the grid did not build it
                                    (built only with ample free device memory) */
 

@@ -256,31 +256,26 @@ cudaError_t build_intervals32(const DeviceGrid& g, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-// K0u: the interval entry of K0d in a 128-B line-aligned layout for the
-// unsorted gather (k_gather_u): {E[k+1], gap, recip(gap), 0, h0, d0, h1, d1,
-// h2, d2, h3, d3, h4, d4, 0, 0}; entry N-1 is zero.
+// K0u: the unsorted gather's interval table (k_gather_u), 96-B entries,
+// 32-B aligned: {E[k+1], gap, h0, d0, h1, d1, h2, d2, h3, d3, h4, d4} with
+// h = hi.c and d = hi.c - lo.c (the operations of K0d); entry N-1 is zero.
 __global__ void k_build_intervals_u(const double* __restrict__ grid, uint64_t total, int64_t N,
                                     double* __restrict__ IV) {
   for (uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; t < total;
        t += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
-    double* o = IV + t * 16;
+    double* o = IV + t * 12;
     if (static_cast<int64_t>(t % static_cast<uint64_t>(N)) == N - 1) {
-      for (int q = 0; q < 16; ++q) o[q] = 0.0;
+      for (int q = 0; q < 12; ++q) o[q] = 0.0;
       continue;
     }
     const double* lo = grid + t * 6;
     const double* hi = lo + 6;
-    const double bd = dsub(hi[0], lo[0]);
     o[0] = hi[0];
-    o[1] = bd;
-    o[2] = recip_nr(bd);
-    o[3] = 0.0;
+    o[1] = dsub(hi[0], lo[0]);
     for (int c = 0; c < 5; ++c) {
-      o[4 + 2 * c] = hi[1 + c];
-      o[5 + 2 * c] = dsub(hi[1 + c], lo[1 + c]);
+      o[2 + 2 * c] = hi[1 + c];
+      o[3 + 2 * c] = dsub(hi[1 + c], lo[1 + c]);
     }
-    o[14] = 0.0;
-    o[15] = 0.0;
   }
 }
 

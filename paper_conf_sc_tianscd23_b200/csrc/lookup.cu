@@ -110,7 +110,7 @@ struct Params {
   const double* grid;
   const double* iv;         // interval table [I][N][kIvDoubles] (K0d)
   const double* iv32;       // fp32-variant interval table [I][N][kIv32Doubles] (K0e)
-  const double* ivu;        // 128-B line-aligned interval table [I][N][16] (K0u), or null
+  const double* ivu;        // 32-B aligned interval table [I][N][12] (K0u), or null
   int32_t I;
   int64_t N;
   const double* U;
@@ -2380,17 +2380,17 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
 
 // ------------------------------------------------ k_gather_u (unsorted) --
 // Unsorted (material-bucketed) batches: every (lookup, nuclide) reads one
-// entry of the 128-B line-aligned interval table K0u, {E[k+1], gap,
-// recip(gap), 0 | h0, d0, h1, d1 | h2, d2, h3, d3 | h4, d4, 0, 0}, as four
-// 32-byte loads (LDG.256) by the lookup's four lanes: one L1 wavefront and
-// one 128-B line per (lookup, nuclide), where the record-pair gather
-// (k_gather) touches 96 B across 1-2 lines with two loads per lane.  Lane 0
-// computes f (R10, division by the stored reciprocal, correctly rounded),
-// lanes 1-3 the channels of their quarter.  Same arithmetic as every other
-// path (bit-identical M).
-constexpr int kGU = 4;                  // lanes per lookup
-constexpr int kLPTU = 32 / kGU;         // lookups per warp task (8)
-constexpr int kIvuDoubles = 16;         // K0u entry (128 B)
+// 96-B entry of the 32-B aligned interval table K0u, {E[k+1], gap, h0, d0 |
+// h1, d1, h2, d2 | h3, d3, h4, d4} (h = hi.c, d = hi.c - lo.c), as three
+// 32-byte loads (LDG.256) by the lookup's three lanes: three DRAM sectors
+// and one load instruction per (lookup, nuclide), where the record-pair
+// gather (k_gather) needs two loads per lane over 3-4 sectors.  Lane 0
+// computes f (R10: correctly rounded division, reciprocal refined on the
+// fly) and its channel, lanes 1-2 two channels each.  Same arithmetic as
+// every other path (bit-identical M).
+constexpr int kGU = 3;                  // lanes per lookup
+constexpr int kLPTU = 32 / kGU;         // lookups per warp task (10)
+constexpr int kIvuDoubles = 12;         // K0u entry (96 B)
 
 __device__ __forceinline__ double4 ld_nc_256(const double* p) {
   double4 v;
@@ -2441,14 +2441,14 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
   const uint32_t warps_per_block = blockDim.x >> 5;
   const uint32_t gw = blockIdx.x * warps_per_block + (threadIdx.x >> 5);
   const uint32_t nw = gridDim.x * warps_per_block;
-  const double* __restrict__ ivu = P.ivu + r * 4;   // this lane's quarter of an entry
+  const double* __restrict__ ivu = P.ivu + r * 4;   // this lane's third of an entry
 
   unsigned long long acc_v = 0, acc_n = 0;
   int m = 0;
   for (uint32_t task = gw; task < total_tasks; task += nw) {
     while (task >= S.toff[m + 1]) ++m;
     const uint32_t slot = (task - S.toff[m]) * kLPTU + g;
-    const bool valid = slot < S.cnt[m];
+    const bool valid = (g < kLPTU) && (slot < S.cnt[m]);
     LookupRec rec{0.5, 0u, 0};
     if (valid) rec = load_rec(P, S.off[m] + slot);
     const double p = rec.p;
@@ -2496,14 +2496,14 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
         if (TAIL) off = j < nw_loop ? off : 0u;
         v[t] = ld_nc_256(ivu + static_cast<uint64_t>(off) * kIvuDoubles);
       }
-      // A6: f from lane 0's quarter {E[k+1], gap, recip}; every lane computes
-      // it from its own quarter (branch-free), lane 0's value is broadcast
+      // A6: f from lane 0's third {E[k+1], gap, ...}; every lane computes
+      // it from its own third (branch-free), lane 0's value is broadcast
       double fl[U];
       bool fast = true;
 #pragma unroll
       for (int t = 0; t < U; ++t) {
         const double an = dsub(v[t].x, p);
-        fl[t] = div_by_recip(an, v[t].y, v[t].z);
+        fl[t] = div_nr(an, v[t].y);
         if (CHECK) fast &= (r != 0) || div_in_range(an, v[t].y);
       }
       if (CHECK && !__all_sync(0xffffffffu, fast)) {
@@ -2515,6 +2515,7 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
       for (int t = 0; t < U; ++t) {
         const int j = j0 + t;
         const double f = __shfl_sync(0xffffffffu, fl[t], base);
+        // lane 0: (E, gap | h0, d0) -> channel 0 in acc_b; lanes 1-2: (h, d) x 2
         const double xa = dsub(v[t].x, dmul(f, v[t].y));
         const double xb = dsub(v[t].z, dmul(f, v[t].w));
         if (!TAIL || j < nw_loop) {  // warp-uniform
@@ -2527,13 +2528,13 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
     int j0 = 0;
     for (; j0 + U <= nw_loop; j0 += U) round(j0, std::false_type{});
     if (j0 < nw_loop) round(j0, std::true_type{});
-    // A8: channels (t, s, a, f, nf) = (a@r1, b@r1, a@r2, b@r2, a@r3)
+    // A8: channels (t, s, a, f, nf) = (b@r0, a@r1, b@r1, a@r2, b@r2)
     double M[5];
-    M[0] = __shfl_sync(0xffffffffu, acc_a, base + 1);
-    M[1] = __shfl_sync(0xffffffffu, acc_b, base + 1);
-    M[2] = __shfl_sync(0xffffffffu, acc_a, base + 2);
-    M[3] = __shfl_sync(0xffffffffu, acc_b, base + 2);
-    M[4] = __shfl_sync(0xffffffffu, acc_a, base + 3);
+    M[0] = __shfl_sync(0xffffffffu, acc_b, base);
+    M[1] = __shfl_sync(0xffffffffu, acc_a, base + 1);
+    M[2] = __shfl_sync(0xffffffffu, acc_b, base + 1);
+    M[3] = __shfl_sync(0xffffffffu, acc_a, base + 2);
+    M[4] = __shfl_sync(0xffffffffu, acc_b, base + 2);
     if (valid && r == 0) {
       double mx = -1.0;
       int vi = 0;
@@ -2864,6 +2865,312 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   }
 }
 
+// ------------------------------------ k_gather_s5 (s4 + task prefetch) --
+// k_gather_s4 with the task prologue taken off the critical path (unionized
+// grid, partitioned A2): while a warp works on its task q, the energies (and
+// positions) of task q + 2 stream into shared memory, and the A4 bounds of
+// task q + 1 (two IGT/IG entries per nuclide at the task's extreme energies,
+// found from its prefetched energies through the equal-width table) are
+// fetched by 4-byte cp.async; the next task then starts from shared memory.
+// Same arithmetic and results as k_gather_s4.
+template <int C, int R, bool F32>
+__host__ __device__ constexpr size_t s5_warp_bytes(int max_nucs) {
+  return 2 * static_cast<size_t>(C) * (F32 ? kIv32Doubles : kIvDoubles) * 8 +  // buffers
+         2 * static_cast<size_t>(max_nucs) * 8 +                                // bounds x2
+         ((static_cast<size_t>(max_nucs) + 15) / 16) * 16 +                     // offsets
+         2 * 32 * R * 8 + 2 * 32 * R * 4 +                                      // records x2
+         64;                                                                    // mbarriers
+}
+
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32>
+__global__ void __launch_bounds__(32 * NW, 1) k_gather_s5(Params P) {
+  static_assert(GT == XS_GRID_UNIONIZED, "the prefetch reads the unionized index grid");
+  if (gated_off(P)) return;
+  using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
+  constexpr int kTask = 32 * R;
+  constexpr int kE = Acc::kE;
+  constexpr int LPN = 32 / D;
+  static_assert(D >= 1 && D <= 32 && (32 % D) == 0, "group size divides the warp");
+  static_assert(C <= 254, "buffer offsets are bytes");
+  constexpr uint8_t kNoOff = 0xff;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GatherSmem4& G = *reinterpret_cast<GatherSmem4*>(smem_raw);
+  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem4));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    uint32_t run = 0, trun = 0, roff = 0;
+    for (int m = 0; m < P.n_mats; ++m) {
+      const uint32_t c = P.counts[m];
+      G.num[m] = P.num_nucs[m];
+      G.off[m] = run;
+      G.cnt[m] = c;
+      G.toff[m] = trun;
+      G.roff[m] = roff;
+      run += c;
+      trun += (c + kTask - 1) / kTask;
+      roff += static_cast<uint32_t>(P.num_nucs[m]);
+    }
+    G.off[P.n_mats] = run;
+    G.toff[P.n_mats] = trun;
+    G.roff[P.n_mats] = roff;
+  }
+  __syncthreads();
+  const int tab = static_cast<int>(G.roff[P.n_mats]);
+  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
+    int m = 0;
+    while (static_cast<uint32_t>(i) >= G.roff[m + 1]) ++m;
+    const int src = m * P.max_nucs + (i - static_cast<int>(G.roff[m]));
+    const int32_t n = P.mats[src];
+    MatEntry me;
+    me.conc = P.concs[src];
+    me.noff = static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N);
+    me.n = n;
+    s_tab[i] = me;
+  }
+  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab) + ((tab * sizeof(MatEntry) + 15) / 16) * 16;
+  unsigned char* mine = wbase + s5_warp_bytes<C, R, F32>(P.max_nucs) * warp;
+  double2* s_buf = reinterpret_cast<double2*>(mine);                                 // [2][C * kE]
+  unsigned char* cur = mine + 2 * static_cast<size_t>(C) * kE * 16;
+  int2* s_kk = reinterpret_cast<int2*>(cur);                                         // [2][max_nucs]
+  cur += 2 * static_cast<size_t>(P.max_nucs) * 8;
+  uint8_t* s_off = cur;                                                              // [max_nucs]
+  cur += ((static_cast<size_t>(P.max_nucs) + 15) / 16) * 16;
+  double* s_rp = reinterpret_cast<double*>(cur);                                     // [2][kTask]
+  cur += 2 * kTask * 8;
+  uint32_t* s_ri = reinterpret_cast<uint32_t*>(cur);                                 // [2][kTask]
+  cur += 2 * kTask * 4;
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(cur);  // [0,1] groups, [2,3] bounds, [4,5] records
+  if (lane == 0) {
+    for (int b = 0; b < 6; ++b) mbar_init(&s_bar[b], 32);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  const uint32_t total_tasks = G.toff[P.n_mats];
+  const uint32_t gw = blockIdx.x * NW + warp;
+  const uint32_t nwarps = gridDim.x * NW;
+  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(F32 ? P.iv32 : P.iv);
+  uint32_t phase = 0;  // parity bit per mbarrier (bit b)
+  auto wait_bar = [&](int b) {
+    mbar_wait(&s_bar[b], (phase >> b) & 1u);
+    phase ^= 1u << b;
+  };
+  auto mat_of = [&](uint32_t task) {
+    int mm = 0;
+    while (task >= G.toff[mm + 1]) ++mm;
+    return mm;
+  };
+  // records of `task` -> s_rp/s_ri[b] (8-/4-byte cp.async: bucket offsets are arbitrary)
+  auto issue_records = [&](uint32_t task, int b) {
+    if (task < total_tasks) {
+      const int mm = mat_of(task);
+      const uint32_t s0 = (task - G.toff[mm]) * kTask;
+      const uint32_t rem = G.cnt[mm] - s0;
+      const uint32_t n = rem < static_cast<uint32_t>(kTask) ? rem : static_cast<uint32_t>(kTask);
+      const uint32_t at = G.off[mm] + s0;
+      for (uint32_t i = lane; i < n; i += 32) {
+        cp_async8(s_rp + b * kTask + i, P.sp + at + i);
+        if (P.sidx) cp_async4(s_ri + b * kTask + i, P.sidx + at + i);
+      }
+    }
+    cp_async_mbar_arrive(&s_bar[4 + b]);
+  };
+  // A3 + A4 of `task` from its energies in s_rp[b]: bounds -> s_kk[b]
+  auto prefetch_bounds = [&](uint32_t task, int b) {
+    if (task < total_tasks) {
+      const int mm = mat_of(task);
+      const uint32_t s0 = (task - G.toff[mm]) * kTask;
+      double plo = 2.0, phi = -1.0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint32_t slot = lane * R + r;
+        if (s0 + slot < G.cnt[mm]) {
+          const double e = s_rp[b * kTask + slot];
+          plo = e < plo ? e : plo;
+          phi = e > phi ? e : phi;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        const double x = __shfl_xor_sync(0xffffffffu, plo, o);
+        const double y = __shfl_xor_sync(0xffffffffu, phi, o);
+        plo = x < plo ? x : plo;
+        phi = y > phi ? y : phi;
+      }
+      const int32_t ulo = union_lower_tab(P, plo), uhi = union_upper_tab(P, phi);
+      const int nn2 = G.num[mm];
+      const MatEntry* row2 = s_tab + G.roff[mm];
+      for (int j = lane; j < nn2; j += 32) {
+        const int32_t n = row2[j].n;
+        int2* dst = s_kk + b * P.max_nucs + j;
+        if (P.index_t) {
+          cp_async4(&dst->x, P.index_t + static_cast<int64_t>(n) * P.NU + ulo);
+          cp_async4(&dst->y, P.index_t + static_cast<int64_t>(n) * P.NU + uhi);
+        } else {
+          cp_async4(&dst->x, P.index + static_cast<int64_t>(ulo) * P.I + n);
+          cp_async4(&dst->y, P.index + static_cast<int64_t>(uhi) * P.I + n);
+        }
+      }
+    }
+    cp_async_mbar_arrive(&s_bar[2 + b]);
+  };
+
+  unsigned long long acc_v = 0, acc_n = 0;
+  int m = 0;
+  uint32_t task = gw;
+  if (task < total_tasks) {  // pipeline fill
+    issue_records(task, 0);
+    issue_records(task + nwarps, 1);
+    wait_bar(4);
+    prefetch_bounds(task, 0);
+  }
+  for (int q = 0; task < total_tasks; task += nwarps, ++q) {
+    const int b = q & 1;
+    while (task >= G.toff[m + 1]) ++m;
+    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
+    double p[R];
+    uint32_t idx[R];
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      valid[r] = slot0 + r < G.cnt[m];
+      p[r] = valid[r] ? s_rp[b * kTask + lane * R + r] : 0.5;
+      idx[r] = (valid[r] && P.sidx) ? s_ri[b * kTask + lane * R + r] : 0u;
+    }
+#pragma unroll
+    for (int pass = 0; pass < R; ++pass) {
+#pragma unroll
+      for (int r = pass & 1; r + 1 < R; r += 2) {
+        const bool swap = (valid[r + 1] && !valid[r]) ||
+                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
+        if (swap) {
+          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
+          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
+          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
+        }
+      }
+    }
+    double plo = valid[0] ? p[0] : 2.0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const double x = __shfl_xor_sync(0xffffffffu, plo, o);
+      plo = x < plo ? x : plo;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
+    const int nn = G.num[m];
+    const MatEntry* row = s_tab + G.roff[m];
+    const int2* kk = s_kk + b * P.max_nucs;
+    wait_bar(2 + b);  // this task's bounds
+    for (int j0 = 0; j0 < nn; j0 += 32) {  // group-buffer offsets (segmented scan)
+      const int j = j0 + lane;
+      const int2 w = j < nn ? kk[j] : make_int2(0, 0);
+      const int32_t n_int = w.y - w.x;
+      const int size = (j < nn && n_int < C) ? n_int + 1 : 0;
+      int incl = size;
+#pragma unroll
+      for (int o = 1; o < D; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if ((lane & (D - 1)) >= o) incl += v;
+      }
+      if (j < nn) s_off[j] = (size > 0 && incl <= C) ? static_cast<uint8_t>(incl - size) : kNoOff;
+    }
+    __syncwarp();  // offsets written; every lane has read its records from s_rp[b]
+    // prefetch: bounds of the next task (its energies arrived during the
+    // previous task), energies of the one after
+    wait_bar(4 + (b ^ 1));
+    prefetch_bounds(task + nwarps, b ^ 1);
+    issue_records(task + 2 * nwarps, b);
+
+    auto issue_group = [&](int g) {
+      if (g * D >= nn) return;  // warp-uniform
+      const int j = g * D + lane / LPN;
+      if (j < nn && s_off[j] != kNoOff) {
+        const int2 w = kk[j];
+        const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(w.x)) * kE;
+        double2* dst = s_buf + (g & 1) * (C * kE) + s_off[j] * kE;
+        const int nch = (w.y - w.x + 1) * kE;
+        for (int c = lane % LPN; c < nch; c += LPN) cp_async16(dst + c, src + c);
+      }
+      cp_async_mbar_arrive(&s_bar[g & 1]);
+    };
+    issue_group(0);
+    issue_group(1);
+
+    Acc acc;
+    acc.zero();
+    for (int j = 0; j < nn; ++j) {
+      if (j % D == 0) {
+        const int g = j / D;
+        if (g >= 1) {
+          __syncwarp();
+          issue_group(g + 1);
+        }
+        wait_bar(g & 1);
+      }
+      const int2 w = kk[j];
+      const uint32_t off = s_off[j];
+      const MatEntry me = row[j];
+      const int n_int = w.y - w.x;
+      if (off != kNoOff) {
+        stage_nuclide_iv<R, true>(s_buf + ((j / D) & 1) * (C * kE) + off * kE, n_int, me.conc, p, acc);
+      } else {
+        const double2* g2 = iv2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(w.x)) * kE;
+        stage_nuclide_iv<R, false>(g2, n_int, me.conc, p, acc);
+      }
+      if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
+    }
+    if (nn & (kF32Block - 1)) acc.flush();
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!valid[r]) continue;
+      double mx = -1.0;
+      int vi = 0;
+#pragma unroll
+      for (int c = 0; c < 5; ++c)
+        if (acc.get(r, c) > mx) {
+          mx = acc.get(r, c);
+          vi = c;
+        }
+      acc_v += static_cast<unsigned long long>(vi + 1);
+      acc_n += 1;
+      if (P.out_v) P.out_v[idx[r]] = vi + 1;
+      if (P.out_M) {
+        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
+#pragma unroll
+        for (int c = 0; c < 5; ++c) o[c] = acc.get(r, c);
+      }
+    }
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");  // prefetches past the last task
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
+    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
+  }
+  __shared__ unsigned long long s_red[2][NW];
+  if (lane == 0) {
+    s_red[0][warp] = acc_v;
+    s_red[1][warp] = acc_n;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, n = 0;
+    for (int w = 0; w < NW; ++w) {
+      v += s_red[0][w];
+      n += s_red[1][w];
+    }
+    if (n) {
+      atomicAdd(P.vsum, v);
+      atomicAdd(P.vsum + 1, n);
+    }
+  }
+}
+
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -3048,10 +3355,10 @@ template <int GT, bool CHECK>
 static cudaError_t launch_gather_v(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   if (g.ivu && (g.unroll == 0 || (g.unroll >= 51 && g.unroll <= 54))) {
     switch (g.unroll) {  // k_gather_u (nuclides per round U, min blocks of 256)
-      case 52: return launch_gather_un<GT, 8, 2, CHECK>(g, P, st);
-      case 53: return launch_gather_un<GT, 4, 4, CHECK>(g, P, st);
-      case 54: return launch_gather_un<GT, 8, 3, CHECK>(g, P, st);
-      default: return launch_gather_un<GT, 4, 3, CHECK>(g, P, st);  // 51
+      case 51: return launch_gather_un<GT, 3, 3, CHECK>(g, P, st);
+      case 53: return launch_gather_un<GT, 3, 4, CHECK>(g, P, st);
+      case 54: return launch_gather_un<GT, 6, 3, CHECK>(g, P, st);
+      default: return launch_gather_un<GT, 6, 2, CHECK>(g, P, st);  // 52 (measured best, large)
     }
   }
   switch (g.unroll) {
@@ -3146,6 +3453,28 @@ static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false>
+static cudaError_t launch_gather_s5(const DeviceGrid& g, const Params& P, cudaStream_t st) {
+  if (GT != XS_GRID_UNIONIZED || !P.sp || P.need_gidx)  // prefetch needs the partitioned A2
+    return launch_gather_s4<GT, R, D, C, NW, CHECK, F32>(g, P, st);
+  constexpr int GTU = XS_GRID_UNIONIZED;
+  const size_t smem = sizeof(GatherSmem4) + ((static_cast<size_t>(g.tab_total) * sizeof(MatEntry) + 15) / 16) * 16 +
+                      NW * s5_warp_bytes<C, R, F32>(g.max_nucs);
+  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
+  auto kern = k_gather_s5<GTU, R, D, C, NW, CHECK, F32>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = g.blocks_per_sm;
+  if (per_sm <= 0) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
+  return cudaGetLastError();
+}
+
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
@@ -3193,6 +3522,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 44: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK>(g, P, st);
     case 45: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK>(g, P, st);
     case 49: return launch_gather_s4<GT, 3, 4, 8, 24, CHECK>(g, P, st);
+    case 55: return launch_gather_s5<GT, 4, 8, 20, 16, CHECK>(g, P, st);
+    case 56: return launch_gather_s5<GT, 4, 8, 16, 16, CHECK>(g, P, st);
     case 50: return launch_gather_s4<GT, 3, 8, 16, 20, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
@@ -3212,6 +3543,7 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
     case 35: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
     case 47: return launch_gather_s4<GT, 4, 8, 20, 20, CHECK, true>(g, P, st);
     case 48: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK, true>(g, P, st);
+    case 57: return launch_gather_s5<GT, 4, 8, 20, 16, CHECK, true>(g, P, st);
     default: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true>(g, P, st);  // = 46
   }
 }
@@ -3371,7 +3703,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
-                      (variant >= 40 && variant <= 50);
+                      (variant >= 40 && variant <= 50) || (variant >= 55 && variant <= 57);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)

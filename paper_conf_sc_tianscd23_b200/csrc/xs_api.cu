@@ -295,8 +295,8 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
   // K0u (unsorted gather): optional, only where it leaves ample memory free
-  // (large: 514 MB; XL: 10.9 GB); without it unsorted batches use k_gather
-  const size_t ivu_bytes = static_cast<size_t>(I) * N * 16 * sizeof(double);
+  // (large: 385 MB; XL: 8.1 GB); without it unsorted batches use k_gather
+  const size_t ivu_bytes = static_cast<size_t>(I) * N * 12 * sizeof(double);
   {
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
@@ -738,7 +738,7 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
       src = G.iv32; len = static_cast<uint64_t>(G.I) * G.N * kIv32Doubles; break;
     case XS_TABLE_INTERVALS_U:
       if (!G.ivu) return fail(XS_ERR_UNSUPPORTED, "grid has no K0u table");
-      src = G.ivu; len = static_cast<uint64_t>(G.I) * G.N * 16; break;
+      src = G.ivu; len = static_cast<uint64_t>(G.I) * G.N * 12; break;
     case XS_TABLE_NUM_NUCS: src = G.num_nucs; len = G.n_mats; es = 4; break;
     case XS_TABLE_MATS: src = G.mats; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; es = 4; break;
     case XS_TABLE_CONCS: src = G.concs; len = static_cast<uint64_t>(G.n_mats) * G.max_nucs; break;
@@ -759,8 +759,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
           (value >= 17 && value <= 28) || (value >= 31 && value <= 36) ||
-          (value >= 40 && value <= 54)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-54");
+          (value >= 40 && value <= 57)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-57");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");

@@ -447,7 +447,7 @@ class Grid:
                 XS_TABLE_INDEX_GRID_T: i.index_grid_len if i.index_layout & 2 else 0,
                 XS_TABLE_INTERVALS: i.n_isotopes * i.n_gridpoints * 14,
                 XS_TABLE_INTERVALS32: i.n_isotopes * i.n_gridpoints * 10,
-                XS_TABLE_INTERVALS_U: i.n_isotopes * i.n_gridpoints * 16}
+                XS_TABLE_INTERVALS_U: i.n_isotopes * i.n_gridpoints * 12}
         dt = np.int32 if which in (XS_TABLE_INDEX_GRID, XS_TABLE_NUM_NUCS, XS_TABLE_MATS,
                                    XS_TABLE_INDEX_GRID_T) \
             else np.float64

@@ -144,10 +144,10 @@ def test_device_tables_full(X, name):
     _assert_equal("IV hi", iv[:, :-1, 4::2], hi[..., 1:])
     _assert_equal("IV d", iv[:, :-1, 5::2], hi[..., 1:] - lo[..., 1:])
     assert not np.any(iv[:, -1]) and not np.any(iv[:, :, 3])
-    # K0u: the same entry, 128-B line-aligned (unsorted gather)
-    ivu = g.table(X.XS_TABLE_INTERVALS_U).reshape(I, N, 16)
-    _assert_equal("IVU", ivu[:, :, :14], iv)
-    assert not np.any(ivu[:, :, 14:])
+    # K0u (unsorted gather): {E[k+1], gap, (hi.c, hi.c - lo.c) x 5}, 96 B
+    ivu = g.table(X.XS_TABLE_INTERVALS_U).reshape(I, N, 12)
+    _assert_equal("IVU head", ivu[:, :, :2], iv[:, :, :2])
+    _assert_equal("IVU channels", ivu[:, :, 2:], iv[:, :, 4:])
     # fp32 table K0e: h = RN32(hi.c), d = RN32(h - RN32(lo.c)) (R18)
     iv32 = g.table(X.XS_TABLE_INTERVALS32).reshape(I, N, 10)
     _assert_equal("IV32 head", iv32[:, :-1, :3], iv[:, :-1, :3])
