@@ -2865,312 +2865,6 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   }
 }
 
-// ------------------------------------ k_gather_s5 (s4 + task prefetch) --
-// k_gather_s4 with the task prologue taken off the critical path (unionized
-// grid, partitioned A2): while a warp works on its task q, the energies (and
-// positions) of task q + 2 stream into shared memory, and the A4 bounds of
-// task q + 1 (two IGT/IG entries per nuclide at the task's extreme energies,
-// found from its prefetched energies through the equal-width table) are
-// fetched by 4-byte cp.async; the next task then starts from shared memory.
-// Same arithmetic and results as k_gather_s4.
-template <int C, int R, bool F32>
-__host__ __device__ constexpr size_t s5_warp_bytes(int max_nucs) {
-  return 2 * static_cast<size_t>(C) * (F32 ? kIv32Doubles : kIvDoubles) * 8 +  // buffers
-         2 * static_cast<size_t>(max_nucs) * 8 +                                // bounds x2
-         ((static_cast<size_t>(max_nucs) + 15) / 16) * 16 +                     // offsets
-         2 * 32 * R * 8 + 2 * 32 * R * 4 +                                      // records x2
-         64;                                                                    // mbarriers
-}
-
-template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32>
-__global__ void __launch_bounds__(32 * NW, 1) k_gather_s5(Params P) {
-  static_assert(GT == XS_GRID_UNIONIZED, "the prefetch reads the unionized index grid");
-  if (gated_off(P)) return;
-  using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
-  constexpr int kTask = 32 * R;
-  constexpr int kE = Acc::kE;
-  constexpr int LPN = 32 / D;
-  static_assert(D >= 1 && D <= 32 && (32 % D) == 0, "group size divides the warp");
-  static_assert(C <= 254, "buffer offsets are bytes");
-  constexpr uint8_t kNoOff = 0xff;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  GatherSmem4& G = *reinterpret_cast<GatherSmem4*>(smem_raw);
-  MatEntry* s_tab = reinterpret_cast<MatEntry*>(smem_raw + sizeof(GatherSmem4));
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-
-  if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0, roff = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      G.num[m] = P.num_nucs[m];
-      G.off[m] = run;
-      G.cnt[m] = c;
-      G.toff[m] = trun;
-      G.roff[m] = roff;
-      run += c;
-      trun += (c + kTask - 1) / kTask;
-      roff += static_cast<uint32_t>(P.num_nucs[m]);
-    }
-    G.off[P.n_mats] = run;
-    G.toff[P.n_mats] = trun;
-    G.roff[P.n_mats] = roff;
-  }
-  __syncthreads();
-  const int tab = static_cast<int>(G.roff[P.n_mats]);
-  for (int i = threadIdx.x; i < tab; i += blockDim.x) {
-    int m = 0;
-    while (static_cast<uint32_t>(i) >= G.roff[m + 1]) ++m;
-    const int src = m * P.max_nucs + (i - static_cast<int>(G.roff[m]));
-    const int32_t n = P.mats[src];
-    MatEntry me;
-    me.conc = P.concs[src];
-    me.noff = static_cast<uint32_t>(n) * static_cast<uint32_t>(P.N);
-    me.n = n;
-    s_tab[i] = me;
-  }
-  unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab) + ((tab * sizeof(MatEntry) + 15) / 16) * 16;
-  unsigned char* mine = wbase + s5_warp_bytes<C, R, F32>(P.max_nucs) * warp;
-  double2* s_buf = reinterpret_cast<double2*>(mine);                                 // [2][C * kE]
-  unsigned char* cur = mine + 2 * static_cast<size_t>(C) * kE * 16;
-  int2* s_kk = reinterpret_cast<int2*>(cur);                                         // [2][max_nucs]
-  cur += 2 * static_cast<size_t>(P.max_nucs) * 8;
-  uint8_t* s_off = cur;                                                              // [max_nucs]
-  cur += ((static_cast<size_t>(P.max_nucs) + 15) / 16) * 16;
-  double* s_rp = reinterpret_cast<double*>(cur);                                     // [2][kTask]
-  cur += 2 * kTask * 8;
-  uint32_t* s_ri = reinterpret_cast<uint32_t*>(cur);                                 // [2][kTask]
-  cur += 2 * kTask * 4;
-  uint64_t* s_bar = reinterpret_cast<uint64_t*>(cur);  // [0,1] groups, [2,3] bounds, [4,5] records
-  if (lane == 0) {
-    for (int b = 0; b < 6; ++b) mbar_init(&s_bar[b], 32);
-    mbar_fence_init();
-  }
-  __syncthreads();
-
-  const uint32_t total_tasks = G.toff[P.n_mats];
-  const uint32_t gw = blockIdx.x * NW + warp;
-  const uint32_t nwarps = gridDim.x * NW;
-  const double2* __restrict__ iv2 = reinterpret_cast<const double2*>(F32 ? P.iv32 : P.iv);
-  uint32_t phase = 0;  // parity bit per mbarrier (bit b)
-  auto wait_bar = [&](int b) {
-    mbar_wait(&s_bar[b], (phase >> b) & 1u);
-    phase ^= 1u << b;
-  };
-  auto mat_of = [&](uint32_t task) {
-    int mm = 0;
-    while (task >= G.toff[mm + 1]) ++mm;
-    return mm;
-  };
-  // records of `task` -> s_rp/s_ri[b] (8-/4-byte cp.async: bucket offsets are arbitrary)
-  auto issue_records = [&](uint32_t task, int b) {
-    if (task < total_tasks) {
-      const int mm = mat_of(task);
-      const uint32_t s0 = (task - G.toff[mm]) * kTask;
-      const uint32_t rem = G.cnt[mm] - s0;
-      const uint32_t n = rem < static_cast<uint32_t>(kTask) ? rem : static_cast<uint32_t>(kTask);
-      const uint32_t at = G.off[mm] + s0;
-      for (uint32_t i = lane; i < n; i += 32) {
-        cp_async8(s_rp + b * kTask + i, P.sp + at + i);
-        if (P.sidx) cp_async4(s_ri + b * kTask + i, P.sidx + at + i);
-      }
-    }
-    cp_async_mbar_arrive(&s_bar[4 + b]);
-  };
-  // A3 + A4 of `task` from its energies in s_rp[b]: bounds -> s_kk[b]
-  auto prefetch_bounds = [&](uint32_t task, int b) {
-    if (task < total_tasks) {
-      const int mm = mat_of(task);
-      const uint32_t s0 = (task - G.toff[mm]) * kTask;
-      double plo = 2.0, phi = -1.0;
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const uint32_t slot = lane * R + r;
-        if (s0 + slot < G.cnt[mm]) {
-          const double e = s_rp[b * kTask + slot];
-          plo = e < plo ? e : plo;
-          phi = e > phi ? e : phi;
-        }
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        const double x = __shfl_xor_sync(0xffffffffu, plo, o);
-        const double y = __shfl_xor_sync(0xffffffffu, phi, o);
-        plo = x < plo ? x : plo;
-        phi = y > phi ? y : phi;
-      }
-      const int32_t ulo = union_lower_tab(P, plo), uhi = union_upper_tab(P, phi);
-      const int nn2 = G.num[mm];
-      const MatEntry* row2 = s_tab + G.roff[mm];
-      for (int j = lane; j < nn2; j += 32) {
-        const int32_t n = row2[j].n;
-        int2* dst = s_kk + b * P.max_nucs + j;
-        if (P.index_t) {
-          cp_async4(&dst->x, P.index_t + static_cast<int64_t>(n) * P.NU + ulo);
-          cp_async4(&dst->y, P.index_t + static_cast<int64_t>(n) * P.NU + uhi);
-        } else {
-          cp_async4(&dst->x, P.index + static_cast<int64_t>(ulo) * P.I + n);
-          cp_async4(&dst->y, P.index + static_cast<int64_t>(uhi) * P.I + n);
-        }
-      }
-    }
-    cp_async_mbar_arrive(&s_bar[2 + b]);
-  };
-
-  unsigned long long acc_v = 0, acc_n = 0;
-  int m = 0;
-  uint32_t task = gw;
-  if (task < total_tasks) {  // pipeline fill
-    issue_records(task, 0);
-    issue_records(task + nwarps, 1);
-    wait_bar(4);
-    prefetch_bounds(task, 0);
-  }
-  for (int q = 0; task < total_tasks; task += nwarps, ++q) {
-    const int b = q & 1;
-    while (task >= G.toff[m + 1]) ++m;
-    const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
-    double p[R];
-    uint32_t idx[R];
-    bool valid[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      valid[r] = slot0 + r < G.cnt[m];
-      p[r] = valid[r] ? s_rp[b * kTask + lane * R + r] : 0.5;
-      idx[r] = (valid[r] && P.sidx) ? s_ri[b * kTask + lane * R + r] : 0u;
-    }
-#pragma unroll
-    for (int pass = 0; pass < R; ++pass) {
-#pragma unroll
-      for (int r = pass & 1; r + 1 < R; r += 2) {
-        const bool swap = (valid[r + 1] && !valid[r]) ||
-                          (valid[r] == valid[r + 1] && p[r + 1] < p[r]);
-        if (swap) {
-          const double tp = p[r]; p[r] = p[r + 1]; p[r + 1] = tp;
-          const uint32_t ti = idx[r]; idx[r] = idx[r + 1]; idx[r + 1] = ti;
-          const bool tv = valid[r]; valid[r] = valid[r + 1]; valid[r + 1] = tv;
-        }
-      }
-    }
-    double plo = valid[0] ? p[0] : 2.0;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      const double x = __shfl_xor_sync(0xffffffffu, plo, o);
-      plo = x < plo ? x : plo;
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
-    const int nn = G.num[m];
-    const MatEntry* row = s_tab + G.roff[m];
-    const int2* kk = s_kk + b * P.max_nucs;
-    wait_bar(2 + b);  // this task's bounds
-    for (int j0 = 0; j0 < nn; j0 += 32) {  // group-buffer offsets (segmented scan)
-      const int j = j0 + lane;
-      const int2 w = j < nn ? kk[j] : make_int2(0, 0);
-      const int32_t n_int = w.y - w.x;
-      const int size = (j < nn && n_int < C) ? n_int + 1 : 0;
-      int incl = size;
-#pragma unroll
-      for (int o = 1; o < D; o <<= 1) {
-        const int v = __shfl_up_sync(0xffffffffu, incl, o);
-        if ((lane & (D - 1)) >= o) incl += v;
-      }
-      if (j < nn) s_off[j] = (size > 0 && incl <= C) ? static_cast<uint8_t>(incl - size) : kNoOff;
-    }
-    __syncwarp();  // offsets written; every lane has read its records from s_rp[b]
-    // prefetch: bounds of the next task (its energies arrived during the
-    // previous task), energies of the one after
-    wait_bar(4 + (b ^ 1));
-    prefetch_bounds(task + nwarps, b ^ 1);
-    issue_records(task + 2 * nwarps, b);
-
-    auto issue_group = [&](int g) {
-      if (g * D >= nn) return;  // warp-uniform
-      const int j = g * D + lane / LPN;
-      if (j < nn && s_off[j] != kNoOff) {
-        const int2 w = kk[j];
-        const double2* src = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(w.x)) * kE;
-        double2* dst = s_buf + (g & 1) * (C * kE) + s_off[j] * kE;
-        const int nch = (w.y - w.x + 1) * kE;
-        for (int c = lane % LPN; c < nch; c += LPN) cp_async16(dst + c, src + c);
-      }
-      cp_async_mbar_arrive(&s_bar[g & 1]);
-    };
-    issue_group(0);
-    issue_group(1);
-
-    Acc acc;
-    acc.zero();
-    for (int j = 0; j < nn; ++j) {
-      if (j % D == 0) {
-        const int g = j / D;
-        if (g >= 1) {
-          __syncwarp();
-          issue_group(g + 1);
-        }
-        wait_bar(g & 1);
-      }
-      const int2 w = kk[j];
-      const uint32_t off = s_off[j];
-      const MatEntry me = row[j];
-      const int n_int = w.y - w.x;
-      if (off != kNoOff) {
-        stage_nuclide_iv<R, true>(s_buf + ((j / D) & 1) * (C * kE) + off * kE, n_int, me.conc, p, acc);
-      } else {
-        const double2* g2 = iv2 + static_cast<uint64_t>(me.noff + static_cast<uint32_t>(w.x)) * kE;
-        stage_nuclide_iv<R, false>(g2, n_int, me.conc, p, acc);
-      }
-      if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
-    }
-    if (nn & (kF32Block - 1)) acc.flush();
-    __syncwarp();
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!valid[r]) continue;
-      double mx = -1.0;
-      int vi = 0;
-#pragma unroll
-      for (int c = 0; c < 5; ++c)
-        if (acc.get(r, c) > mx) {
-          mx = acc.get(r, c);
-          vi = c;
-        }
-      acc_v += static_cast<unsigned long long>(vi + 1);
-      acc_n += 1;
-      if (P.out_v) P.out_v[idx[r]] = vi + 1;
-      if (P.out_M) {
-        double* o = P.out_M + static_cast<uint64_t>(idx[r]) * 5;
-#pragma unroll
-        for (int c = 0; c < 5; ++c) o[c] = acc.get(r, c);
-      }
-    }
-  }
-  asm volatile("cp.async.wait_all;" ::: "memory");  // prefetches past the last task
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    acc_v += __shfl_xor_sync(0xffffffffu, acc_v, o);
-    acc_n += __shfl_xor_sync(0xffffffffu, acc_n, o);
-  }
-  __shared__ unsigned long long s_red[2][NW];
-  if (lane == 0) {
-    s_red[0][warp] = acc_v;
-    s_red[1][warp] = acc_n;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, n = 0;
-    for (int w = 0; w < NW; ++w) {
-      v += s_red[0][w];
-      n += s_red[1][w];
-    }
-    if (n) {
-      atomicAdd(P.vsum, v);
-      atomicAdd(P.vsum + 1, n);
-    }
-  }
-}
-
 // --------------------------------------------------- XSBench-shape baseline
 // One thread per lookup, no bucketing, serial nuclide loop (the shape of the
 // CUDA kernels the paper measured).  Same exact
@@ -3453,28 +3147,6 @@ static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
-template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false>
-static cudaError_t launch_gather_s5(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  if (GT != XS_GRID_UNIONIZED || !P.sp || P.need_gidx)  // prefetch needs the partitioned A2
-    return launch_gather_s4<GT, R, D, C, NW, CHECK, F32>(g, P, st);
-  constexpr int GTU = XS_GRID_UNIONIZED;
-  const size_t smem = sizeof(GatherSmem4) + ((static_cast<size_t>(g.tab_total) * sizeof(MatEntry) + 15) / 16) * 16 +
-                      NW * s5_warp_bytes<C, R, F32>(g.max_nucs);
-  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
-  auto kern = k_gather_s5<GTU, R, D, C, NW, CHECK, F32>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = g.blocks_per_sm;
-  if (per_sm <= 0) {
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * NW, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) per_sm = 1;
-  }
-  kern<<<g.sm_count * per_sm, 32 * NW, smem, st>>>(P);
-  return cudaGetLastError();
-}
-
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
@@ -3522,8 +3194,7 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 44: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK>(g, P, st);
     case 45: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK>(g, P, st);
     case 49: return launch_gather_s4<GT, 3, 4, 8, 24, CHECK>(g, P, st);
-    case 55: return launch_gather_s5<GT, 4, 8, 20, 16, CHECK>(g, P, st);
-    case 56: return launch_gather_s5<GT, 4, 8, 16, 16, CHECK>(g, P, st);
+
     case 50: return launch_gather_s4<GT, 3, 8, 16, 20, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
@@ -3543,7 +3214,7 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
     case 35: return launch_gather_s3<GT, 4, 2, 8, 24, CHECK, false, true>(g, P, st);
     case 47: return launch_gather_s4<GT, 4, 8, 20, 20, CHECK, true>(g, P, st);
     case 48: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK, true>(g, P, st);
-    case 57: return launch_gather_s5<GT, 4, 8, 20, 16, CHECK, true>(g, P, st);
+
     default: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true>(g, P, st);  // = 46
   }
 }
@@ -3703,7 +3374,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
-                      (variant >= 40 && variant <= 50) || (variant >= 55 && variant <= 57);
+                      (variant >= 40 && variant <= 50);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)

@@ -80,7 +80,7 @@ def _check_vs_binary64(o, first, count, mode, M32, mat):
     return q12.max()
 
 
-@pytest.mark.parametrize("variant", [0, 31, 32, 33, 34, 36, 46, 47, 48, 57])
+@pytest.mark.parametrize("variant", [0, 31, 32, 33, 34, 36, 46, 47, 48])
 @pytest.mark.parametrize("first,count", [(0, 1), (5, 31), (999_999, 4097), (3, 70_001)])
 def test_f32_shapes_and_ragged(X, variant, first, count):
     g = X.Grid.from_preset("tiny")
