@@ -3152,18 +3152,21 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
   // blocks); 9-12 TMA-staged record windows (R, stages D, window W records,
   // warps per block); 17-20 TMA-staged interval-table windows (R, group
-  // size D, window W entries, warps per block).  Measured best on B200 (large,
-  // large-hash, small): k_gather_s3 (4, 4, 6, 16) = variant 25, while a
-  // task's windows stay short.  Density d = N * 128 / count (interval entries a
-  // 128-lookup task of one material spans per nuclide, up to the material's
-  // share): with long windows fewer lookups per lane win, variant 20 (2, 2, 8,
-  // 24).  Measured crossover: large/small 8M lookups (d 0.18)
-  // 1.75 vs 1.82 ms, 4M (d 0.36) 1.23 vs 1.16 ms; XL 170M (d 0.18, N 238,847,
-  // cold 9.5 GB interval table) 36.5 vs 33.5 ms gather.
+  // size D, window W entries, warps per block); 40-50 k_gather_s4 (R, group
+  // size D, group buffer C entries, warps per block).  Density d = N * 128 /
+  // count (interval entries a 128-lookup task of one material spans per
+  // nuclide; for an energy-range shard count is the whole batch's, whose
+  // density the shard keeps).  Measured on B200: d < 0.12 (large
+  // and small at 17M) k_gather_s4 (4, 8, 20, 16) = variant 40 (large 2.31 vs
+  // 2.47 ms for k_gather_s3 variant 25); 0.12 <= d < 0.25 k_gather_s4 with 2
+  // lookups per lane, variant 44 (large 8M: 1.44 vs 1.48 / 1.61 ms for 40 /
+  // 20); d >= 0.25 (large 4M: 1.02 vs 1.07 / 1.14 ms), or d >= 0.15 on grids of
+  // >= 100k points (XL 170M: 33.5 vs 41.4 ms) k_gather_s3 (2, 2, 8, 24) =
+  // variant 20.
   int v = g.unroll;
   if (v == 0) {
     const double d = static_cast<double>(g.N) * 128.0 / static_cast<double>(P.count ? P.count : 1);
-    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : 40;
+    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : (d >= 0.12 ? 44 : 40);
   }
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
