@@ -1,5 +1,5 @@
 """Summarise an ncu --set full report (raw page) into a small JSON + text
-table for profiles/.  Usage: python tools/ncu_summary.py REPORT.ncu-rep OUT_PREFIX [LOOKUPS]"""
+table for profiles/.  Usage: python tools/ncu_summary.py REPORT.ncu-rep|RAW.csv OUT_PREFIX [LOOKUPS]"""
 import csv
 import io
 import json
@@ -23,8 +23,11 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 def main():
     rep, out = sys.argv[1], sys.argv[2]
     lookups = int(sys.argv[3]) if len(sys.argv) > 3 else None
-    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    if rep.endswith(".csv"):  # an exported `ncu -i ... --page raw --csv`
+        raw = open(rep).read()
+    else:
+        raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
+                             text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
     res = []
