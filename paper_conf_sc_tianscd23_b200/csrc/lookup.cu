@@ -1937,15 +1937,54 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s(Params P) {
 //    windows longer than W entries (sparse tasks) take a global-memory path.
 //  * Bulk copies are issued D at a time by D lanes into a ring of 2D slots
 //    (D to 2D nuclides ahead), completing on per-slot mbarriers.
+// Window access for the staged gathers (16-B units u of an interval-table
+// window): through a generic pointer to shared memory, through the read-only
+// path from global memory, or through a 32-bit shared-memory address (no
+// generic-to-shared conversion in the loop).
+struct WinPtr {
+  const double2* q;
+  __device__ __forceinline__ double2 ld2(int u) const { return q[u]; }
+  __device__ __forceinline__ float4 ld4f(int u) const { return *reinterpret_cast<const float4*>(q + u); }
+  __device__ __forceinline__ double ld1(int u) const { return reinterpret_cast<const double*>(q + u)[0]; }
+  __device__ __forceinline__ WinPtr at(int u) const { return WinPtr{q + u}; }
+};
+struct WinGlobal {
+  const double2* q;
+  __device__ __forceinline__ double2 ld2(int u) const { return __ldg(q + u); }
+  __device__ __forceinline__ float4 ld4f(int u) const { return __ldg(reinterpret_cast<const float4*>(q + u)); }
+  __device__ __forceinline__ double ld1(int u) const { return __ldg(reinterpret_cast<const double*>(q + u)); }
+  __device__ __forceinline__ WinGlobal at(int u) const { return WinGlobal{q + u}; }
+};
+struct WinSmem {
+  uint32_t a;  // shared-memory byte address
+  __device__ __forceinline__ double2 ld2(int u) const {
+    double2 v;
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a + 16u * u));
+    return v;
+  }
+  __device__ __forceinline__ float4 ld4f(int u) const {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                 : "r"(a + 16u * u));
+    return v;
+  }
+  __device__ __forceinline__ double ld1(int u) const {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a + 16u * u));
+    return v;
+  }
+  __device__ __forceinline__ WinSmem at(int u) const { return WinSmem{a + 16u * u}; }
+};
+
 // Same operations in the same order as the oracle (bit-identical M).
 // Entry layout (7 x 16 B): {E[k+1], gap} {recip(gap), 0} {hi.c, hi.c - lo.c} x 5.
 // A6 + A7 for lookups r in [r0, r1) that all lie in entry q (channel terms are
 // read from the window per channel to keep register pressure low).
-template <int R, bool CHECK, bool SHARED>
-__device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R], double conc,
+template <int R, bool CHECK, class Win>
+__device__ __forceinline__ void iv_interp(const Win q, const double (&p)[R], double conc,
                                           double (&M)[R][5], int r0, int r1) {
-  auto ld = [&](int u) -> double2 { return SHARED ? q[u] : __ldg(q + u); };
-  const double2 a0 = ld(0), a1 = ld(1);
+  const double2 a0 = q.ld2(0), a1 = q.ld2(1);
   double f[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -1956,7 +1995,7 @@ __device__ __forceinline__ void iv_interp(const double2* q, const double (&p)[R]
   }
 #pragma unroll
   for (int c = 0; c < 5; ++c) {
-    const double2 hd = ld(2 + c);
+    const double2 hd = q.ld2(2 + c);
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (r < r0 || r >= r1) continue;
@@ -1991,10 +2030,10 @@ struct AccF64 {  // binary64 (R10, R11): entry = K0d, 7 x 16 B
   }
   __device__ __forceinline__ double get(int r, int c) const { return M[r][c]; }
   __device__ __forceinline__ void flush() {}  // one accumulation level (R11)
-  template <bool SHARED>
-  __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
+  template <class Win>
+  __device__ __forceinline__ void interp(const Win q, const double (&p)[R], double conc, int r0,
                                          int r1) {
-    iv_interp<R, CHECK, SHARED>(q, p, conc, M, r0, r1);
+    iv_interp<R, CHECK>(q, p, conc, M, r0, r1);
   }
 };
 
@@ -2027,15 +2066,11 @@ struct AccF32 {  // binary32 variant (R18): entry = K0e, 5 x 16 B
   __device__ __forceinline__ double get(int r, int c) const {
     return static_cast<double>((r & 1) ? T[r >> 1][c].y : T[r >> 1][c].x);
   }
-  template <bool SHARED>
-  __device__ __forceinline__ void interp(const double2* q, const double (&p)[R], double conc, int r0,
+  template <class Win>
+  __device__ __forceinline__ void interp(const Win q, const double (&p)[R], double conc, int r0,
                                          int r1) {
-    auto ld = [&](int u) -> double2 { return SHARED ? q[u] : __ldg(q + u); };
-    auto ldf = [&](int u) -> float4 {
-      const float4* f4 = reinterpret_cast<const float4*>(q + u);
-      return SHARED ? *f4 : __ldg(f4);
-    };
-    const double2 a0 = ld(0), a1 = ld(1);
+    auto ldf = [&](int u) -> float4 { return q.ld4f(u); };
+    const double2 a0 = q.ld2(0), a1 = q.ld2(1);
     float nf[R];  // -f, f = binary64 weight rounded once to binary32
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -2072,17 +2107,14 @@ struct AccF32 {  // binary32 variant (R18): entry = K0e, 5 x 16 B
 // One nuclide of a task: win = interval entries k_lo .. k_lo + n_int.
 // i(p) = max{t in [0, n_int] : t = 0 or E[k_lo + t] <= p} by binary lifting
 // (warp-uniform trip count; loads clamped so the loop has no branches).
-template <int R, bool SHARED, class Acc>
-__device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, double conc,
+template <int R, class Win, class Acc>
+__device__ __forceinline__ void stage_nuclide_iv(const Win win, int n_int, double conc,
                                                  const double (&p)[R], Acc& acc) {
   constexpr int kE = Acc::kE;
   // E[k_lo + t] = first double of entry t - 1
-  auto E = [&](int t) -> double {
-    const double* q = reinterpret_cast<const double*>(win + (t - 1) * kE);
-    return SHARED ? q[0] : __ldg(q);
-  };
+  auto E = [&](int t) -> double { return win.ld1((t - 1) * kE); };
   if (n_int == 0) {  // one entry: every lookup of the task lies in it (warp-uniform)
-    acc.template interp<SHARED>(win, p, conc, 0, R);
+    acc.interp(win, p, conc, 0, R);
     return;
   }
   if (n_int == 1) {  // two entries (the common multi-entry case): one shared probe
@@ -2091,11 +2123,11 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
 #pragma unroll
     for (int r = 0; r < R; ++r) i[r] = e <= p[r] ? 1 : 0;
     if (__all_sync(0xffffffffu, i[0] == i[R - 1])) {  // p sorted within the lane
-      acc.template interp<SHARED>(win + i[0] * kE, p, conc, 0, R);
+      acc.interp(win.at(i[0] * kE), p, conc, 0, R);
       return;
     }
 #pragma unroll
-    for (int r = 0; r < R; ++r) acc.template interp<SHARED>(win + i[r] * kE, p, conc, r, r + 1);
+    for (int r = 0; r < R; ++r) acc.interp(win.at(i[r] * kE), p, conc, r, r + 1);
     return;
   }
   int i0, iL;
@@ -2110,7 +2142,7 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     }
   }
   if (__all_sync(0xffffffffu, i0 == iL)) {
-    acc.template interp<SHARED>(win + i0 * kE, p, conc, 0, R);
+    acc.interp(win.at(i0 * kE), p, conc, 0, R);
     return;
   }
   int i[R];
@@ -2129,7 +2161,7 @@ __device__ __forceinline__ void stage_nuclide_iv(const double2* win, int n_int, 
     }
   }
 #pragma unroll
-  for (int r = 0; r < R; ++r) acc.template interp<SHARED>(win + i[r] * kE, p, conc, r, r + 1);
+  for (int r = 0; r < R; ++r) acc.interp(win.at(i[r] * kE), p, conc, r, r + 1);
 }
 
 template <int GT, int R, int D, int W, int NW, bool CHECK, bool DYN = false, bool F32 = false>
@@ -2318,10 +2350,10 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       const int2 kk = s_k[j];
       const int n_int = kk.y - kk.x;
       if (n_int < W) {
-        stage_nuclide_iv<R, true>(s_win + slot * W * kE, n_int, conc, p, acc);
+        stage_nuclide_iv<R>(WinPtr{s_win + slot * W * kE}, n_int, conc, p, acc);
       } else {
         const double2* g2 = iv2 + static_cast<uint64_t>(row[j].noff + static_cast<uint32_t>(kk.x)) * kE;
-        stage_nuclide_iv<R, false>(g2, n_int, conc, p, acc);
+        stage_nuclide_iv<R>(WinGlobal{g2}, n_int, conc, p, acc);
       }
       if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
     }
@@ -2593,7 +2625,8 @@ __global__ void __launch_bounds__(kGatherThreads, MINB) k_gather_u(Params P) {
 struct alignas(16) NucWin {
   int32_t klo, khi;   // bracket range of the task's extreme energies (A4)
   uint32_t noff;      // n * N
-  uint32_t off;       // entry offset in the group buffer, kNoBuf = read in place
+  uint32_t off;       // shared-memory byte address of the window in its group
+                      // buffer, kNoBuf = read in place from global memory
 };
 constexpr uint32_t kNoBuf = 0xffffffffu;
 
@@ -2661,6 +2694,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   double2* s_buf = reinterpret_cast<double2*>(mine);                            // [2][C * kE]
   NucWin* s_k = reinterpret_cast<NucWin*>(mine + 2 * static_cast<size_t>(C) * kE * 16);
   uint64_t* s_bar = reinterpret_cast<uint64_t*>(s_k + P.max_nucs);              // [2]
+  const uint32_t buf_base = smem_u32(s_buf);
   if (lane == 0) {
     mbar_init(&s_bar[0], 32);
     mbar_init(&s_bar[1], 32);
@@ -2771,7 +2805,9 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
         w.klo = klo;
         w.khi = khi;
         w.noff = noff;
-        w.off = (size > 0 && incl <= C) ? static_cast<uint32_t>(incl - size) : kNoBuf;
+        w.off = (size > 0 && incl <= C)
+                    ? buf_base + static_cast<uint32_t>(((j / D) & 1) * C + (incl - size)) * (kE * 16)
+                    : kNoBuf;
         s_k[j] = w;
       }
     }
@@ -2785,9 +2821,8 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
         const NucWin w = s_k[j];
         if (w.off != kNoBuf) {
           const double2* src = iv2 + static_cast<uint64_t>(w.noff + static_cast<uint32_t>(w.klo)) * kE;
-          double2* dst = s_buf + (g & 1) * (C * kE) + w.off * kE;
           const int nch = (w.khi - w.klo + 1) * kE;
-          for (int c = lane % LPN; c < nch; c += LPN) cp_async16(dst + c, src + c);
+          for (int c = lane % LPN; c < nch; c += LPN) cp_async16_s(w.off + 16u * c, src + c);
         }
       }
       cp_async_mbar_arrive(&s_bar[g & 1]);
@@ -2811,10 +2846,10 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
       const double conc = row[j].conc;
       const int n_int = w.khi - w.klo;
       if (w.off != kNoBuf) {
-        stage_nuclide_iv<R, true>(s_buf + ((j / D) & 1) * (C * kE) + w.off * kE, n_int, conc, p, acc);
+        stage_nuclide_iv<R>(WinSmem{w.off}, n_int, conc, p, acc);
       } else {
         const double2* g2 = iv2 + static_cast<uint64_t>(w.noff + static_cast<uint32_t>(w.klo)) * kE;
-        stage_nuclide_iv<R, false>(g2, n_int, conc, p, acc);
+        stage_nuclide_iv<R>(WinGlobal{g2}, n_int, conc, p, acc);
       }
       if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
     }
