@@ -2644,7 +2644,7 @@ __host__ __device__ constexpr size_t s4_warp_bytes(int max_nucs) {
          static_cast<size_t>(max_nucs) * sizeof(NucWin) + 16;                   // windows + bars
 }
 
-template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32>
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32, bool DYN>
 __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   if (gated_off(P)) return;
   using Acc = typename std::conditional<F32, AccF32<R, CHECK>, AccF64<R, CHECK>>::type;
@@ -2710,7 +2710,11 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
 
   unsigned long long acc_v = 0, acc_n = 0;
   int m = 0;
-  for (uint32_t task = gw; task < total_tasks; task += nwarps) {
+  // DYN: after its first task a warp takes the next one from a global counter
+  // (tasks in material order, fuel first), fetched one task ahead
+  uint32_t next = 0;
+  if (DYN && lane == 0) next = nwarps + atomicAdd(P.task_next, 1u);
+  for (uint32_t task = gw; task < total_tasks;) {
     while (task >= G.toff[m + 1]) ++m;
     const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
     double p[R];
@@ -2874,6 +2878,12 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
 #pragma unroll
         for (int c = 0; c < 5; ++c) o[c] = acc.get(r, c);
       }
+    }
+    if (DYN) {
+      task = __shfl_sync(0xffffffffu, next, 0);
+      if (lane == 0 && task < total_tasks) next = nwarps + atomicAdd(P.task_next, 1u);
+    } else {
+      task += nwarps;
     }
   }
 #pragma unroll
@@ -3157,7 +3167,7 @@ static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaSt
   return cudaGetLastError();
 }
 
-template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false>
+template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false, bool DYN = false>
 static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   int tab = 0;
   {
@@ -3167,7 +3177,7 @@ static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaSt
   }
   const size_t smem = sizeof(GatherSmem4) + ((static_cast<size_t>(tab) * sizeof(MatEntry) + 15) / 16) * 16 +
                       NW * s4_warp_bytes<C, NW, F32>(g.max_nucs);
-  auto kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32>;
+  auto kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32, DYN>;
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
@@ -3187,21 +3197,26 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // variants 1-4: k_gather_t (lookups per lane R, nuclides per round U, min
   // blocks); 9-12 TMA-staged record windows (R, stages D, window W records,
   // warps per block); 17-20 TMA-staged interval-table windows (R, group
-  // size D, window W entries, warps per block); 40-50 k_gather_s4 (R, group
-  // size D, group buffer C entries, warps per block).  Density d = N * 128 /
-  // count (interval entries a 128-lookup task of one material spans per
-  // nuclide; for an energy-range shard count is the whole batch's, whose
-  // density the shard keeps).  Measured on B200: d < 0.12 (large
-  // and small at 17M) k_gather_s4 (4, 8, 20, 16) = variant 40 (large 2.31 vs
-  // 2.47 ms for k_gather_s3 variant 25); 0.12 <= d < 0.25 k_gather_s4 with 2
-  // lookups per lane, variant 44 (large 8M: 1.44 vs 1.48 / 1.61 ms for 40 /
-  // 20); d >= 0.25 (large 4M: 1.02 vs 1.07 / 1.14 ms), or d >= 0.15 on grids of
-  // >= 100k points (XL 170M: 33.5 vs 41.4 ms) k_gather_s3 (2, 2, 8, 24) =
-  // variant 20.
+  // size D, window W entries, warps per block); 40-58 k_gather_s4 (R, group
+  // size D, group buffer C entries, warps per block; 55/56 take tasks from a
+  // global counter after their first).  Density d = N * 128 / count (interval
+  // entries a 128-lookup task of one material spans per nuclide; for an
+  // energy-range shard count is the whole batch's, whose density the shard
+  // keeps).  Measured on B200: d < 0.12 (large and small at
+  // 17M) variant 55 = (4, 8, 20, 16, dynamic): large 2.21 ms vs 2.24 static
+  // (40) and 2.47 for k_gather_s3 (25); 0.12 <= d < 0.25 variant 56 = (2, 8, 16,
+  // 24, dynamic): large 8M 1.41 vs 1.42 / 1.48 / 1.61 ms for 44 / 40 / 20;
+  // d >= 0.25, N < 100k: k_gather_s3 (2, 2, 8, 24) = variant 20 (large 4M 1.02
+  // vs 1.07 ms for 44, small 4M 0.29 vs 0.31); d >= 0.15 on grids of >= 100k
+  // points per nuclide (XL 170M, cold 9.5 GB interval table): variant 57 =
+  // (2, 4, 16, 24): 32.2 vs 33.5 ms for 20.
   int v = g.unroll;
   if (v == 0) {
     const double d = static_cast<double>(g.N) * 128.0 / static_cast<double>(P.count ? P.count : 1);
-    v = (d >= 0.25 || (d >= 0.15 && g.N >= 100000)) ? 20 : (d >= 0.12 ? 44 : 40);
+    if (d >= 0.15 && g.N >= 100000)
+      v = 57;
+    else
+      v = d >= 0.25 ? 20 : (d >= 0.12 ? 56 : 55);
   }
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
@@ -3234,6 +3249,10 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     case 49: return launch_gather_s4<GT, 3, 4, 8, 24, CHECK>(g, P, st);
 
     case 50: return launch_gather_s4<GT, 3, 8, 16, 20, CHECK>(g, P, st);
+    case 55: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, false, true>(g, P, st);
+    case 56: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK, false, true>(g, P, st);
+    case 57: return launch_gather_s4<GT, 2, 4, 16, 24, CHECK>(g, P, st);
+    case 58: return launch_gather_s4<GT, 2, 2, 12, 24, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
 }
@@ -3412,7 +3431,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
-                      (variant >= 40 && variant <= 50);
+                      (variant >= 40 && variant <= 50) || (variant >= 55 && variant <= 58);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)

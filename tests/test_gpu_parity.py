@@ -75,7 +75,8 @@ def _compare(out, ref, mode_index=True):
                                      "sort-v20", "sort-v21", "sort-v22", "sort-v23",
                                      "sort-v24", "sort-v25", "sort-v26", "sort-v27", "sort-v28",
                                      "sort-v40", "sort-v41", "sort-v42", "sort-v43", "sort-v44",
-                                     "sort-v45", "sort-v49", "sort-v50"])
+                                     "sort-v45", "sort-v49", "sort-v50", "sort-v55", "sort-v56",
+                                     "sort-v57", "sort-v58"])
 def test_tiny_full_parity(X, variant):
     g = X.Grid.from_preset("tiny")
     kw = {}
@@ -453,7 +454,7 @@ def test_explicit_host_io_chunked(X, sort):
 
 
 @pytest.mark.parametrize("variant", [0, 9, 17, 19, 20, 21, 25, 28, 40, 41, 42, 43, 44, 45, 49,
-                                     50])
+                                     50, 55, 56, 57, 58])
 @pytest.mark.parametrize("grid_type,bins", [("unionized", 0), ("hash", 97)])
 def test_vsum_only_sorted(X, variant, grid_type, bins):
     """Sorted batches with only vsum requested (no per-lookup outputs: the
