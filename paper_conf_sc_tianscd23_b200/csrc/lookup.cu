@@ -601,6 +601,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_scatter(Params P) {
 // Only shared-memory atomics.  Order inside a fine bin is arbitrary: results
 // never depend on it.
 constexpr int kPartItems = kPrepItems;
+constexpr int kPlaceThreads = 512;  // k_part_place: 2 chunks of a tile in flight (one block per SM)
 constexpr uint32_t kPartChunk = kPrepThreads * kPartItems;  // lookups per block round
 // tiles of 8 chunks up to 2^15 tiles (268M lookups; H [tiles][nkeys] is
 // 218 MB there, reserved by workspace_layout), longer tiles beyond
@@ -642,11 +643,12 @@ __device__ __forceinline__ bool in_shard(const Params& P, double p) {
 // chunk's first lookup, tA, tC = LCG^(2 kPartItems t).
 __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint64_t sc, uint64_t tA,
                                              uint64_t tC, const uint8_t* s_pick,
-                                             Sample (&smp)[kPartItems], bool (&ok)[kPartItems]) {
+                                             Sample (&smp)[kPartItems], bool (&ok)[kPartItems],
+                                             uint32_t tid = threadIdx.x) {
   uint64_t st = (tA * sc + tC) & kMask63;
 #pragma unroll
   for (int it = 0; it < kPartItems; ++it) {
-    const uint64_t i = c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it;
+    const uint64_t i = c0 + static_cast<uint64_t>(kPartItems) * tid + it;
     ok[it] = i < P.count;
     if (P.in_energy) {
       smp[it] = ok[it] ? get_lookup(P, static_cast<uint32_t>(i)) : Sample{0.0, 0};
@@ -665,12 +667,13 @@ __device__ __forceinline__ void part_samples(const Params& P, uint64_t c0, uint6
 // fast-forward per tile.
 struct PartStream {
   uint64_t cA, cC, tA, tC;
-  __device__ __forceinline__ void init(const Params& P) {
+  __device__ __forceinline__ void init(const Params& P, uint32_t tid = threadIdx.x,
+                                       uint32_t chunk_stride = 1) {
     cA = tA = 1;
     cC = tC = 0;
     if (P.in_energy) return;
-    affine_pow(2ull * kPartChunk, cA, cC);
-    affine_pow(2ull * kPartItems * threadIdx.x, tA, tC);
+    affine_pow(2ull * kPartChunk * chunk_stride, cA, cC);
+    affine_pow(2ull * kPartItems * tid, tA, tC);
   }
   __device__ __forceinline__ uint64_t at(const Params& P, uint64_t first) const {
     return P.in_energy ? 0 : fast_forward(P.seed, 2 * (P.first_id + first));
@@ -882,8 +885,13 @@ __global__ void __launch_bounds__(1024) k_part_keyscan(Params P) {
 // to its rank inside the tile's coarse-key order in shared memory (the tile's
 // per-key counts are the differences of the scanned H rows), then the tile
 // leaves as runs of consecutive positions (coalesced stores).
-template <int GT>
-__global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
+// NT threads per block: NT / kPrepThreads chunks of the tile in flight at
+// once (each kPrepThreads-thread slice samples every (NT / kPrepThreads)-th
+// chunk; the tile and its order are those of k_part_count)
+template <int GT, int NT>
+__global__ void __launch_bounds__(NT) k_part_place(Params P) {
+  constexpr uint32_t kSlices = NT / kPrepThreads;
+  static_assert(NT % kPrepThreads == 0, "whole chunk slices");
   extern __shared__ __align__(16) unsigned char smem_pl[];
   const int nkeys = (P.n_mats + 1) * P.nkr;
   const int nvalid = P.n_mats * P.nkr;
@@ -898,19 +906,22 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
   uint32_t* s_i = reinterpret_cast<uint32_t*>(s_k + tlen);
   __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
   pick_table_fill(s_pick);  // (first use after the tile loop's barrier)
+  const uint32_t slice = threadIdx.x / kPrepThreads, lt = threadIdx.x % kPrepThreads;
   PartStream ps;
-  ps.init(P);
+  ps.init(P, lt, kSlices);
+  uint64_t sA = 1, sC = 0;  // LCG^(2 kPartChunk slice): this slice's first chunk
+  if (!P.in_energy) affine_pow(2ull * kPartChunk * slice, sA, sC);
   for (uint32_t tl = blockIdx.x; tl < ntiles; tl += gridDim.x) {
     const uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
     const uint32_t* nxt = tl + 1 < ntiles ? row + nkeys : nullptr;
     // local exclusive scan of the tile's per-key counts (keys in order; the
     // invalid material's keys come last)
-    const int per = (nkeys + kPrepThreads - 1) / kPrepThreads;
+    const int per = (nkeys + NT - 1) / NT;
     const int k0 = threadIdx.x * per, k1 = min(nkeys, k0 + per);
     uint32_t sum = 0;
     for (int k = k0; k < k1; ++k) sum += (nxt ? nxt[k] : P.key_tot[k]) - row[k];
     uint32_t ex;
-    block_excl_scan_n<kPrepThreads>(sum, &ex);
+    block_excl_scan_n<NT>(sum, &ex);
     for (int k = k0; k < k1; ++k) {
       s_ls[k] = ex;
       s_lc[k] = ex;
@@ -920,7 +931,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
     __syncthreads();
     const uint32_t nloc = s_ls[nvalid];  // valid lookups of the tile
     if (P.slab_p) {  // shard: the tile's lookups of the shard, kept by k_part_count
-      for (uint32_t i = threadIdx.x; i < nloc; i += kPrepThreads) {
+      for (uint32_t i = threadIdx.x; i < nloc; i += NT) {
         const uint64_t at = static_cast<uint64_t>(tl) * tlen + i;
         const uint64_t kk = P.slab_k[at];
         const uint32_t key = static_cast<uint32_t>(kk & 0xffffu);
@@ -931,12 +942,13 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
       }
     }
     uint64_t sc = ps.at(P, tl * tlen);
-    for (uint32_t c = 0; c < tchunks && !P.slab_p; ++c, sc = ps.next(sc)) {
+    sc = (sA * sc + sC) & kMask63;
+    for (uint32_t c = slice; c < tchunks && !P.slab_p; c += kSlices, sc = ps.next(sc)) {
       const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
       if (c0 >= P.count) break;
       Sample smp[kPartItems];
       bool ok[kPartItems];
-      part_samples(P, c0, sc, ps.tA, ps.tC, s_pick, smp, ok);
+      part_samples(P, c0, sc, ps.tA, ps.tC, s_pick, smp, ok, lt);
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
         if (!ok[it] || smp[it].mat >= P.n_mats) continue;  // invalid lookups are not gathered
@@ -945,11 +957,11 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_place(Params P) {
         s_p[q] = smp[it].p;
         s_k[q] = static_cast<uint16_t>(key);
         if (P.sidx_tmp)
-          s_i[q] = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it);
+          s_i[q] = static_cast<uint32_t>(c0 + static_cast<uint64_t>(kPartItems) * lt + it);
       }
     }
     __syncthreads();
-    for (uint32_t i = threadIdx.x; i < nloc; i += kPrepThreads) {
+    for (uint32_t i = threadIdx.x; i < nloc; i += NT) {
       const uint32_t k = s_k[i];
       const uint32_t d = s_gb[k] + (i - s_ls[k]);
       P.sp_tmp[d] = s_p[i];
@@ -2695,6 +2707,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   NucWin* s_k = reinterpret_cast<NucWin*>(mine + 2 * static_cast<size_t>(C) * kE * 16);
   uint64_t* s_bar = reinterpret_cast<uint64_t*>(s_k + P.max_nucs);              // [2]
   const uint32_t buf_base = smem_u32(s_buf);
+  const uint32_t sk_base = smem_u32(s_k);
   if (lane == 0) {
     mbar_init(&s_bar[0], 32);
     mbar_init(&s_bar[1], 32);
@@ -2771,6 +2784,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
       if (!valid[r]) p[r] = r > 0 ? p[r - 1] : plo;
     const int nn = G.num[m];
     const MatEntry* row = s_tab + G.roff[m];
+    const uint32_t row_base = smem_u32(row);
     // A4 for the two extremes of every nuclide, and each window's place in
     // its group buffer (segmented scan of the sizes over groups of D lanes;
     // 32 nuclides per round, so groups never straddle rounds)
@@ -2846,8 +2860,14 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
         mbar_wait(&s_bar[g & 1], (phase >> (g & 1)) & 1u);
         phase ^= 1u << (g & 1);
       }
-      const NucWin w = s_k[j];
-      const double conc = row[j].conc;
+      // the step's window record and concentration through 32-bit shared
+      // addresses (no generic-to-shared conversion per step)
+      NucWin w;
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(w.klo), "=r"(w.khi), "=r"(w.noff), "=r"(w.off)
+                   : "r"(sk_base + 16u * j));
+      double conc;
+      asm volatile("ld.shared.f64 %0, [%1];" : "=d"(conc) : "r"(row_base + 16u * j));
       const int n_int = w.khi - w.klo;
       if (w.off != kNoBuf) {
         stage_nuclide_iv<R>(WinSmem{w.off}, n_int, conc, p, acc);
@@ -3492,10 +3512,10 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     k_part_keyscan<<<1, 1024, 0, st>>>(P);
     {
       const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup);
-      e = cudaFuncSetAttribute(k_part_place<GT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               static_cast<int>(pl_smem));
+      e = cudaFuncSetAttribute(k_part_place<GT, kPlaceThreads>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(pl_smem));
       if (e != cudaSuccess) return e;
-      k_part_place<GT><<<nb, kPrepThreads, pl_smem, st>>>(P);
+      k_part_place<GT, kPlaceThreads><<<nb, kPlaceThreads, pl_smem, st>>>(P);
     }
     {
       // window: fine_cap energies (2/3 of it with batch positions), default
