@@ -799,6 +799,8 @@ def run_ours(a, pre, cfg):
             "a9_allreduce_ms_per_step": a9_ms,
             "gpu_launches": int(tm["kernel_launches"]),
             "hash": D.global_hash(vglob), "lookups_per_step": vglob[1],
+            "oracle_hash": (gold.get("hash_f32" if f32 else "hash") if gold and
+                            vglob[1] == gold["lookups"] else None),
             "hash_matches_oracle": hash_check, "init_s": round(init_s, 2),
             "grid_device_bytes": int(g.info.device_bytes)}
     # ------------------------------------------------------------- e2e leg
