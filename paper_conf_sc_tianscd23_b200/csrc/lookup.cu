@@ -155,6 +155,8 @@ struct Params {
   int kc_lo;
   int shard;            // 1: only lookups with e_lo <= p < e_hi are looked up
   double e_lo, e_hi;    //    (energy-range shard, xs_lookup_batch_shard)
+  uint64_t s_lo, s_hi;  // the same range on the raw LCG state of the energy draw:
+                        // e_lo <= RN(s) 2^-63 < e_hi <=> s_lo <= s < s_hi
   double* slab_p;       // shard mode: k_part_count keeps the tile's lookups of the
   uint64_t* slab_k;     // shard (energy; position << 16 | key) for k_part_place
   int fine_direct;      // k_part_fine scatters directly above this many windows
@@ -749,7 +751,6 @@ constexpr int kShardWarps = kPrepThreads / 32;
 __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
   extern __shared__ uint32_t s_h[];  // [nkeys]
   __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
-  __shared__ double s_cp[kShardWarps][32 * kPartItems];
   __shared__ uint64_t s_cs[kShardWarps][32 * kPartItems];
   __shared__ uint32_t s_ci[kShardWarps][32 * kPartItems];
   __shared__ uint32_t s_kept;
@@ -771,25 +772,26 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
       if (c0 >= P.count) break;
       uint64_t st = (ps.tA * sc + ps.tC) & kMask63;
       uint32_t run = 0;
+      const bool full = c0 + kPartChunk <= P.count;
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
         const uint64_t i = c0 + static_cast<uint64_t>(kPartItems) * threadIdx.x + it;
-        st = lcg_next(st);
-        const double pe = lcg_double(st);
-        st = lcg_next(st);
-        const bool keep = i < P.count && pe >= P.e_lo && pe < P.e_hi;
+        const uint64_t s1 = lcg_next(st);  // the energy draw's state
+        st = lcg_next(s1);
+        // range test on the state (no conversion for the ~(n-1)/n dropped)
+        const bool keep = (full || i < P.count) && s1 >= P.s_lo && s1 < P.s_hi;
         const uint32_t ball = __ballot_sync(0xffffffffu, keep);
         if (keep) {
           const uint32_t q = run + __popc(ball & ((1u << lane) - 1u));
-          s_cp[warp][q] = pe;
-          s_cs[warp][q] = st;
+          s_cs[warp][q] = s1;
           s_ci[warp][q] = static_cast<uint32_t>(i);
         }
         run += __popc(ball);
       }
       __syncwarp();
       for (uint32_t q = lane; q < run; q += 32) {
-        const Sample smp{s_cp[warp][q], pick_material_tab(s_pick, s_cs[warp][q])};
+        const uint64_t s1 = s_cs[warp][q];
+        const Sample smp{lcg_double(s1), pick_material_tab(s_pick, lcg_next(s1))};
         const uint32_t key = part_key(P, smp);
         atomicAdd(&s_h[key], 1u);
         const uint32_t at_q = atomicAdd(&s_kept, 1u);
@@ -3474,6 +3476,20 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     P.shard = a.shard ? 1 : 0;
     P.e_lo = a.e_lo;
     P.e_hi = a.e_hi;
+    if (a.shard) {  // min{s : RN(s) 2^-63 >= e} by bisection (RN is monotone)
+      auto first_at_least = [](double e) -> uint64_t {
+        if (!(e > 0.0)) return 0;
+        if (lcg_double(kMask63) < e) return kMask63 + 1;
+        uint64_t lo = 0, hi = kMask63;  // lcg_double(lo) < e <= lcg_double(hi)
+        while (hi - lo > 1) {
+          const uint64_t mid = lo + (hi - lo) / 2;
+          if (lcg_double(mid) >= e) hi = mid; else lo = mid;
+        }
+        return hi;
+      };
+      P.s_lo = first_at_least(a.e_lo);
+      P.s_hi = first_at_least(a.e_hi);
+    }
     P.fine_direct = g.fine_direct;
     const int nkeys = static_cast<int>(pk.nkeys(g.n_mats));
     const uint32_t ntiles = part_tiles(a.count);
