@@ -282,13 +282,15 @@ xs_status xs_nuclide_index(const xs_grid* g, const double* energy, const int32_t
 xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_t count,
                        void* host_dst);
 
-/* Tuning knobs: "variant" (gather kernel: 0 = default, 1-4, 9-12, 17-28,
- * 31-36 = the kernel shapes listed in DESIGN.md §4), "blocks_per_sm"
+/* Tuning knobs: "variant" (gather kernel: 0 = the default, chosen by batch
+ * density for sorted batches and k_gather_u for unsorted ones; 1-4, 9-12,
+ * 17-28, 31-36, 40-58 = the kernel shapes listed in DESIGN.md §4 and
+ * lookup.cu), "blocks_per_sm"
  * (0 = occupancy calculator), "legacy_sort" (1: XS_FLAG_SORT through the
  * global-atomic bins and a permutation instead of the partitioned counting
  * sort; comparison only), "part_cbits" (coarse energy bits of the partitioned
  * sort, 6-9; 0 = the default, 7; a value whose tables do not fit the batch
- * falls back to 7), "fine_direct" (the sort's fine pass scatters a coarse
+ * or the workspace falls back to the widest that does), "fine_direct" (the sort's fine pass scatters a coarse
  * key's segment in one pass when it exceeds this many shared-memory windows,
  * else sorts it window by window; default 2), "fine_cap" (that window in
  * energies, 2048-24576; 0 = the default 24576) and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in

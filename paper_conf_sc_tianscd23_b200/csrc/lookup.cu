@@ -157,6 +157,8 @@ struct Params {
   double e_lo, e_hi;    //    (energy-range shard, xs_lookup_batch_shard)
   uint64_t s_lo, s_hi;  // the same range on the raw LCG state of the energy draw:
                         // e_lo <= RN(s) 2^-63 < e_hi <=> s_lo <= s < s_hi
+  uint32_t place_cap;   // k_part_place: tile lookups staged in shared memory (rank >= cap:
+                        // stored straight to global memory; = tile length unless sharded)
   double* slab_p;       // shard mode: k_part_count keeps the tile's lookups of the
   uint64_t* slab_k;     // shard (energy; position << 16 | key) for k_part_place
   int fine_direct;      // k_part_fine scatters directly above this many windows
@@ -903,9 +905,10 @@ __global__ void __launch_bounds__(NT) k_part_place(Params P) {
   uint32_t* s_ls = reinterpret_cast<uint32_t*>(smem_pl);   // [nkeys + 1] local starts
   uint32_t* s_lc = s_ls + nkeys + 1;                       // [nkeys] local cursors
   uint32_t* s_gb = s_lc + nkeys;                           // [nkeys] global bases
+  const uint32_t cap = P.place_cap;  // staged lookups per tile
   double* s_p = reinterpret_cast<double*>(smem_pl + ((3 * static_cast<size_t>(nkeys) + 1) * 4 + 15) / 16 * 16);
-  uint16_t* s_k = reinterpret_cast<uint16_t*>(s_p + tlen);
-  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_k + tlen);
+  uint16_t* s_k = reinterpret_cast<uint16_t*>(s_p + cap);
+  uint32_t* s_i = reinterpret_cast<uint32_t*>(s_k + cap);
   __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
   pick_table_fill(s_pick);  // (first use after the tile loop's barrier)
   const uint32_t slice = threadIdx.x / kPrepThreads, lt = threadIdx.x % kPrepThreads;
@@ -938,9 +941,15 @@ __global__ void __launch_bounds__(NT) k_part_place(Params P) {
         const uint64_t kk = P.slab_k[at];
         const uint32_t key = static_cast<uint32_t>(kk & 0xffffu);
         const uint32_t q = atomicAdd(&s_lc[key], 1u);
-        s_p[q] = P.slab_p[at];
-        s_k[q] = static_cast<uint16_t>(key);
-        if (P.sidx_tmp) s_i[q] = static_cast<uint32_t>(kk >> 16);
+        if (q < cap) {
+          s_p[q] = P.slab_p[at];
+          s_k[q] = static_cast<uint16_t>(key);
+          if (P.sidx_tmp) s_i[q] = static_cast<uint32_t>(kk >> 16);
+        } else {  // beyond the staging capacity: straight to its place
+          const uint32_t d = s_gb[key] + (q - s_ls[key]);
+          P.sp_tmp[d] = P.slab_p[at];
+          if (P.sidx_tmp) P.sidx_tmp[d] = static_cast<uint32_t>(kk >> 16);
+        }
       }
     }
     uint64_t sc = ps.at(P, tl * tlen);
@@ -963,7 +972,8 @@ __global__ void __launch_bounds__(NT) k_part_place(Params P) {
       }
     }
     __syncthreads();
-    for (uint32_t i = threadIdx.x; i < nloc; i += NT) {
+    const uint32_t nst = nloc < cap ? nloc : cap;
+    for (uint32_t i = threadIdx.x; i < nst; i += NT) {
       const uint32_t k = s_k[i];
       const uint32_t d = s_gb[k] + (i - s_ls[k]);
       P.sp_tmp[d] = s_p[i];
@@ -2652,7 +2662,7 @@ struct alignas(16) GatherSmem4 {
   uint32_t roff[kMaxMats + 1];  // first table entry of material m (CSR)
 };
 
-template <int C, int NW, bool F32>
+template <int C, bool F32>
 __host__ __device__ constexpr size_t s4_warp_bytes(int max_nucs) {
   return 2 * static_cast<size_t>(C) * (F32 ? kIv32Doubles : kIvDoubles) * 8 +  // buffers
          static_cast<size_t>(max_nucs) * sizeof(NucWin) + 16;                   // windows + bars
@@ -2704,7 +2714,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
     s_tab[i] = me;
   }
   unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab) + ((tab * sizeof(MatEntry) + 15) / 16) * 16;
-  unsigned char* mine = wbase + s4_warp_bytes<C, NW, F32>(P.max_nucs) * warp;
+  unsigned char* mine = wbase + s4_warp_bytes<C, F32>(P.max_nucs) * warp;
   double2* s_buf = reinterpret_cast<double2*>(mine);                            // [2][C * kE]
   NucWin* s_k = reinterpret_cast<NucWin*>(mine + 2 * static_cast<size_t>(C) * kE * 16);
   uint64_t* s_bar = reinterpret_cast<uint64_t*>(s_k + P.max_nucs);              // [2]
@@ -3191,14 +3201,10 @@ static cudaError_t launch_gather_s3(const DeviceGrid& g, const Params& P, cudaSt
 
 template <int GT, int R, int D, int C, int NW, bool CHECK, bool F32 = false, bool DYN = false>
 static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaStream_t st) {
-  int tab = 0;
-  {
-    // packed material table size: launch-time upper bound n_mats * max_nucs
-    // would waste shared memory; the kernel packs sum(num_nucs) entries
-    tab = g.tab_total;
-  }
-  const size_t smem = sizeof(GatherSmem4) + ((static_cast<size_t>(tab) * sizeof(MatEntry) + 15) / 16) * 16 +
-                      NW * s4_warp_bytes<C, NW, F32>(g.max_nucs);
+  // the kernel stages the packed material table: sum(num_nucs) entries
+  const size_t smem = sizeof(GatherSmem4) +
+                      ((static_cast<size_t>(g.tab_total) * sizeof(MatEntry) + 15) / 16) * 16 +
+                      NW * s4_warp_bytes<C, F32>(g.max_nucs);
   auto kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32, DYN>;
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -3527,7 +3533,18 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       k_part_colscan<2, 512><<<(nkeys + 1) / 2, dim3(2, 512), 0, st>>>(P, static_cast<int>(ntiles));
     k_part_keyscan<<<1, 1024, 0, st>>>(P);
     {
-      const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup);
+      // staging: the whole tile, or (shard) its expected share with a wide
+      // margin (ranks beyond it are stored directly), so that several blocks
+      // share an SM
+      const uint32_t tlen = part_tile_chunks(a.count) * kPartChunk;
+      P.place_cap = tlen;
+      if (a.shard) {
+        const double lo = a.e_lo > 0.0 ? a.e_lo : 0.0, hi = a.e_hi < 1.0 ? a.e_hi : 1.0;
+        const double want = (hi > lo ? hi - lo : 0.0) * 1.25 * tlen + 1024.0;
+        if (want < tlen) P.place_cap = (static_cast<uint32_t>(want) + 255u) & ~255u;
+      }
+      const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup) -
+                             static_cast<size_t>(tlen - P.place_cap) * (per_lookup ? 14 : 10);
       e = cudaFuncSetAttribute(k_part_place<GT, kPlaceThreads>,
                                cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(pl_smem));
       if (e != cudaSuccess) return e;
