@@ -54,3 +54,17 @@ def test_reference_arm_rsbench():
     assert len(lines) == 1
     d = _check(lines[0], "rs-tiny")
     assert d["metric"] == "RS lookups/sec"
+
+
+def test_reference_arm_self_launch_two_ranks():
+    """`bench.py --gpus 2` outside torchrun starts the two ranks itself
+    (torch.distributed.run on 127.0.0.1) and relays rank 0's single line."""
+    e = {k: v for k, v in os.environ.items()
+         if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "MASTER_ADDR", "MASTER_PORT")}
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--impl", "reference",
+                        "--config", "tiny", "--steps", "2", "--warmup", "1", "--cpu-seconds", "0.3"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=600, env=e)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    assert _check(lines[0])["n_gpus"] == 2
