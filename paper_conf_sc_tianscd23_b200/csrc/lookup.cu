@@ -2862,16 +2862,15 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
 
     Acc acc;
     acc.zero();
-    for (int j = 0; j < nn; ++j) {
-      if (j % D == 0) {
-        const int g = j / D;
-        if (g >= 1) {
-          __syncwarp();  // every lane is done with buffer (g + 1) & 1 (group g - 1)
-          issue_group(g + 1);
-        }
-        mbar_wait(&s_bar[g & 1], (phase >> (g & 1)) & 1u);
-        phase ^= 1u << (g & 1);
+    for (int g = 0; g * D < nn; ++g) {  // groups of D nuclides
+      if (g >= 1) {
+        __syncwarp();  // every lane is done with buffer (g + 1) & 1 (group g - 1)
+        issue_group(g + 1);
       }
+      mbar_wait(&s_bar[g & 1], (phase >> (g & 1)) & 1u);
+      phase ^= 1u << (g & 1);
+      const int jend = (g + 1) * D < nn ? (g + 1) * D : nn;
+    for (int j = g * D; j < jend; ++j) {
       // the step's window record and concentration through 32-bit shared
       // addresses (no generic-to-shared conversion per step)
       NucWin w;
@@ -2888,6 +2887,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
         stage_nuclide_iv<R>(WinGlobal{g2}, n_int, conc, p, acc);
       }
       if ((j & (kF32Block - 1)) == kF32Block - 1) acc.flush();
+    }
     }
     if (nn & (kF32Block - 1)) acc.flush();
     __syncwarp();
