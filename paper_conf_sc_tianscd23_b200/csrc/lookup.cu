@@ -2315,7 +2315,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s3(Params P) {
       const MatEntry me = row[j];
       int32_t klo, khi;
       if (GT == XS_GRID_UNIONIZED) {
-        if (P.index_t) {
+        if (!P.index) {  // column layout only without rows (a row read is 2 x ~1.4 KB per task)
           klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
           khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
         } else {
@@ -2808,7 +2808,7 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
         const MatEntry me = row[j];
         noff = me.noff;
         if (GT == XS_GRID_UNIONIZED) {
-          if (P.index_t) {
+          if (!P.index) {  // column layout only without rows (a row read is 2 x ~1.4 KB per task)
             klo = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + ulo);
             khi = __ldg(P.index_t + static_cast<int64_t>(me.n) * P.NU + uhi);
           } else {
@@ -3312,12 +3312,28 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
 template <int GT>
 static cudaError_t launch_gather_u1(const DeviceGrid& g, const Params& P, bool sorted, bool f32,
                                     bool check, cudaStream_t st) {
+#ifndef XS_DEV_FAST
   if (f32)
     return check ? launch_gather_f32<GT, true>(g, P, st) : launch_gather_f32<GT, false>(g, P, st);
+#endif
   const bool thread_kernel = sorted || (GT == XS_GRID_UNIONIZED && !g.index);
+#ifdef XS_DEV_FAST
+  // development build (timing experiments only): unionized, unchecked, sorted
+  if constexpr (GT == XS_GRID_UNIONIZED) {
+    if (!check && thread_kernel) {
+      switch (g.unroll) {
+        case 56: return launch_gather_s4<GT, 2, 8, 16, 24, false, false, true>(g, P, st);
+        case 20: return launch_gather_s3<GT, 2, 2, 8, 24, false>(g, P, st);
+        default: return launch_gather_s4<GT, 4, 8, 20, 16, false, false, true>(g, P, st);
+      }
+    }
+  }
+  return cudaErrorNotSupported;
+#else
   if (thread_kernel)
     return check ? launch_gather_tv<GT, true>(g, P, st) : launch_gather_tv<GT, false>(g, P, st);
   return check ? launch_gather_v<GT, true>(g, P, st) : launch_gather_v<GT, false>(g, P, st);
+#endif
 }
 
 // Generated energies (dyadic grid) never need the division range checks;

@@ -26,9 +26,10 @@ def main():
     ap.add_argument("--shards", default="1")
     ap.add_argument("--f32", action="store_true")
     ap.add_argument("--reps", type=int, default=10)
+    ap.add_argument("--index-layout", default="auto")
     a = ap.parse_args()
     gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")))[a.config]
-    g = X.Grid.from_preset(a.config)
+    g = X.Grid.from_preset(a.config, index_layout=a.index_layout)
     L = a.lookups or X.PRESETS[a.config]["lookups"]
     st = torch.cuda.current_stream()
     for v in [int(x) for x in a.variants.split(",")]:
