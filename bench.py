@@ -59,7 +59,7 @@ def parse():
     ap.add_argument("--lookups", type=int, default=0, help="override lookups per GPU (weak)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo: host-side A9, for single-GPU testing "
                          "of the multi-rank path; ranks then share GPUs round-robin)")
