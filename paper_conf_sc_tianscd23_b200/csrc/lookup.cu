@@ -157,6 +157,8 @@ struct Params {
   double e_lo, e_hi;    //    (energy-range shard, xs_lookup_batch_shard)
   uint64_t s_lo, s_hi;  // the same range on the raw LCG state of the energy draw:
                         // e_lo <= RN(s) 2^-63 < e_hi <=> s_lo <= s < s_hi
+  uint32_t tchunks;     // chunks per A2 tile (part_tile_chunks, times the shard
+                        // multiplier for energy-range shards)
   uint32_t place_cap;   // k_part_place: tile lookups staged in shared memory (rank >= cap:
                         // stored straight to global memory; = tile length unless sharded)
   double* slab_p;       // shard mode: k_part_count keeps the tile's lookups of the
@@ -689,7 +691,7 @@ template <int GT>
 __global__ void __launch_bounds__(kPrepThreads) k_part_count(Params P) {
   extern __shared__ uint32_t s_h[];  // [nkeys]
   const int nkeys = (P.n_mats + 1) * P.nkr;
-  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint32_t tchunks = P.tchunks;
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
   const bool outputs = P.out_E || P.out_mat || P.out_gidx || P.out_M || P.out_v;
@@ -757,7 +759,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
   __shared__ uint32_t s_ci[kShardWarps][32 * kPartItems];
   __shared__ uint32_t s_kept;
   const int nkeys = (P.n_mats + 1) * P.nkr;
-  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint32_t tchunks = P.tchunks;
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -899,7 +901,7 @@ __global__ void __launch_bounds__(NT) k_part_place(Params P) {
   extern __shared__ __align__(16) unsigned char smem_pl[];
   const int nkeys = (P.n_mats + 1) * P.nkr;
   const int nvalid = P.n_mats * P.nkr;
-  const uint32_t tchunks = part_tile_chunks(P.count);
+  const uint32_t tchunks = P.tchunks;
   const uint64_t tlen = static_cast<uint64_t>(tchunks) * kPartChunk;
   const uint32_t ntiles = static_cast<uint32_t>((P.count + tlen - 1) / tlen);
   uint32_t* s_ls = reinterpret_cast<uint32_t*>(smem_pl);   // [nkeys + 1] local starts
@@ -3375,8 +3377,8 @@ static cudaError_t launch_gather_u(const DeviceGrid& g, const Params& P, bool so
   return launch_gather_u1<GT>(g, Q, sorted, f32, true, st);
 }
 
-static uint32_t part_tiles(uint64_t count) {
-  const uint64_t tlen = static_cast<uint64_t>(part_tile_chunks(count)) * kPartChunk;
+static uint32_t part_tiles(uint64_t count, uint32_t tchunks = 0) {
+  const uint64_t tlen = static_cast<uint64_t>(tchunks ? tchunks : part_tile_chunks(count)) * kPartChunk;
   const uint64_t t = (count + tlen - 1) / tlen;
   return static_cast<uint32_t>(t < 1 ? 1 : t);
 }
@@ -3490,6 +3492,17 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)
   PartKeys pk = part_keys(a, part_cbits(a.count, g.n_mats, g.part_cbits));
+  if (a.shard && g.part_cbits == 0) {
+    // an energy-range shard whose coarse segments would average more than two
+    // fine-pass windows (XL) takes one more coarse bit: its tile histograms
+    // are small (long shard tiles), and shorter segments sort faster (XL,
+    // 8 shards: A2 0.73 -> 0.58 ms)
+    const double frac = (a.e_hi < 1.0 ? a.e_hi : 1.0) - (a.e_lo > 0.0 ? a.e_lo : 0.0);
+    const double per_key = static_cast<double>(a.count) * (frac > 0.0 ? frac : 0.0) /
+                           (static_cast<double>(g.n_mats) * pk.nkr);
+    if (per_key > 2.0 * kFineCapP && part_cbits_fit(a.count, g.n_mats, pk.cbits + 1))
+      pk = part_keys(a, pk.cbits + 1);
+  }
   while (pk.cbits > kPartCbitsMin &&
          part_bins_need(a.count, pk.nkeys(g.n_mats)) > ws.bins_bytes)
     pk = part_keys(a, pk.cbits - 1);
@@ -3524,7 +3537,22 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
     }
     P.fine_direct = g.fine_direct;
     const int nkeys = static_cast<int>(pk.nkeys(g.n_mats));
-    const uint32_t ntiles = part_tiles(a.count);
+    // an energy-range shard keeps ~1/n of each tile's lookups: its tiles are
+    // n/2 times longer (up to 16x), so that the tile histograms, their column
+    // scan and the per-tile stream setup shrink while k_part_place still
+    // stages few enough lookups per tile for two blocks per SM (measured,
+    // large: n/2 beats 1 and n at n = 2, 4, 8)
+    uint32_t tmult = 1;
+    if (a.shard) {
+      const double lo = a.e_lo > 0.0 ? a.e_lo : 0.0, hi = a.e_hi < 1.0 ? a.e_hi : 1.0;
+      const double inv = hi > lo ? 0.5 / (hi - lo) : 16.0;
+      tmult = inv >= 16.0 ? 16u : static_cast<uint32_t>(inv);
+      const uint32_t cap = g.shard_tiles ? static_cast<uint32_t>(g.shard_tiles) : 16u;
+      if (tmult > cap) tmult = cap;
+      if (tmult < 1) tmult = 1;
+    }
+    P.tchunks = part_tile_chunks(a.count) * tmult;
+    const uint32_t ntiles = part_tiles(a.count, P.tchunks);
     const unsigned nb = ntiles < static_cast<uint32_t>(g.sm_count) * 16 ? ntiles : g.sm_count * 16;
     P.bins = ws.bins;  // H [ntiles][nkeys]
     P.key_tot = ws.bins + static_cast<size_t>(ntiles) * nkeys;
@@ -3562,15 +3590,15 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
       // staging: the whole tile, or (shard) its expected share with a wide
       // margin (ranks beyond it are stored directly), so that several blocks
       // share an SM
-      const uint32_t tlen = part_tile_chunks(a.count) * kPartChunk;
+      const uint32_t tlen = P.tchunks * kPartChunk;
       P.place_cap = tlen;
       if (a.shard) {
         const double lo = a.e_lo > 0.0 ? a.e_lo : 0.0, hi = a.e_hi < 1.0 ? a.e_hi : 1.0;
         const double want = (hi > lo ? hi - lo : 0.0) * 1.25 * tlen + 1024.0;
         if (want < tlen) P.place_cap = (static_cast<uint32_t>(want) + 255u) & ~255u;
       }
-      const size_t pl_smem = part_place_smem(a.count, g.n_mats, P.cbits, per_lookup) -
-                             static_cast<size_t>(tlen - P.place_cap) * (per_lookup ? 14 : 10);
+      const size_t pl_smem = (static_cast<size_t>(3 * nkeys + 1) * 4 + 15) / 16 * 16 +
+                             static_cast<size_t>(P.place_cap) * (per_lookup ? 14 : 10);
       e = cudaFuncSetAttribute(k_part_place<GT, kPlaceThreads>,
                                cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(pl_smem));
       if (e != cudaSuccess) return e;

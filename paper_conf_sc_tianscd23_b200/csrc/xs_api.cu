@@ -782,6 +782,9 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
     if (value != 0 && (value < 2048 || value > 24576))
       return fail(XS_ERR_INVALID_ARG, "fine_cap is 0 (default) or 2048-24576");
     G.fine_cap = static_cast<int>(value);
+  } else if (!std::strcmp(name, "shard_tiles")) {
+    if (value < 0 || value > 16) return fail(XS_ERR_INVALID_ARG, "shard_tiles in [0,16]");
+    G.shard_tiles = static_cast<int>(value);
   } else {
     return fail(XS_ERR_INVALID_ARG, std::string("unknown parameter ") + name);
   }

@@ -54,6 +54,7 @@ struct DeviceGrid {
   int part_cbits = 0;      // partitioned A2 coarse energy bits (0 = default)
   int fine_direct = 2;     // k_part_fine: direct scatter above this many windows
   int fine_cap = 0;        // k_part_fine window in energies (0 = default 24576)
+  int shard_tiles = 0;     // energy-range shards: A2 tile-length multiplier cap (0 = default)
   // instrumentation (host side)
   uint64_t launches = 0;   // kernels launched by lookup calls
 };
