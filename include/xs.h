@@ -289,8 +289,12 @@ xs_status xs_get_table(const xs_grid* g, int32_t table, uint64_t offset, uint64_
  * (0 = occupancy calculator), "legacy_sort" (1: XS_FLAG_SORT through the
  * global-atomic bins and a permutation instead of the partitioned counting
  * sort; comparison only), "part_cbits" (coarse energy bits of the partitioned
- * sort, 6-9; 0 = the default, 7; a value whose tables do not fit the batch
- * or the workspace falls back to the widest that does), "fine_direct" (the sort's fine pass scatters a coarse
+ * sort, 6-9; 0 = the default, 7, or 8 for an energy-range shard whose coarse
+ * segments would average more than two fine-pass windows; a value whose
+ * tables do not fit the batch or the workspace falls back to the widest that
+ * does), "shard_tiles" (energy-range shards: cap on the factor by which the
+ * sort's tiles are lengthened, 1-16; 0 = the default, n/2 for a 1/n shard),
+ * "fine_direct" (the sort's fine pass scatters a coarse
  * key's segment in one pass when it exceeds this many shared-memory windows,
  * else sorts it window by window; default 2), "fine_cap" (that window in
  * energies, 2048-24576; 0 = the default 24576) and "host_chunk" (XS_FLAG_HOST_IO explicit lookups upload their inputs in

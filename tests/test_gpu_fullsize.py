@@ -247,6 +247,58 @@ def test_energy_shards_large_f32_and_hash(X):
         g.close()
 
 
+@pytest.mark.parametrize("R,tiles,cbits", [(8, 1, 0), (8, 16, 0), (3, 2, 8), (8, 0, 8), (32, 0, 0)])
+def test_energy_shard_tiles_and_keys(X, R, tiles, cbits):
+    """The shard A2 knobs (tile-length factor, coarse key bits) never change
+    results: R shards of the 17M small batch sum to the oracle's verification
+    sum (R = 32 lengthens the tiles 16-fold), and the shards of a tiny batch
+    reproduce every lookup."""
+    g = X.Grid.from_preset("small")
+    g.set_param("shard_tiles", tiles)
+    g.set_param("part_cbits", cbits)
+    L = 17_000_000
+    vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+    for r in range(R):
+        g.lookup_shard(0, L, r, R, vsum=vsum)
+    torch.cuda.synchronize()
+    assert [int(x) for x in vsum.cpu()] == [GOLDEN["small"]["sum_v"], L]
+    g.close()
+    g = X.Grid.from_preset("tiny")
+    g.set_param("shard_tiles", tiles)
+    g.set_param("part_cbits", cbits)
+    L, first = 100_000, 5
+    S, ref = _oracle("tiny", 0).run(first, L, mode=oracle.UNIONIZED, nthreads=NT, outputs=True)
+    _, outs = g.lookup_shard(first, L, 0, R, want=("macro_xs", "verification"))
+    total = torch.zeros(2, dtype=torch.int64, device="cuda")
+    for r in range(R):
+        g.lookup_shard(first, L, r, R, vsum=total, outputs=outs)
+    torch.cuda.synchronize()
+    assert [int(x) for x in total.cpu()] == [S, L]
+    _assert_equal("macro_xs", outs["macro_xs"].cpu().numpy(), ref["M"])
+    _assert_equal("verification", outs["verification"].cpu().numpy(), ref["v"])
+    with pytest.raises(X.XSError):
+        g.set_param("shard_tiles", 17)
+
+
+def test_energy_shards_xl(X):
+    """XL, the north_star's 8-GPU configuration: the 8 energy-range shards of
+    the 170M batch (the launch bench.py's projection times; its shards take
+    the longer tiles and the extra coarse key bit) sum to the oracle's
+    verification sum."""
+    free, _ = torch.cuda.mem_get_info()
+    if free < 140e9:
+        pytest.skip("XL needs ~130 GB of device memory")
+    gold = GOLDEN["xl"]
+    L = gold["lookups"]
+    g = X.Grid.from_preset("xl")
+    vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+    for r in range(8):
+        g.lookup_shard(0, L, r, 8, vsum=vsum)
+    torch.cuda.synchronize()
+    assert [int(x) for x in vsum.cpu()] == [gold["sum_v"], L]
+    g.close()
+
+
 def test_energy_shard_arguments(X):
     g = X.Grid.from_preset("tiny")
     vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
