@@ -755,8 +755,10 @@ constexpr int kShardWarps = kPrepThreads / 32;
 __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
   extern __shared__ uint32_t s_h[];  // [nkeys]
   __shared__ __align__(16) uint8_t s_pick[kPickBuckets];
-  __shared__ uint64_t s_cs[kShardWarps][32 * kPartItems];
-  __shared__ uint32_t s_ci[kShardWarps][32 * kPartItems];
+  // a warp's kept lookups are processed in batches of at least 32 * kPartItems
+  // (all lanes busy): room for one more chunk on top of that
+  __shared__ uint64_t s_cs[kShardWarps][2 * 32 * kPartItems];
+  __shared__ uint32_t s_ci[kShardWarps][2 * 32 * kPartItems];
   __shared__ uint32_t s_kept;
   const int nkeys = (P.n_mats + 1) * P.nkr;
   const uint32_t tchunks = P.tchunks;
@@ -771,11 +773,29 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
     if (threadIdx.x == 0) s_kept = 0;
     __syncthreads();
     uint64_t sc = ps.at(P, tl * tlen);
+    uint32_t run = 0;  // kept lookups staged for this warp
+    // the pick, key, histogram and slab entry of the staged lookups; the
+    // warp's slab slots come from one shared atomic per batch
+    auto flush = [&]() {
+      uint32_t base = 0;
+      if (lane == 0 && run) base = atomicAdd(&s_kept, run);
+      base = __shfl_sync(0xffffffffu, base, 0);
+      for (uint32_t q = lane; q < run; q += 32) {
+        const uint64_t s1 = s_cs[warp][q];
+        const Sample smp{lcg_double(s1), pick_material_tab(s_pick, lcg_next(s1))};
+        const uint32_t key = part_key(P, smp);
+        atomicAdd(&s_h[key], 1u);
+        const uint64_t at = static_cast<uint64_t>(tl) * tlen + base + q;
+        P.slab_p[at] = smp.p;
+        P.slab_k[at] = (static_cast<uint64_t>(s_ci[warp][q]) << 16) | key;
+      }
+      __syncwarp();
+      run = 0;
+    };
     for (uint32_t c = 0; c < tchunks; ++c, sc = ps.next(sc)) {
       const uint64_t c0 = tl * tlen + static_cast<uint64_t>(c) * kPartChunk;
       if (c0 >= P.count) break;
       uint64_t st = (ps.tA * sc + ps.tC) & kMask63;
-      uint32_t run = 0;
       const bool full = c0 + kPartChunk <= P.count;
 #pragma unroll
       for (int it = 0; it < kPartItems; ++it) {
@@ -793,18 +813,9 @@ __global__ void __launch_bounds__(kPrepThreads) k_part_count_shard(Params P) {
         run += __popc(ball);
       }
       __syncwarp();
-      for (uint32_t q = lane; q < run; q += 32) {
-        const uint64_t s1 = s_cs[warp][q];
-        const Sample smp{lcg_double(s1), pick_material_tab(s_pick, lcg_next(s1))};
-        const uint32_t key = part_key(P, smp);
-        atomicAdd(&s_h[key], 1u);
-        const uint32_t at_q = atomicAdd(&s_kept, 1u);
-        const uint64_t at = static_cast<uint64_t>(tl) * tlen + at_q;
-        P.slab_p[at] = smp.p;
-        P.slab_k[at] = (static_cast<uint64_t>(s_ci[warp][q]) << 16) | key;
-      }
-      __syncwarp();
+      if (run >= 32 * kPartItems) flush();
     }
+    flush();
     __syncthreads();
     uint32_t* row = P.bins + static_cast<uint64_t>(tl) * nkeys;
     for (int t = threadIdx.x; t < nkeys; t += blockDim.x) row[t] = s_h[t];
@@ -938,19 +949,32 @@ __global__ void __launch_bounds__(NT) k_part_place(Params P) {
     __syncthreads();
     const uint32_t nloc = s_ls[nvalid];  // valid lookups of the tile
     if (P.slab_p) {  // shard: the tile's lookups of the shard, kept by k_part_count
-      for (uint32_t i = threadIdx.x; i < nloc; i += NT) {
-        const uint64_t at = static_cast<uint64_t>(tl) * tlen + i;
-        const uint64_t kk = P.slab_k[at];
-        const uint32_t key = static_cast<uint32_t>(kk & 0xffffu);
-        const uint32_t q = atomicAdd(&s_lc[key], 1u);
-        if (q < cap) {
-          s_p[q] = P.slab_p[at];
-          s_k[q] = static_cast<uint16_t>(key);
-          if (P.sidx_tmp) s_i[q] = static_cast<uint32_t>(kk >> 16);
-        } else {  // beyond the staging capacity: straight to its place
-          const uint32_t d = s_gb[key] + (q - s_ls[key]);
-          P.sp_tmp[d] = P.slab_p[at];
-          if (P.sidx_tmp) P.sidx_tmp[d] = static_cast<uint32_t>(kk >> 16);
+      // kSlabIlp slab entries in flight per thread (the loop is load-latency bound)
+      constexpr int kSlabIlp = 4;
+      for (uint32_t i0 = threadIdx.x; i0 < nloc; i0 += kSlabIlp * NT) {
+        uint64_t kk[kSlabIlp];
+        double pp[kSlabIlp];
+#pragma unroll
+        for (int u = 0; u < kSlabIlp; ++u) {
+          const uint32_t i = i0 + u * NT;
+          const uint64_t at = static_cast<uint64_t>(tl) * tlen + i;
+          kk[u] = i < nloc ? P.slab_k[at] : 0ull;
+          pp[u] = i < nloc ? P.slab_p[at] : 0.0;
+        }
+#pragma unroll
+        for (int u = 0; u < kSlabIlp; ++u) {
+          if (i0 + u * NT >= nloc) continue;
+          const uint32_t key = static_cast<uint32_t>(kk[u] & 0xffffu);
+          const uint32_t q = atomicAdd(&s_lc[key], 1u);
+          if (q < cap) {
+            s_p[q] = pp[u];
+            s_k[q] = static_cast<uint16_t>(key);
+            if (P.sidx_tmp) s_i[q] = static_cast<uint32_t>(kk[u] >> 16);
+          } else {  // beyond the staging capacity: straight to its place
+            const uint32_t d = s_gb[key] + (q - s_ls[key]);
+            P.sp_tmp[d] = pp[u];
+            if (P.sidx_tmp) P.sidx_tmp[d] = static_cast<uint32_t>(kk[u] >> 16);
+          }
         }
       }
     }
