@@ -621,19 +621,24 @@ def _time_fn(fn, stream, k, warm=2):
     return e0.elapsed_time(e1) / k
 
 
-def strong_projection(g, L, f32, stream, value1, ms1, steps=5):
+def strong_projection(g, L, f32, stream, value1, ms1, steps=5, passes=2):
     """One-GPU projection of strong scaling (L fixed): every rank's shard is
     timed alone on this GPU; the R-GPU step is the slowest shard (the A9
     all-reduce of 16 bytes, ~20 us over NVLink, is not included).  Two
     partitions: energy-range shards (the bench's multi-GPU default,
-    xs_lookup_batch_shard) and contiguous id ranges."""
+    xs_lookup_batch_shard) and contiguous id ranges.  A shard's time is the
+    lower of `passes` means over `steps` steps, so that a transient on the
+    one shared GPU (a clock dip while one shard is timed) does not stand in
+    for that rank's step."""
     out = {}
     for R in (2, 4, 8):
         per_e, per_i = [], []
         for r in range(R):
-            per_e.append(_time_fn(lambda: g.lookup_shard(0, L, r, R, f32=f32), stream, steps))
+            per_e.append(min(_time_fn(lambda: g.lookup_shard(0, L, r, R, f32=f32), stream, steps)
+                             for _ in range(passes)))
             a, b = r * L // R, (r + 1) * L // R
-            per_i.append(_time_fn(lambda: g.lookup(a, b - a, sort=True, f32=f32), stream, steps))
+            per_i.append(min(_time_fn(lambda: g.lookup(a, b - a, sort=True, f32=f32), stream, steps)
+                             for _ in range(passes)))
         me, mi = max(per_e), max(per_i)
         out[str(R)] = {"energy_shards": {"ms_per_step": me, "value": L / (me / 1e3),
                                          "speedup": ms1 / me, "efficiency": ms1 / me / R,
@@ -849,9 +854,9 @@ def run_ours(a, pre, cfg):
         if sort and pre["lookups"] >= 1_000_000:
             line["projection_strong"] = {
                 "note": "one-GPU projection of strong scaling (L fixed): each rank's shard "
-                        "timed alone on this GPU, R-GPU step = slowest shard; A9 (16-byte "
-                        "all-reduce) not included; weak scaling (L per rank, no exchange "
-                        "but A9) projects to R x value",
+                        "timed alone on this GPU (the lower of two 5-step means), R-GPU "
+                        "step = slowest shard; A9 (16-byte all-reduce) not included; weak "
+                        "scaling (L per rank, no exchange but A9) projects to R x value",
                 **strong_projection(g, L, f32, stream, value, ms / a.steps)}
         # config 3 unsorted and the paper's kernel shape, as context
         if sort and not f32:
