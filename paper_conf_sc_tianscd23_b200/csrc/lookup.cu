@@ -3517,14 +3517,17 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   // may allow a wider key than the batch the workspace was sized for)
   PartKeys pk = part_keys(a, part_cbits(a.count, g.n_mats, g.part_cbits));
   if (a.shard && g.part_cbits == 0) {
-    // an energy-range shard whose coarse segments would average more than two
-    // fine-pass windows (XL) takes one more coarse bit: its tile histograms
-    // are small (long shard tiles), and shorter segments sort faster (XL,
-    // 8 shards: A2 0.73 -> 0.58 ms)
+    // an energy-range shard takes one more coarse bit when its coarse
+    // segments would average more than two fine-pass windows (XL) or when its
+    // keys would give the fine pass (one block per key and SM) fewer than
+    // ~2.5 waves (8 shards): its tile histograms are small (long shard
+    // tiles), and more, shorter segments sort faster (A2 per shard, 8 shards:
+    // XL 0.73 -> 0.58 ms, large 0.067 -> 0.057 ms)
     const double frac = (a.e_hi < 1.0 ? a.e_hi : 1.0) - (a.e_lo > 0.0 ? a.e_lo : 0.0);
     const double per_key = static_cast<double>(a.count) * (frac > 0.0 ? frac : 0.0) /
                            (static_cast<double>(g.n_mats) * pk.nkr);
-    if (per_key > 2.0 * kFineCapP && part_cbits_fit(a.count, g.n_mats, pk.cbits + 1))
+    const bool few_keys = 2 * g.n_mats * pk.nkr < 5 * g.sm_count;
+    if ((per_key > 2.0 * kFineCapP || few_keys) && part_cbits_fit(a.count, g.n_mats, pk.cbits + 1))
       pk = part_keys(a, pk.cbits + 1);
   }
   while (pk.cbits > kPartCbitsMin &&

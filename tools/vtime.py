@@ -29,16 +29,19 @@ def main():
     ap.add_argument("--index-layout", default="auto")
     ap.add_argument("--cbits", default="0", help="part_cbits values (comma list) tried per variant")
     ap.add_argument("--shard-tiles", default="0", help="shard_tiles values (comma list)")
+    ap.add_argument("--fine-cap", default="0", help="fine_cap values (comma list)")
     a = ap.parse_args()
     gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_hashes.json")))[a.config]
     g = X.Grid.from_preset(a.config, index_layout=a.index_layout)
     L = a.lookups or X.PRESETS[a.config]["lookups"]
     st = torch.cuda.current_stream()
-    for v, cb, stl in [(int(x), int(c), int(t)) for x in a.variants.split(",")
-                       for c in a.cbits.split(",") for t in a.shard_tiles.split(",")]:
+    for v, cb, stl, fc in [(int(x), int(c), int(t), int(f)) for x in a.variants.split(",")
+                           for c in a.cbits.split(",") for t in a.shard_tiles.split(",")
+                           for f in a.fine_cap.split(",")]:
         g.set_param("variant", v)
         g.set_param("part_cbits", cb)
         g.set_param("shard_tiles", stl)
+        g.set_param("fine_cap", fc)
         for R in [int(x) for x in a.shards.split(",")]:
             worst, worst_ph, vs_tot = 0.0, None, [0, 0]
             for r in range(R):
@@ -70,7 +73,7 @@ def main():
                     worst, worst_ph = ms, ph
             key = "sum_v_f32" if a.f32 else "sum_v"
             ok = vs_tot == [gold[key], L] if L == gold["lookups"] else None
-            print(f"{a.config} L={L} f32={a.f32} variant={v} cbits={cb} stiles={stl} shards={R}: step {worst:.4f} ms "
+            print(f"{a.config} L={L} f32={a.f32} variant={v} cbits={cb} stiles={stl} fcap={fc} shards={R}: step {worst:.4f} ms "
                   f"(count {worst_ph[0]:.4f} bucket {worst_ph[1]:.4f} gather {worst_ph[2]:.4f}) "
                   f"{L / worst / 1e6:.1f} M lookups/ms-equiv  vsum_ok={ok}", flush=True)
 
