@@ -34,6 +34,11 @@ if which == "xs":
         g.lookup_shard(0, L, r, 3, vsum=vs)
     torch.cuda.synchronize()
     print("shards", vs.tolist(), flush=True)
+    vs.zero_()   # 8 shards: lengthened tiles, one more coarse bit
+    for r in range(8):
+        g.lookup_shard(0, L, r, 8, vsum=vs)
+    torch.cuda.synchronize()
+    print("shards8", vs.tolist(), flush=True)
     vs, _ = g.lookup_history(0, 500, 4)
     torch.cuda.synchronize()
     print("history", vs.tolist(), flush=True)
