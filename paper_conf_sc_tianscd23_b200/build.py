@@ -36,24 +36,36 @@ def _stale(out, srcs):
     return any(os.path.getmtime(s) > t for s in srcs)
 
 
+def _nvcc(src: str, verbose: bool) -> None:
+    s = os.path.join(CSRC, src)
+    o = os.path.join(BUILD, src + ".o")
+    cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
+           "-Xptxas", "-v", "-c", s, "-o", o]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if verbose or r.returncode:
+        sys.stderr.write(r.stderr)
+    if r.returncode:
+        raise RuntimeError(f"nvcc failed for {src}")
+    with open(o + ".ptxas.txt", "w") as f:
+        f.write(r.stderr)
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
+    from concurrent.futures import ThreadPoolExecutor
     os.makedirs(BUILD, exist_ok=True)
     objs = []
     deps = _deps()
+    stale = []
     for src in CU_SOURCES:
         s = os.path.join(CSRC, src)
         o = os.path.join(BUILD, src + ".o")
         objs.append(o)
         if force or _stale(o, [s, *deps, __file__]):
-            cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
-                   "-Xptxas", "-v", "-c", s, "-o", o]
-            r = subprocess.run(cmd, capture_output=True, text=True)
-            if verbose or r.returncode:
-                sys.stderr.write(r.stderr)
-            if r.returncode:
-                raise RuntimeError(f"nvcc failed for {src}")
-            with open(o + ".ptxas.txt", "w") as f:
-                f.write(r.stderr)
+            stale.append(src)
+    # the translation units compile concurrently (lookup.cu dominates)
+    with ThreadPoolExecutor(max_workers=max(1, len(stale))) as ex:
+        for f in [ex.submit(_nvcc, src, verbose) for src in stale]:
+            f.result()
     for gen in ("xs_gen", "rs_gen"):
         g = os.path.join(ROOT, "gen", gen + ".cpp")
         go = os.path.join(BUILD, gen + ".o")
