@@ -295,9 +295,12 @@ static xs_status init_common(const xs_grid_data* d, int device, cudaStream_t st,
     return fail(XS_ERR_OUT_OF_MEMORY, "device allocation of the grid tables", e);
   }
   // K0u (unsorted gather): optional, only where it leaves ample memory free
-  // (large: 385 MB; XL: 8.1 GB); without it unsorted batches use k_gather
+  // (large: 385 MB; XL: 8.1 GB); without it unsorted batches use k_gather.
+  // A unionized grid without the row layout (XL) never runs k_gather_u
+  // (its unsorted batches take the staged gather): no K0u
   const size_t ivu_bytes = static_cast<size_t>(I) * N * 12 * sizeof(double);
-  {
+  const bool ivu_usable = !(G.grid_type == XS_GRID_UNIONIZED && !(G.index_layout & XS_INDEX_ROW));
+  if (ivu_usable) {
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     if (free_b > ivu_bytes + (static_cast<size_t>(24) << 30) && cudaMalloc(&G.ivu, ivu_bytes) != cudaSuccess) {
