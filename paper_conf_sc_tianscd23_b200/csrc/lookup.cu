@@ -2679,6 +2679,10 @@ struct alignas(16) NucWin {
                       // buffer, kNoBuf = read in place from global memory
 };
 constexpr uint32_t kNoBuf = 0xffffffffu;
+#ifndef XS_S4_PREFETCH
+#define XS_S4_PREFETCH 1
+#endif
+constexpr bool kS4Prefetch = XS_S4_PREFETCH;
 
 struct alignas(16) GatherSmem4 {
   int32_t num[kMaxMats];
@@ -2688,10 +2692,18 @@ struct alignas(16) GatherSmem4 {
   uint32_t roff[kMaxMats + 1];  // first table entry of material m (CSR)
 };
 
-template <int C, bool F32>
+// the next task's energies are prefetched (1 KB per warp) by the 4-lookups-
+// per-lane shapes with 16 warps (the default for dense batches), whose shared
+// memory leaves room for it
+template <int R, int NW>
+__host__ __device__ constexpr bool s4_prefetch() {
+  return kS4Prefetch && R == 4 && NW <= 16;
+}
+template <int C, bool F32, bool PF = false>
 __host__ __device__ constexpr size_t s4_warp_bytes(int max_nucs) {
   return 2 * static_cast<size_t>(C) * (F32 ? kIv32Doubles : kIvDoubles) * 8 +  // buffers
-         static_cast<size_t>(max_nucs) * sizeof(NucWin) + 16;                   // windows + bars
+         static_cast<size_t>(max_nucs) * sizeof(NucWin) + 16 +                  // windows + bars
+         (PF ? 32 * 4 * 8 : 0);                                                  // next energies
 }
 
 // OUT = false: no per-lookup outputs (verification sum only), so the batch
@@ -2742,10 +2754,13 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
     s_tab[i] = me;
   }
   unsigned char* wbase = reinterpret_cast<unsigned char*>(s_tab) + ((tab * sizeof(MatEntry) + 15) / 16) * 16;
-  unsigned char* mine = wbase + s4_warp_bytes<C, F32>(P.max_nucs) * warp;
+  constexpr bool PF = s4_prefetch<R, NW>();
+  unsigned char* mine = wbase + s4_warp_bytes<C, F32, PF>(P.max_nucs) * warp;
   double2* s_buf = reinterpret_cast<double2*>(mine);                            // [2][C * kE]
   NucWin* s_k = reinterpret_cast<NucWin*>(mine + 2 * static_cast<size_t>(C) * kE * 16);
   uint64_t* s_bar = reinterpret_cast<uint64_t*>(s_k + P.max_nucs);              // [2]
+  // the next task's energies, copied by cp.async during this task (R <= 4)
+  const uint32_t pf_base = smem_u32(s_bar + 2) + static_cast<uint32_t>(lane) * 32u;
   const uint32_t buf_base = smem_u32(s_buf);
   const uint32_t sk_base = smem_u32(s_k);
   if (lane == 0) {
@@ -2767,6 +2782,8 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   // (tasks in material order, fuel first), fetched one task ahead
   uint32_t next = 0;
   if (DYN && lane == 0) next = nwarps + atomicAdd(P.task_next, 1u);
+  const bool pre = PF && !OUT && P.sp && !P.sidx;
+  bool have_pf = false;  // this lane's energies of the task were prefetched
   for (uint32_t task = gw; task < total_tasks;) {
     while (task >= G.toff[m + 1]) ++m;
     const uint32_t slot0 = (task - G.toff[m]) * kTask + lane * R;
@@ -2774,14 +2791,37 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
     int32_t gidx[R];
     uint32_t idx[R];
     bool valid[R];
+    if (have_pf) asm volatile("cp.async.wait_all;" ::: "memory");
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       valid[r] = slot0 + r < G.cnt[m];
       LookupRec rec{0.5, 0u, 0};
-      if (valid[r]) rec = load_rec(P, G.off[m] + slot0 + r);
+      if (have_pf) {
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(rec.p) : "r"(pf_base + 8u * r));
+      } else if (valid[r]) {
+        rec = load_rec(P, G.off[m] + slot0 + r);
+      }
       p[r] = rec.p;
       gidx[r] = rec.gidx;
       idx[r] = OUT ? rec.idx : 0u;
+    }
+    if (pre) {  // the next task's energies (whole lane groups only)
+      const uint32_t nt = DYN ? __shfl_sync(0xffffffffu, next, 0) : task + nwarps;
+      have_pf = false;
+      if (nt < total_tasks) {
+        int mn = m;
+        while (nt >= G.toff[mn + 1]) ++mn;
+        const uint32_t s0n = (nt - G.toff[mn]) * kTask + lane * R;
+        if (s0n + R <= G.cnt[mn]) {
+          const double* src = P.sp + G.off[mn] + s0n;
+#pragma unroll
+          for (int r = 0; r < R; ++r)
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(pf_base + 8u * r),
+                         "l"(src + r)
+                         : "memory");
+          have_pf = true;
+        }
+      }
     }
 #pragma unroll
     for (int pass = 0; pass < R; ++pass) {
@@ -3236,7 +3276,7 @@ static cudaError_t launch_gather_s4(const DeviceGrid& g, const Params& P, cudaSt
   // the kernel stages the packed material table: sum(num_nucs) entries
   const size_t smem = sizeof(GatherSmem4) +
                       ((static_cast<size_t>(g.tab_total) * sizeof(MatEntry) + 15) / 16) * 16 +
-                      NW * s4_warp_bytes<C, F32>(g.max_nucs);
+                      NW * s4_warp_bytes<C, F32, s4_prefetch<R, NW>()>(g.max_nucs);
   auto kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32, DYN, true>;
   if constexpr (SPEC) {
     if (!P.out_v && !P.out_M) kern = k_gather_s4<GT, R, D, C, NW, CHECK, F32, DYN, false>;

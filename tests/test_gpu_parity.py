@@ -142,6 +142,12 @@ def test_ragged_batches(X, first, count, variant):
         vs, out = _full_outputs(g, first, count, sort=sort)
         _compare(out, ref)
         assert vs == [S, count]
+    # the verification sum alone (the bench's launch: output-free gather
+    # instances, next-task energies prefetched; ragged last tasks)
+    vsum = torch.zeros(2, dtype=torch.int64, device="cuda")
+    g.lookup(first, count, sort=True, vsum=vsum)
+    torch.cuda.synchronize()
+    assert [int(x) for x in vsum.cpu()] == [S, count]
 
 
 def test_empty_batch_and_accumulation(X):
