@@ -189,7 +189,10 @@ typedef struct {
                                    32-B aligned entries (K0u): {E[k+1], gap,
                                    (hi.c, hi.c - lo.c) x 5}; entry N-1 is zero;
                                    UNSUPPORTED when the grid did not build it
-                                   (built only with ample free device memory) */
+                                   (built only with ample free device memory,
+                                   and never for a unionized grid without the
+                                   row layout, whose unsorted batches take the
+                                   staged gather) */
 
 uint32_t xs_abi_version(void);
 
