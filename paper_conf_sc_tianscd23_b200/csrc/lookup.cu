@@ -3306,8 +3306,13 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // entries a 128-lookup task of one material spans per nuclide; for an
   // energy-range shard count is the whole batch's, whose density the shard
   // keeps).  Measured on B200: d < 0.12 (large and small at
-  // 17M) variant 55 = (4, 8, 20, 16, dynamic): large 2.21 ms vs 2.24 static
-  // (40) and 2.47 for k_gather_s3 (25); 0.12 <= d < 0.25 variant 56 = (2, 8, 16,
+  // 17M) variant 59 = variant 55 with 32-entry group buffers (fewer windows
+  // read in place: large gather 1.968 vs 1.980 ms, small 0.723 vs 0.734; 55
+  // when the shared memory does not fit, and for the hash grid, whose
+  // prologue searches read the nuclide grid through L1: large-hash step 2.68
+  // vs 2.58 ms with 59); variant 55 = (4, 8, 20, 16,
+  // dynamic): large 2.21 ms vs 2.24 static (40) and 2.47 for k_gather_s3
+  // (25); 0.12 <= d < 0.25 variant 56 = (2, 8, 16,
   // 24, dynamic): large 8M 1.41 vs 1.42 / 1.48 / 1.61 ms for 44 / 40 / 20;
   // d >= 0.25, N < 100k: k_gather_s3 (2, 2, 8, 24) = variant 20 (large 4M 1.02
   // vs 1.07 ms for 44, small 4M 0.29 vs 0.31); d >= 0.15 on grids of >= 100k
@@ -3319,7 +3324,7 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
     if (d >= 0.15 && g.N >= 100000)
       v = 57;
     else
-      v = d >= 0.25 ? 20 : (d >= 0.12 ? 56 : 55);
+      v = d >= 0.25 ? 20 : (d >= 0.12 ? 56 : (GT == XS_GRID_HASH ? 55 : 59));
   }
   switch (v) {
     case 1: return launch_gather_t<GT, 8, 1, 2, CHECK>(g, P, st);
@@ -3353,6 +3358,11 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
 
     case 50: return launch_gather_s4<GT, 3, 8, 16, 20, CHECK>(g, P, st);
     case 55: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, false, true, true>(g, P, st);
+    case 59: {  // variant 55 with 32-entry group buffers, when the shared memory allows
+      const cudaError_t e = launch_gather_s4<GT, 4, 8, 32, 16, CHECK, false, true, true>(g, P, st);
+      if (e != cudaErrorInvalidConfiguration) return e;
+      return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, false, true, true>(g, P, st);
+    }
     case 56: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK, false, true, true>(g, P, st);
     case 57: return launch_gather_s4<GT, 2, 4, 16, 24, CHECK, false, false, true>(g, P, st);
     case 58: return launch_gather_s4<GT, 2, 2, 12, 24, CHECK>(g, P, st);
@@ -3397,10 +3407,11 @@ static cudaError_t launch_gather_u1(const DeviceGrid& g, const Params& P, bool s
   if constexpr (GT == XS_GRID_UNIONIZED) {
     if (!check && thread_kernel) {
       switch (g.unroll) {
-        case 56: return launch_gather_s4<GT, 2, 8, 16, 24, false, false, true>(g, P, st);
+        case 56: return launch_gather_s4<GT, 2, 8, 16, 24, false, false, true, true>(g, P, st);
         case 20: return launch_gather_s3<GT, 2, 2, 8, 24, false>(g, P, st);
 
-        default: return launch_gather_s4<GT, 4, 8, 20, 16, false, false, true, true>(g, P, st);
+        case 55: return launch_gather_s4<GT, 4, 8, 20, 16, false, false, true, true>(g, P, st);
+        default: return launch_gather_s4<GT, 4, 8, 32, 16, false, false, true, true>(g, P, st);
       }
     }
   }
@@ -3551,7 +3562,7 @@ static cudaError_t run_lookup_t(const DeviceGrid& g, const LookupArgs& a, const 
   P.mat8 = ws.mat8;
   const bool f32 = (a.flags & XS_FLAG_F32) != 0;
   const bool staged = f32 || variant == 0 || (variant >= 17 && variant <= 28) ||
-                      (variant >= 40 && variant <= 50) || (variant >= 55 && variant <= 58);
+                      (variant >= 40 && variant <= 50) || (variant >= 55 && variant <= 59);
   // partitioned A2: the widest coarse key at or below the request whose tile
   // histograms fit the workspace's bin area (a chunk of a host-input batch
   // may allow a wider key than the batch the workspace was sized for)

@@ -762,8 +762,8 @@ xs_status xs_set_param(xs_grid* g, const char* name, int64_t value) {
   if (!std::strcmp(name, "variant")) {
     if (!(value == 0 || (value >= 1 && value <= 4) || (value >= 9 && value <= 12) ||
           (value >= 17 && value <= 28) || (value >= 31 && value <= 36) ||
-          (value >= 40 && value <= 58)))
-      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-58");
+          (value >= 40 && value <= 59)))
+      return fail(XS_ERR_INVALID_ARG, "variant must be 0, 1-4, 9-12, 17-28, 31-36 or 40-59");
     G.unroll = static_cast<int>(value);
   } else if (!std::strcmp(name, "host_chunk")) {
     if (value < 1024) return fail(XS_ERR_INVALID_ARG, "host_chunk >= 1024 lookups");
