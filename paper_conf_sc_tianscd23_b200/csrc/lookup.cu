@@ -3371,8 +3371,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
 }
 
 // fp32 variant (R18): the staged interval-table gather for every batch
-// (variants 31-34 select its shape; any other value the default, 24 warps
-// per block: binary32 accumulators leave room for 80 registers per thread).
+// (variants 31-36 and 46-49 select its shape; any other value the default,
+// k_gather_s4 with 32-entry group buffers and dynamic tasks).
 template <int GT, bool CHECK>
 static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaStream_t st) {
   switch (g.unroll) {
@@ -3385,7 +3385,18 @@ static cudaError_t launch_gather_f32(const DeviceGrid& g, const Params& P, cudaS
     case 47: return launch_gather_s4<GT, 4, 8, 20, 20, CHECK, true>(g, P, st);
     case 48: return launch_gather_s4<GT, 4, 8, 16, 24, CHECK, true>(g, P, st);
 
-    default: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true, false, true>(g, P, st);  // = 46
+    case 46: return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true, false, true>(g, P, st);
+    case 49: return launch_gather_s4<GT, 4, 8, 32, 16, CHECK, true, false, true>(g, P, st);
+    default: {
+      // = 50: 32-entry group buffers, tasks from the global counter (large
+      // gather 1.51 vs 1.54 ms for 46, small 0.594 vs 0.603); 46 for the hash
+      // grid (as in binary64) and when the shared memory does not fit
+      if (GT != XS_GRID_HASH) {
+        const cudaError_t e = launch_gather_s4<GT, 4, 8, 32, 16, CHECK, true, true, true>(g, P, st);
+        if (e != cudaErrorInvalidConfiguration) return e;
+      }
+      return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, true, false, true>(g, P, st);
+    }
   }
 }
 
