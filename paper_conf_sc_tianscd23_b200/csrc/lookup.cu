@@ -3317,7 +3317,8 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
   // d >= 0.25, N < 100k: k_gather_s3 (2, 2, 8, 24) = variant 20 (large 4M 1.02
   // vs 1.07 ms for 44, small 4M 0.29 vs 0.31); d >= 0.15 on grids of >= 100k
   // points per nuclide (XL 170M, cold 9.5 GB interval table): variant 57 =
-  // (2, 4, 16, 24): 32.2 vs 33.5 ms for 20.
+  // (2, 4, 16, 24, dynamic): 32.2 vs 33.5 ms for 20 (static); the dynamic
+  // task order: gather 30.7 vs 31.5 ms, 8-shard rank 4.74 vs 4.89 ms.
   int v = g.unroll;
   if (v == 0) {
     const double d = static_cast<double>(g.N) * 128.0 / static_cast<double>(P.count ? P.count : 1);
@@ -3364,7 +3365,7 @@ static cudaError_t launch_gather_tv(const DeviceGrid& g, const Params& P, cudaSt
       return launch_gather_s4<GT, 4, 8, 20, 16, CHECK, false, true, true>(g, P, st);
     }
     case 56: return launch_gather_s4<GT, 2, 8, 16, 24, CHECK, false, true, true>(g, P, st);
-    case 57: return launch_gather_s4<GT, 2, 4, 16, 24, CHECK, false, false, true>(g, P, st);
+    case 57: return launch_gather_s4<GT, 2, 4, 16, 24, CHECK, false, true, true>(g, P, st);
     case 58: return launch_gather_s4<GT, 2, 2, 12, 24, CHECK>(g, P, st);
     default: return launch_gather_t<GT, 2, 2, 2, CHECK>(g, P, st);
   }
@@ -3422,6 +3423,7 @@ static cudaError_t launch_gather_u1(const DeviceGrid& g, const Params& P, bool s
         case 20: return launch_gather_s3<GT, 2, 2, 8, 24, false>(g, P, st);
 
         case 55: return launch_gather_s4<GT, 4, 8, 20, 16, false, false, true, true>(g, P, st);
+        case 57: return launch_gather_s4<GT, 2, 4, 16, 24, false, false, true, true>(g, P, st);
         default: return launch_gather_s4<GT, 4, 8, 32, 16, false, false, true, true>(g, P, st);
       }
     }
