@@ -3,18 +3,22 @@
 // A8 verify (BASELINE.json north_star).
 //
 // Pipeline of one xs_lookup_batch call (all on the caller's stream):
+//   sorted batches (XS_FLAG_SORT, the default of bench.py): the partitioned
+//   A2 — k_part_count (A1 + per-tile coarse-key histograms; k_part_count_shard
+//   for an energy-range shard), k_part_colscan / k_part_keyscan (scans),
+//   k_part_place (A1 again, coarse-key order), k_part_fine (fine-key order) —
+//   then the staged gather k_gather_s4 (A3 at each task's extremes, A4-A8;
+//   variant table in launch_gather_tv).
+//   unsorted batches:
 //   k_sample    A1 + A3: sample (p, m) from the counter-based stream (or read
-//               the caller's energies), search u (unionized) / bin b (hash)
-//               when needed, write a 16-B LookupRec in batch order, and count
-//               lookups per material (A2 off) or per (material, energy bin)
-//               with the lookup's rank inside its bin (A2 on).
-//   k_scan_*    A2: exclusive scan of the (material, energy bin) histogram.
-//   k_scatter   A2 on: permutation into (material, energy) order; A2 off:
-//               records into their material buckets.
-//   k_gather*   A4-A8 over material buckets (variants below; the default for
-//               energy-sorted batches is k_gather_s3, for unsorted batches
-//               k_gather), verification v = 1 + argmax fused, one atomic pair
-//               per block into vsum.
+//               the caller's energies), search u (unionized) / bin b (hash),
+//               write a 16-B LookupRec in batch order, count lookups per
+//               material;
+//   k_scatter   records into their material buckets;
+//   k_gather_u  A4-A8 (k_gather without the K0u table).
+//   Every gather fuses the verification v = 1 + argmax and adds one atomic
+//   pair per block into vsum.  (k_sample / k_scan_* / k_scatter with binned
+//   counts are the global-atomic A2, kept for comparison: "legacy_sort".)
 #include <cfloat>
 #include <type_traits>
 
