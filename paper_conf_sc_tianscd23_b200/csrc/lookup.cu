@@ -2688,12 +2688,16 @@ constexpr uint32_t kNoBuf = 0xffffffffu;
 #endif
 constexpr bool kS4Prefetch = XS_S4_PREFETCH;
 
+// Indexed by rank: the materials in decreasing nuclide count (stable), so
+// that tasks are numbered longest first (fuel, then 27, 21, ... nuclides)
+// and the dynamic task order ends with the shortest tasks.
 struct alignas(16) GatherSmem4 {
   int32_t num[kMaxMats];
-  uint32_t off[kMaxMats + 1];   // bucket start of material m
+  uint32_t off[kMaxMats + 1];   // bucket start of the material of rank r
   uint32_t cnt[kMaxMats];
-  uint32_t toff[kMaxMats + 1];  // first task of material m
-  uint32_t roff[kMaxMats + 1];  // first table entry of material m (CSR)
+  uint32_t toff[kMaxMats + 1];  // first task of rank r
+  uint32_t roff[kMaxMats + 1];  // first table entry of rank r (CSR, rank order)
+  int32_t mat[kMaxMats];        // material of rank r
 };
 
 // the next task's energies are prefetched (1 KB per warp) by the 4-lookups-
@@ -2728,15 +2732,30 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   const int lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
-    uint32_t run = 0, trun = 0, roff = 0;
-    for (int m = 0; m < P.n_mats; ++m) {
-      const uint32_t c = P.counts[m];
-      G.num[m] = P.num_nucs[m];
+    uint32_t run = 0;
+    for (int m = 0; m < P.n_mats; ++m) {  // bucket starts in material order
       G.off[m] = run;
-      G.cnt[m] = c;
-      G.toff[m] = trun;
-      G.roff[m] = roff;
-      run += c;
+      run += P.counts[m];
+    }
+    for (int m = 0; m < P.n_mats; ++m) {  // rank order: insertion by nuclide count
+      int r = m;
+      while (r > 0 && P.num_nucs[G.mat[r - 1]] < P.num_nucs[m]) {
+        G.mat[r] = G.mat[r - 1];
+        --r;
+      }
+      G.mat[r] = m;
+    }
+    uint32_t start[kMaxMats];
+    for (int m = 0; m < P.n_mats; ++m) start[m] = G.off[m];
+    uint32_t trun = 0, roff = 0;
+    for (int r = 0; r < P.n_mats; ++r) {
+      const int m = G.mat[r];
+      const uint32_t c = P.counts[m];
+      G.num[r] = P.num_nucs[m];
+      G.off[r] = start[m];
+      G.cnt[r] = c;
+      G.toff[r] = trun;
+      G.roff[r] = roff;
       trun += (c + kTask - 1) / kTask;
       roff += static_cast<uint32_t>(P.num_nucs[m]);
     }
@@ -2747,9 +2766,9 @@ __global__ void __launch_bounds__(32 * NW, 1) k_gather_s4(Params P) {
   __syncthreads();
   const int tab = static_cast<int>(G.roff[P.n_mats]);
   for (int i = threadIdx.x; i < tab; i += blockDim.x) {
-    int m = 0;
-    while (static_cast<uint32_t>(i) >= G.roff[m + 1]) ++m;
-    const int src = m * P.max_nucs + (i - static_cast<int>(G.roff[m]));
+    int r = 0;
+    while (static_cast<uint32_t>(i) >= G.roff[r + 1]) ++r;
+    const int src = G.mat[r] * P.max_nucs + (i - static_cast<int>(G.roff[r]));
     const int32_t n = P.mats[src];
     MatEntry me;
     me.conc = P.concs[src];
